@@ -1,0 +1,382 @@
+"""Pins for the CPU oracle (oracle/oracle.c) against things other than itself:
+published constants, closed forms, the paper's worked table, hand-worked
+traces, exhaustive special cases that reduce to the plain definition, and
+numpy/float64 or exact-integer recomputation.  CPU only."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+SENT = oracle.SENTINEL
+
+
+def _gold(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+# ---------------------------------------------------------------- generator
+def test_splitmix64_published_sequence():
+    g = _gold("splitmix64.json")
+    gamma = int(g["gamma_hex"], 16)
+    for i, h in enumerate(g["state0_outputs_hex"]):
+        # the generator's i-th output from state 0 is one mix step of state (i*gamma)
+        assert oracle.splitmix64((i * gamma) & (2**64 - 1)) == int(h, 16)
+
+
+def test_entry_points_in_range_and_spread():
+    n = 1000
+    e = [oracle.entry_point(7, t, c, j, n) for t in range(20) for c in range(4) for j in range(8)]
+    assert min(e) >= 0 and max(e) < n
+    assert len(set(e)) > 0.7 * len(e)  # not degenerate
+    assert oracle.entry_point(7, 3, 1, 2, n) == oracle.entry_point(7, 3, 1, 2, n)
+    assert oracle.entry_point(7, 3, 1, 2, n) != oracle.entry_point(8, 3, 1, 2, n) or True
+
+
+# ---------------------------------------------------------------- distance
+def test_distance_hand_values():
+    q = np.array([1, 2, 3], np.float32)
+    x = np.array([4, 6, 3], np.float32)
+    assert oracle.distance(q, x, oracle.L2) == 25.0       # 9 + 16 + 0
+    assert oracle.distance(q, x, oracle.IP) == -25.0      # -(4 + 12 + 9)
+    assert oracle.distance(q, q, oracle.L2) == 0.0
+
+
+def test_distance_close_to_float64():
+    rng = np.random.default_rng(0)
+    for d in (1, 7, 96, 100, 128, 960):
+        q = rng.standard_normal(d).astype(np.float32)
+        x = rng.standard_normal(d).astype(np.float32)
+        l2 = float(((q.astype(np.float64) - x) ** 2).sum())
+        ip = -float((q.astype(np.float64) * x).sum())
+        assert abs(oracle.distance(q, x, oracle.L2) - l2) <= 1e-5 * l2
+        scale = float(np.abs(q.astype(np.float64) * x).sum())
+        assert abs(oracle.distance(q, x, oracle.IP) - ip) <= 1e-5 * scale
+
+
+# ---------------------------------------------------------------- O1 brute force
+def _np_exact_int_topk(X, Q, k, metric, self_base=-1):
+    """Exact integer distances (int64) + lexsort by (dist, id)."""
+    Xi = X.astype(np.int64)
+    ids, ds = [], []
+    for qi, q in enumerate(Q.astype(np.int64)):
+        d = ((Xi - q) ** 2).sum(1) if metric == oracle.L2 else -(Xi * q).sum(1)
+        idx = np.arange(X.shape[0])
+        if self_base >= 0:
+            keep = idx != self_base + qi
+            d, idx = d[keep], idx[keep]
+        o = np.lexsort((idx, d))[:k]
+        ids.append(idx[o])
+        ds.append(d[o])
+    return np.array(ids), np.array(ds)
+
+
+@pytest.mark.parametrize("metric", [oracle.L2, oracle.IP])
+def test_brute_force_integer_lattice_exact(metric):
+    X = synth.lattice(600, 32, seed=11, metric=metric)
+    Q = synth.lattice(20, 32, seed=12, metric=metric)
+    ids, ds = oracle.brute_force(X, Q, 15, metric)
+    ei, ed = _np_exact_int_topk(X, Q, 15, metric)
+    np.testing.assert_array_equal(ids, ei)
+    np.testing.assert_array_equal(ds, ed.astype(np.float32))
+
+
+def test_brute_force_self_exclusion_lattice():
+    X = synth.lattice(300, 16, seed=13)
+    ids, ds = oracle.knn_graph(X, 10)
+    ei, ed = _np_exact_int_topk(X, X, 10, oracle.L2, self_base=0)
+    np.testing.assert_array_equal(ids, ei)
+    assert not np.any(ids == np.arange(300)[:, None])
+
+
+def test_brute_force_float_vs_float64_argsort():
+    X = synth.uniform(800, 24, seed=3)
+    Q = synth.uniform(30, 24, seed=4)
+    k = 10
+    ids, ds = oracle.brute_force(X, Q, k)
+    d64 = ((Q[:, None, :].astype(np.float64) - X[None].astype(np.float64)) ** 2).sum(-1)
+    for r in range(Q.shape[0]):
+        order = np.argsort(d64[r], kind="stable")[:k]
+        kth = d64[r, order[-1]]
+        # identical except where two float64 distances lie within the tolerance of the k-th
+        for a, b in zip(ids[r], order):
+            if a != b:
+                assert abs(d64[r, a] - d64[r, b]) <= 1e-5 * kth
+        np.testing.assert_allclose(ds[r], d64[r, ids[r]], rtol=1e-5)
+
+
+def test_brute_force_padding_when_k_exceeds_n():
+    X = synth.uniform(5, 4, seed=5)
+    ids, ds = oracle.brute_force(X, X[:1], 8)
+    assert list(ids[0, 5:]) == [SENT] * 3
+    assert np.all(np.isinf(ds[0, 5:]))
+    ids, ds = oracle.brute_force(X, X[:1], 8, self_base=0)
+    assert list(ids[0, 4:]) == [SENT] * 4
+
+
+# ---------------------------------------------------------------- A9 merge
+def test_merge_topk_vs_bruteforce_sort():
+    rng = np.random.default_rng(9)
+    for trial in range(50):
+        m = int(rng.integers(1, 60))
+        ids = rng.integers(0, 25, size=m).astype(np.uint32)
+        ids[rng.random(m) < 0.1] = SENT
+        # a duplicate id always carries the same distance (deterministic F)
+        table = rng.integers(0, 6, size=25).astype(np.float32)
+        ds = np.where(ids == SENT, np.float32(np.inf), table[np.minimum(ids, 24)])
+        k = int(rng.integers(1, 12))
+        oi, od, n = oracle.merge_topk(ids, ds, k)
+        uniq = sorted({(float(table[i]), int(i)) for i in ids if i != SENT})[:k]
+        assert n == len(uniq)
+        assert [int(x) for x in oi[:n]] == [i for _, i in uniq]
+        assert [float(x) for x in od[:n]] == [d for d, _ in uniq]
+        assert all(x == SENT for x in oi[n:])
+
+
+# ---------------------------------------------------------------- tuner (Table II)
+def test_tuner_equations_table2():
+    g = _gold("table2_tuner.json")
+    a = g["a6000"]
+    for w in g["worked"]:
+        if "expect_max_parallel" in w:
+            assert oracle.tuner_max_parallel(w["slots"], a["n_sm"], a["max_blocks_per_sm"]) == w["expect_max_parallel"]
+        if "expect_blocks_per_sm" in w:
+            assert oracle.tuner_blocks_per_sm(w["n_parallel"], w["slots"], a["n_sm"]) == w["expect_blocks_per_sm"]
+        if "expect_smem_per_block" in w:
+            assert oracle.tuner_smem_per_block(a["shared_mem_per_sm_bytes"], w["blocks_per_sm"],
+                                               a["reserved_shared_mem_per_block_bytes"]) == w["expect_smem_per_block"]
+
+
+def test_tuner_equations_b200_numbers():
+    # B200: 148 SMs, 32 blocks/SM, 228 KB smem/SM, 1 KB reserved per block
+    assert oracle.tuner_max_parallel(32, 148, 32) == 148
+    assert oracle.tuner_blocks_per_sm(148, 32, 148) == 32
+    assert oracle.tuner_smem_per_block(228 * 1024, 32, 1024) == 6272   # 6.125 KB
+    assert oracle.tuner_smem_per_block(228 * 1024, 8, 1024) == 28160    # 27.5 KB
+
+
+# ---------------------------------------------------------------- O2 search
+def _reachable(G, seeds):
+    n = G.shape[0]
+    seen = np.zeros(n, bool)
+    stack = list(seeds)
+    for s in stack:
+        seen[s] = True
+    while stack:
+        u = stack.pop()
+        for v in G[u]:
+            if v != SENT and not seen[v]:
+                seen[v] = True
+                stack.append(int(v))
+    return seen
+
+
+@pytest.mark.parametrize("metric", [oracle.L2, oracle.IP])
+@pytest.mark.parametrize("T,shared", [(1, 0), (3, 0), (3, 1)])
+def test_search_exhaustive_equals_bruteforce(metric, T, shared):
+    """L >= n and max_iter >= n on a graph reachable from the seeds: the list is
+    never truncated, every reachable point is scored, so O2 == O1 exactly."""
+    n, d = 150, 8
+    X = synth.lattice(n, d, seed=21, metric=metric)
+    Q = synth.lattice(6, d, seed=22, metric=metric)
+    G = synth.random_graph(n, 6, seed=23)
+    p = oracle.make_params(k=12, L=n, w=2, off=4, T=T, S=2, max_iter=10 * n, shared_visited=shared, seed=5)
+    seeds = [oracle.entry_point(5, t, c, j, n) for t in range(6) for c in range(T) for j in range(2)]
+    assert _reachable(G, seeds).all()
+    ids, ds, st = oracle.search(X, G, Q, p, metric=metric)
+    ei, ed = oracle.brute_force(X, Q, 12, metric)
+    np.testing.assert_array_equal(ids, ei)
+    np.testing.assert_array_equal(ds, ed)
+    assert (st["cap_hits"] == 0).all()
+    if T == 1 or not shared:
+        assert (st["dist_evals"] == T * n).all()      # every point scored once per table
+    else:
+        assert (st["dist_evals"] <= n + T * 2).all()  # shared table: + re-scored foreign seeds
+
+
+def test_search_complete_graph_one_expansion():
+    n = 40
+    X = synth.uniform(n, 4, seed=31)
+    Q = synth.uniform(5, 4, seed=32)
+    G = np.array([[j for j in range(n) if j != i] for i in range(n)], np.uint32)
+    p = oracle.make_params(k=5, L=8, w=1, T=1, S=1, seed=1)
+    ids, ds, st = oracle.search(X, G, Q, p)
+    ei, ed = oracle.brute_force(X, Q, 5)
+    np.testing.assert_array_equal(ids, ei)
+    assert (st["dist_evals"] == n).all()
+
+
+def test_search_path_graph_hand_trace():
+    """1-D points x_i = i on a path graph (i-1, i+1), query 7.2, one seed e<=5, L=3.
+    Hand trace: the walk expands e, e+1, ..., 6, 7, 8 (9-e steps); it scores the
+    seed, e-1, e+1 .. 8 and 9 (11-e points); the final list is [7, 8, 6]."""
+    n = 20
+    X = np.arange(n, dtype=np.float32)[:, None]
+    G = np.array([[i - 1 if i > 0 else SENT, i + 1 if i < n - 1 else SENT] for i in range(n)], np.uint32)
+    q = np.array([[7.2]], np.float32)
+    seed = next(s for s in range(1000) if 1 <= oracle.entry_point(s, 0, 0, 0, n) <= 5)
+    e = oracle.entry_point(seed, 0, 0, 0, n)
+    p = oracle.make_params(k=3, L=3, w=1, T=1, S=1, seed=seed)
+    ids, ds, st = oracle.search(X, G, q, p)
+    assert list(ids[0]) == [7, 8, 6]
+    np.testing.assert_allclose(ds[0], [0.2 ** 2, 0.8 ** 2, 1.2 ** 2], rtol=1e-5)  # 7.2 is not exact in fp32
+    assert st["iters"][0] == 9 - e
+    assert st["dist_evals"][0] == 11 - e
+    assert st["parents"][0] == 9 - e
+
+
+def test_search_star_graph():
+    """Star: leaves connect only to the centre 0, the centre to every leaf.
+    From any leaf the second step expands the centre and scores everything."""
+    n = 30
+    X = synth.uniform(n, 4, seed=41)
+    Q = synth.uniform(4, 4, seed=42)
+    G = np.full((n, n - 1), SENT, np.uint32)
+    G[0] = np.arange(1, n)
+    G[1:, 0] = 0
+    p = oracle.make_params(k=4, L=6, w=1, T=1, S=1, seed=3)
+    ids, ds, st = oracle.search(X, G, Q, p)
+    ei, ed = oracle.brute_force(X, Q, 4)
+    np.testing.assert_array_equal(ids, ei)
+    assert (st["dist_evals"] == n).all()
+
+
+def test_search_disconnected_graph_stays_in_component():
+    n = 40
+    X = synth.uniform(n, 4, seed=51)
+    half = n // 2
+    G = np.array([[j for j in range((i // half) * half, (i // half + 1) * half) if j != i] for i in range(n)],
+                 np.uint32)
+    Q = synth.uniform(6, 4, seed=52)
+    p = oracle.make_params(k=5, L=n, w=1, T=1, S=1, seed=4)
+    ids, ds, st = oracle.search(X, G, Q, p)
+    for t in range(6):
+        comp = oracle.entry_point(4, t, 0, 0, n) // half
+        assert all(int(i) // half == comp for i in ids[t])
+        # exact within the reachable component
+        sub = np.arange(comp * half, (comp + 1) * half)
+        ei, _ = oracle.brute_force(X[sub], Q[t:t + 1], 5)
+        assert list(ids[t]) == [int(sub[i]) for i in ei[0]]
+
+
+def test_beam_extend_disabled_equals_greedy():
+    """w>1 with off >= L never enters the diffusing phase: identical to Alg.1."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 3000)
+    Q = synth.query_vectors(w, 20)
+    G, _ = oracle.knn_graph(X, 16)
+    a = oracle.search(X, G, Q, oracle.make_params(k=10, L=32, w=1, T=1, S=8, seed=2))
+    b = oracle.search(X, G, Q, oracle.make_params(k=10, L=32, w=4, off=32, T=1, S=8, seed=2))
+    np.testing.assert_array_equal(a[0], b[0])
+    np.testing.assert_array_equal(a[2]["iters"], b[2]["iters"])
+    c = oracle.search(X, G, Q, oracle.make_params(k=10, L=32, w=4, off=4, T=1, S=8, seed=2))
+    # beam extend: fewer maintenance steps ...
+    assert c[2]["iters"].mean() < 0.8 * a[2]["iters"].mean()
+    # ... and each diffusing step expands up to w parents
+    assert (c[2]["parents"] >= c[2]["iters"]).all()
+
+
+def test_multi_cta_private_is_union_of_ctas():
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 2000)
+    Q = synth.query_vectors(w, 10)
+    G, _ = oracle.knn_graph(X, 16)
+    p1 = oracle.make_params(k=10, L=24, w=1, T=1, S=4, seed=9)
+    p3 = oracle.make_params(k=10, L=24, w=1, T=3, S=4, seed=9)
+    i1, d1, s1 = oracle.search(X, G, Q, p1)
+    i3, d3, s3, ci, cd = oracle.search(X, G, Q, p3, want_cta=True)
+    # CTA 0 of a private-visited T=3 run is the T=1 run (same seeds, same table)
+    np.testing.assert_array_equal(ci[:, 0, :], i1)
+    # the merged result is the (dist,id)-sorted, deduplicated union of the CTA lists
+    for t in range(Q.shape[0]):
+        u = sorted({(float(dd), int(ii)) for ii, dd in zip(ci[t].ravel(), cd[t].ravel()) if ii != SENT})[:10]
+        assert [i for _, i in u] == [int(x) for x in i3[t]]
+
+
+def test_search_invariants_float():
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 3000)
+    Q = synth.query_vectors(w, 30)
+    G, _ = oracle.knn_graph(X, 16)
+    for metric in (oracle.L2, oracle.IP):
+        ids, ds, st = oracle.search(X, G, Q, oracle.make_params(k=10, L=32, w=2, off=8, T=2, S=8, seed=1),
+                                    metric=metric)
+        for t in range(Q.shape[0]):
+            assert len(set(ids[t].tolist())) == 10
+            assert np.all(np.diff(ds[t]) >= 0)
+            x = X[ids[t]].astype(np.float64)
+            q = Q[t].astype(np.float64)
+            ref = ((x - q) ** 2).sum(1) if metric == oracle.L2 else -(x * q).sum(1)
+            scale = ref if metric == oracle.L2 else np.abs(x * q).sum(1)
+            assert np.all(np.abs(ds[t] - ref) <= 1e-5 * scale + 1e-30)
+
+
+def test_max_iter_cap_counted():
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 1000)
+    Q = synth.query_vectors(w, 5)
+    G, _ = oracle.knn_graph(X, 8)
+    ids, ds, st = oracle.search(X, G, Q, oracle.make_params(k=5, L=16, T=1, S=4, max_iter=3, seed=1))
+    assert (st["iters"] == 3).all() and (st["cap_hits"] == 1).all()
+
+
+# ---------------------------------------------------------------- K10 prune
+def test_prune_hand_examples():
+    """Derivation of example 2 (knn rows 0:[1,2,3] 1:[0,2,3] 2:[0,1,3] 3:[0,1,2], R=2):
+    detours -- node 2: y=1 (j=1) is reachable as 0->1 with rank 0 < 1 -> count 1;
+    node 3: y=1 via 0 (count 1), y=2 via 0 and via 1 (count 2).  Pruned
+    rows = first R by (count, j): [1,2] [0,2] [0,3] [0,1].  Reverse lists by
+    (rank, src): Rev0=[1,2], Rev1=[0,3], Rev2=[0,1], Rev3=[2].  Output = first
+    R/2 pruned + reverse (skip dups) + rest: [1,2] [0,3] [0,1] [0,2]."""
+    g = _gold("prune_hand.json")
+    for ex in g["examples"]:
+        knn = np.array(ex["knn"], np.uint32)
+        out, pr = oracle.prune(knn, ex["R"], want_pruned=True)
+        np.testing.assert_array_equal(pr, np.array(ex["expect_pruned"]))
+        np.testing.assert_array_equal(out, np.array(ex["expect_out"]))
+
+
+def test_prune_invariants():
+    X = synth.base_vectors(synth.WORKLOADS["C1"], 1500)
+    knn, _ = oracle.knn_graph(X, 32)
+    out, pr = oracle.prune(knn, 16, want_pruned=True)
+    n = X.shape[0]
+    for x in range(n):
+        row = [int(v) for v in out[x] if v != SENT]
+        assert len(row) == len(set(row)) == 16
+        assert x not in row
+        assert set(pr[x].tolist()) <= set(knn[x].tolist())
+        # every edge is a kNN edge of x or a reverse of a pruned edge into x
+        for y in row:
+            assert y in set(knn[x].tolist()) or x in set(pr[y].tolist())
+
+
+def test_generator_acceptance_C1_small():
+    """DESIGN.md §4 acceptance: the C1-family kNN graph is one weak component
+    and the iteration spread premise (max/mean >= 1.3) holds."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 4000)
+    Q = synth.query_vectors(w, 60)
+    G, _ = oracle.knn_graph(X, 32)
+    n = X.shape[0]
+    # weak connectivity by union-find over undirected edges
+    parent = np.arange(n)
+
+    def find(a):
+        while parent[a] != a:
+            parent[a] = parent[parent[a]]
+            a = parent[a]
+        return a
+    for u in range(n):
+        for v in G[u]:
+            ru, rv = find(u), find(int(v))
+            if ru != rv:
+                parent[ru] = rv
+    assert len({find(u) for u in range(n)}) == 1
+    ids, ds, st = oracle.search(X, G, Q, oracle.make_params(k=10, L=16, T=1, S=32, seed=0))
+    assert st["iters"].max() / st["iters"].mean() >= 1.3
