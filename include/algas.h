@@ -1,0 +1,282 @@
+/*
+ * algas.h -- C-ABI of the B200-native ALGAS search library (libalgas.so).
+ *
+ * ALGAS: Chen et al., "ALGAS: A Low-latency GPU-Based Approximate Nearest
+ * Neighbor Search System", IPDPS 2025.  Citations "P:L<n>" point into the
+ * paper text; "R<n>" are the readings listed in
+ * DESIGN.md §3 where the paper is silent or ambiguous.
+ *
+ * Problem: given base vectors P (n x dim) and a query q, return the
+ * k points of P closest to q under F(a,b).  Search runs greedy/beam search
+ * over a fixed-out-degree proximity graph (Alg.1, beam extend
+ * P:L200/P:L249), possibly with several CTAs per query,
+ * each CTA publishing its own top-k and the host merging them.
+ *
+ * Conventions for every entry point:
+ *  - Distances are "internal" distances, ascending = closer:
+ *      ALGAS_L2: squared Euclidean  sum_j (q_j - x_j)^2         (R2)
+ *      ALGAS_IP: negated inner product  -sum_j q_j x_j           (R3)
+ *  - Ties are broken by point id: order is lexicographic (dist, id) (R4).
+ *  - Results are sorted ascending, ids unique, padded with
+ *    (ALGAS_SENTINEL, +inf) when fewer than k points were reached (R12).
+ *  - Pointers: every array argument may be HOST or DEVICE memory of the
+ *    current CUDA device unless stated otherwise; the library detects which
+ *    (cudaPointerGetAttributes) and copies as needed.  All arrays are
+ *    caller-owned; the library never frees or retains caller memory beyond
+ *    the call (except where a function says it copies).
+ *  - Return codes: ALGAS_OK (0) or a negative ALGAS_E* code; the message for
+ *    the last failing call on this thread is in algas_last_error().
+ *  - A CUDA failure is reported as ALGAS_ECUDA, never silently retried and
+ *    never answered on the CPU: the library has no CPU fallback.
+ */
+#ifndef ALGAS_H
+#define ALGAS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+#if defined(__GNUC__)
+#pragma GCC visibility push(default) /* the C-ABI is the only exported surface */
+#endif
+
+#define ALGAS_SENTINEL 0xFFFFFFFFu
+#define ALGAS_MAX_ITOPK 512   /* max candidate-list length L            */
+#define ALGAS_MAX_DEGREE 128  /* max graph out-degree R                 */
+#define ALGAS_MAX_DIM 2048    /* max dim (must also be a multiple of 4) */
+#define ALGAS_MAX_WIDTH 32    /* max parents per beam-extend step       */
+#define ALGAS_MAX_CTAS 64     /* max CTAs per query (N_parallel)        */
+#define ALGAS_MAX_SEEDS 256   /* max random entry points per CTA        */
+
+enum algas_metric { ALGAS_L2 = 0, ALGAS_IP = 1 };
+
+enum algas_status {
+    ALGAS_OK = 0,
+    ALGAS_EINVAL = -1,   /* bad argument (see each function)               */
+    ALGAS_ENOMEM = -2,   /* device or pinned host allocation failed        */
+    ALGAS_ECUDA = -3,    /* a CUDA call or kernel failed                   */
+    ALGAS_EAGAIN = -4,   /* persistent path: no EMPTY slot right now       */
+    ALGAS_ESTATE = -5,   /* object in the wrong state (e.g. server closed) */
+    ALGAS_ENCCL = -6,    /* reserved for the sharded multi-GPU path        */
+    ALGAS_EOVERFLOW = -7 /* a visited table overflowed (result still valid,
+                            exploration was cut short; see stats)          */
+};
+
+/* Visited-table sharing between the CTAs of one query ("sharing the
+ * visited table").  PRIVATE: one exact table per CTA -- deterministic, the
+ * parity mode (R9).  SHARED: one table per query, shared by its CTAs (the
+ * paper's design; nondeterministic which CTA scores a point). */
+enum algas_visited { ALGAS_VISITED_PRIVATE = 0, ALGAS_VISITED_SHARED = 1 };
+
+/* Search parameters.  Field meaning follows P:L213 (TopK, candidate list of
+ * max length L, T CTAs) and P:L249 (offset_beam).  Zero / negative values
+ * select the documented default.  Fill with algas_params_default(). */
+typedef struct algas_params {
+    int32_t k;               /* results per query, 1 <= k <= itopk                    */
+    int32_t itopk;           /* L: candidate-list length, k <= L <= ALGAS_MAX_ITOPK   */
+    int32_t width;           /* w: parents per step once diffusing, 1..32   */
+    int32_t offset_beam;     /* off: diffusing starts when the first
+                                unchecked position >= off; < 0 -> itopk/4;
+                                >= itopk disables beam extend (pure Alg.1)           */
+    int32_t ctas_per_query;  /* T = N_parallel; 0 -> adaptive tuner */
+    int32_t threads_per_cta; /* 32/64/128/256; 0 -> tuner                            */
+    int32_t n_seeds;         /* S random entry points per CTA; 0 -> 32      */
+    int32_t max_iter;        /* per-CTA step cap (R8); 0 -> 4*itopk + 256            */
+    int32_t visited_mode;    /* enum algas_visited                                  */
+    int32_t slots;           /* persistent path: B query slots; 0 -> 32     */
+    int32_t hash_bits;       /* log2 of the per-CTA shared-memory visited hash; 0 -> tuner */
+    int32_t reserved0;
+    uint64_t seed;           /* entry-point generator seed (R5)                      */
+} algas_params;
+
+/* Per-query counters (summed over the query's CTAs unless noted). */
+typedef struct algas_query_stats {
+    uint32_t iters;       /* steps = candidate-list maintenance operations */
+    uint32_t max_iters;   /* max steps over the query's CTAs                       */
+    uint32_t parents;     /* expanded candidate points                             */
+    uint32_t dist_evals;  /* distance computations (vectors gathered)              */
+    uint32_t cap_hits;    /* CTAs stopped by max_iter rather than Finish            */
+    uint32_t spills;      /* CTAs whose shared-memory visited hash spilled to HBM   */
+    uint32_t overflows;   /* CTAs whose visited table overflowed (should be 0)      */
+    uint32_t ctas;        /* T used                                                 */
+    uint64_t t_start_ns;  /* device globaltimer at pickup (persistent/dynamic path) */
+    uint64_t t_end_ns;    /* device globaltimer when the last CTA published         */
+    uint64_t latency_ns;  /* host: submit -> merged result ready (server path)      */
+} algas_query_stats;
+
+/* Optional per-call timing filled by the search entry points. */
+typedef struct algas_run_info {
+    float kernel_ms;          /* search kernel duration (CUDA events on the launch stream) */
+    int32_t grid;             /* CTAs launched                                             */
+    int32_t threads_per_cta;
+    int32_t ctas_per_query;
+    int32_t smem_per_cta;     /* dynamic shared memory bytes                               */
+    int32_t blocks_per_sm;    /* occupancy of the search kernel                            */
+    int32_t hash_bits;
+    int32_t reserved;
+} algas_run_info;
+
+typedef struct algas_index algas_index;   /* opaque; immutable after create */
+typedef struct algas_server algas_server; /* opaque; owns ring + persistent kernel */
+
+/* Fill *p with defaults: k=10, itopk=64, width=1, offset_beam=-1, T=1,
+ * threads=0, n_seeds=32, max_iter=0, PRIVATE, slots=32, seed=0. */
+void algas_params_default(algas_params *p);
+
+/* Thread-local description of the last error (never NULL). */
+const char *algas_last_error(void);
+
+/* Library version string. */
+const char *algas_version(void);
+
+/* ------------------------------------------------------------------ */
+/* Index (graph index G=(V,E) over the vectors of P).            */
+/* ------------------------------------------------------------------ */
+/* Creates an index on the current CUDA device.  The library COPIES data
+ * (n x dim fp32, row-major) and graph (n x degree u32, row-major, entries
+ * in [0,n) or ALGAS_SENTINEL) into HBM; the caller keeps ownership.
+ * graph == NULL builds the graph: exact kNN with 2*degree neighbours
+ * (algas_knn) followed by CAGRA-style pruning to `degree` (algas_prune).
+ * EINVAL (returns NULL): n < 1 or n >= 2^31, dim < 4, dim % 4 != 0,
+ * dim > ALGAS_MAX_DIM, degree < 1 or > ALGAS_MAX_DEGREE, bad metric. */
+algas_index *algas_index_create(const float *data, int64_t n, int32_t dim, int32_t metric,
+                                const uint32_t *graph, int32_t degree);
+int algas_index_destroy(algas_index *idx);
+/* Shape query; any out pointer may be NULL.  *dev_data / *dev_graph are
+ * device pointers owned by the index (graph row stride = *graph_stride). */
+int algas_index_info(const algas_index *idx, int64_t *n, int32_t *dim, int32_t *metric,
+                     int32_t *degree, int32_t *graph_stride, const float **dev_data,
+                     const uint32_t **dev_graph);
+
+/* ------------------------------------------------------------------ */
+/* Static (batch) search: one launch over nq queries (P:L107 batch       */
+/* processing; the search procedure of P:L213-223).                      */
+/* ------------------------------------------------------------------ */
+/* queries: nq x dim fp32.  out_ids / out_dists: nq x k.  Uses
+ * algas_params_default() with the given k, itopk, width. */
+int algas_search(const algas_index *idx, const float *queries, int64_t nq, int32_t k,
+                 int32_t itopk, int32_t width, uint32_t *out_ids, float *out_dists);
+
+/* Full-control batch search.  Query i uses tag = tag0 + i (R23), so a batch
+ * result is reproducible through algas_submit with the same tag.
+ * out_cta_ids / out_cta_dists (nullable): nq x T x k per-CTA results before
+ * the host merge.  out_stats (nullable): nq entries.
+ * stream: cudaStream_t to run on (NULL = the legacy default stream); the
+ * call is synchronous with respect to the host.  info (nullable): kernel
+ * time and launch shape.
+ * Returns EOVERFLOW (results still written) if any visited table overflowed. */
+int algas_search_ex(const algas_index *idx, const float *queries, int64_t nq,
+                    const algas_params *params, uint64_t tag0, uint32_t *out_ids,
+                    float *out_dists, uint32_t *out_cta_ids, float *out_cta_dists,
+                    algas_query_stats *out_stats, void *stream, algas_run_info *info);
+
+/* Dynamic batching from an HBM-resident query queue: a
+ * persistent kernel keeps exactly params->slots queries in flight; a slot
+ * takes the next query the moment its CTAs finish (no batch barrier).
+ * queries must be DEVICE memory (nq x dim); outputs may be host or device.
+ * Per-query stats carry device start/end timestamps (globaltimer). */
+int algas_search_dynamic(const algas_index *idx, const float *queries_dev, int64_t nq,
+                         const algas_params *params, uint64_t tag0, uint32_t *out_ids,
+                         float *out_dists, algas_query_stats *out_stats, void *stream,
+                         algas_run_info *info);
+
+/* ------------------------------------------------------------------ */
+/* Persistent server: host-mapped slot ring + persistent kernel          */
+/* (P:L157-178), host TopK merge.                           */
+/* ------------------------------------------------------------------ */
+/* Launches the persistent kernel (cooperative launch: all slots x T CTAs
+ * co-resident).  params->k / itopk are the per-server maxima; a
+ * submit may ask for smaller k/itopk/width.  *out is NULL on failure. */
+int algas_server_create(const algas_index *idx, const algas_params *params, algas_server **out);
+/* Non-blocking.  query: dim fp32 in HOST memory.  Claims an EMPTY slot
+ * (EMPTY -> READY); ALGAS_EAGAIN if every slot is busy.
+ * k <= server k, itopk <= server itopk, width <= 32 (0 -> server value). */
+int algas_submit(algas_server *s, const float *query, uint64_t tag, int32_t k, int32_t itopk,
+                 int32_t width);
+/* Non-blocking.  Moves up to max_results completed queries into caller
+ * HOST buffers: tags[i], ids[i*kmax .. ), dists[i*kmax .. ) where kmax is
+ * the server's k (rows padded with SENTINEL / +inf), stats[i] (nullable).
+ * *n_out = number returned. */
+int algas_poll(algas_server *s, uint64_t *tags, uint32_t *ids, float *dists,
+               algas_query_stats *stats, int32_t max_results, int32_t *n_out);
+/* Number of submitted-but-not-yet-polled queries. */
+int algas_server_inflight(const algas_server *s, int64_t *n);
+/* Sets QUIT, joins the kernel and the poller, frees the ring. */
+int algas_server_destroy(algas_server *s);
+
+/* ------------------------------------------------------------------ */
+/* Host TopK merge & filter, exposed for tests and shard mode.  */
+/* ------------------------------------------------------------------ */
+/* Merges m (id, dist) HOST entries by (dist, id), drops SENTINEL and
+ * repeated ids (keeps the smallest key, R11), writes k (padded).  Returns
+ * the number of real entries written. */
+int32_t algas_merge_topk(const uint32_t *ids, const float *dists, int32_t m, int32_t k,
+                         uint32_t *out_ids, float *out_dists);
+
+/* ------------------------------------------------------------------ */
+/* Adaptive tuning.                                        */
+/* ------------------------------------------------------------------ */
+typedef struct algas_device_props {
+    int32_t n_sm;                 /* N_SM                         */
+    int32_t max_blocks_per_sm;    /* N_max_block_per_SM           */
+    int64_t smem_per_sm;          /* M_per_SM (bytes)             */
+    int64_t smem_reserved_per_block; /* driver reservation (bytes) */
+    int64_t smem_per_block_optin; /* largest dynamic smem per CTA */
+    int32_t max_threads_per_sm;
+    int32_t regs_per_sm;
+} algas_device_props;
+
+typedef struct algas_tuning {
+    int32_t ctas_per_query;   /* N_parallel                 */
+    int32_t blocks_per_sm;    /* N_block_per_SM             */
+    int64_t smem_avail_per_block; /* M_avail_per_block bound */
+    int64_t smem_per_block;   /* bytes the search kernel will use    */
+    int32_t threads_per_cta;
+    int32_t width;
+    int32_t offset_beam;
+    int32_t hash_bits;
+} algas_tuning;
+
+/* Properties of the current device (props of P:L280-291 Table II). */
+int algas_device_query(algas_device_props *out);
+/* The three printed equations, exactly (align() = ceil, R13). */
+int32_t algas_tuner_max_parallel(int32_t slots, int32_t n_sm, int32_t max_blocks_per_sm);
+int32_t algas_tuner_blocks_per_sm(int32_t n_parallel, int32_t slots, int32_t n_sm);
+int64_t algas_tuner_smem_per_block(int64_t smem_per_sm, int32_t blocks_per_sm,
+                                   int64_t smem_reserved_per_block);
+/* Full tuner: picks T, threads/CTA, width, offset_beam and the visited hash
+ * size for `slots` concurrent queries of this shape so that every slot's
+ * CTAs are co-resident and the per-block shared memory respects
+ * P:L245 with M_reserved sized for the dimension.
+ * props NULL -> algas_device_query().  Returns EINVAL if no configuration fits. */
+int algas_tune(const algas_device_props *props, int32_t slots, int32_t dim, int32_t degree,
+               int32_t itopk, int32_t k, algas_tuning *out);
+
+/* ------------------------------------------------------------------ */
+/* Graph construction (supporting code, not the search hot path):        */
+/* exact kNN + CAGRA-style pruning (graph named P:L293; ref [25] P:L430). */
+/* ------------------------------------------------------------------ */
+/* Exact k nearest base points of every query, fp32 distances,
+ * (dist,id) order.  self_base >= 0 excludes base id (self_base + i) from
+ * query i's answer (kNN graph of the base set: queries = base, self_base=0).
+ * k <= 1024.  out_ids/out_dists: nq x k. */
+int algas_knn(const float *base, int64_t n, const float *queries, int64_t nq, int32_t dim,
+              int32_t metric, int32_t k, int64_t self_base, uint32_t *out_ids, float *out_dists);
+/* CAGRA-style reading R24: rank-based detour count, keep `degree` edges,
+ * add reverse edges, merge.  knn: n x knn_degree (sorted rows, no self).
+ * out_graph: n x degree. */
+int algas_prune(const uint32_t *knn, int64_t n, int32_t knn_degree, int32_t degree,
+                uint32_t *out_graph);
+/* algas_knn(self) with knn_degree neighbours, then algas_prune if prune != 0
+ * (else the first `degree` kNN columns).  out_graph: n x degree. */
+int algas_build_graph(const float *data, int64_t n, int32_t dim, int32_t metric,
+                      int32_t knn_degree, int32_t degree, int32_t prune, uint32_t *out_graph);
+
+#if defined(__GNUC__)
+#pragma GCC visibility pop
+#endif
+#ifdef __cplusplus
+}
+#endif
+#endif /* ALGAS_H */

@@ -1,0 +1,136 @@
+// internal.h -- declarations shared by the translation units of libalgas.so.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdarg>
+#include <cstdint>
+#include <mutex>
+#include <string>
+
+#include "../../include/algas.h"
+#include "search_core.cuh"
+
+namespace algas {
+
+// ------------------------------------------------------------------ errors
+int set_error(int code, const char* fmt, ...);
+#define ALGAS_CUDA_TRY(expr)                                                                     \
+  do {                                                                                           \
+    cudaError_t _e = (expr);                                                                     \
+    if (_e != cudaSuccess)                                                                       \
+      return ::algas::set_error(ALGAS_ECUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(_e), \
+                                __FILE__, __LINE__);                                             \
+  } while (0)
+
+bool is_device_ptr(const void* p);
+
+// ------------------------------------------------------------------ index
+struct Workspace {
+  std::mutex mu;
+  unsigned long long* gtab = nullptr;  // epoch-tagged spill tables
+  size_t gtab_entries = 0;
+  int* counters = nullptr;             // small device scratch (work counters ...)
+  uint32_t epoch = 1;                  // next epoch for the spill tables
+};
+
+}  // namespace algas
+
+struct algas_index {
+  int device = 0;
+  int64_t n = 0;
+  int32_t dim = 0, d4 = 0, metric = 0, degree = 0, rp4 = 0;
+  float* d_data = nullptr;      // n x dim
+  uint32_t* d_graph = nullptr;  // n x (4*rp4), sentinel padded
+  algas::Workspace* ws = nullptr;
+};
+
+namespace algas {
+
+// ------------------------------------------------------------------ launch plumbing
+// Resolved launch configuration for one search call.
+struct Plan {
+  int nt;          // threads per CTA
+  int ccfg;        // chunk config (TL, CPL) index
+  int T;           // CTAs per query
+  int smem;        // dynamic shared memory bytes
+  int blocks_per_sm;
+  SearchCfg cfg;   // L/w/off/S/max_iter/hash filled
+  int k;
+  int visited_mode;
+  int metric;
+};
+
+int chunk_config_for(int d4);          // -1 if unsupported
+int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent);
+
+// spill tables: ensure >= entries, returns base pointer (workspace locked by caller)
+int ensure_gtab(algas_index* idx, size_t entries);
+
+// kernel launchers (search_kernels.cu)
+struct BatchLaunch {
+  const float4* queries;
+  int64_t nq;
+  uint64_t tag0;
+  ResultEntry* res;       // nq x T x k (device)
+  CtaStats* stats;        // nq x T (device, nullable)
+  unsigned long long* gtab;
+  uint32_t epoch_base;
+  int* work_counter;      // device int, zeroed by the launcher
+  int grid;
+};
+int launch_batch(const Plan& pl, const BatchLaunch& bl, cudaStream_t st);
+
+// persistent kernel arguments (ring and device-queue feeds)
+struct alignas(64) RingSlot {
+  volatile uint32_t state;  // host-written: (epoch << 8) | {0 EMPTY, 1 READY, 2 QUIT}
+  int32_t k, L, w;
+  uint64_t tag;
+  uint32_t pad[10];
+};
+enum { kSlotEmpty = 0, kSlotReady = 1, kSlotQuit = 2 };
+
+struct PersistArgs {
+  int mode;                 // 0 ring, 1 device queue
+  int slots, T, kmax;
+  // device queue
+  const float4* queries;
+  int64_t nq;
+  uint64_t tag0;
+  int* queue_head;
+  ResultEntry* dq_res;      // nq x T x kmax
+  CtaStats* dq_stats;       // nq x T
+  // host ring (mapped pointers)
+  RingSlot* ring;
+  const float4* ring_q;     // slots x d4
+  ResultEntry* ring_res;    // slots x T x kmax
+  CtaStats* ring_stats;     // slots x T
+  uint32_t* ring_done;      // slots x T
+  // device mailbox
+  unsigned long long* mbox; // slots
+  float4* qbuf;             // slots x d4
+  int4* dparams;            // slots: {k, L, w, 0}
+  unsigned long long* dtag; // slots
+  unsigned int* slot_fin;   // slots
+  unsigned long long* gtab;
+  uint32_t epoch_base;
+};
+int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st);
+
+// device control block of a persistent launch: queue head | dparams (16-B) |
+// mbox | dtag | slot_fin, every array naturally aligned
+inline size_t control_bytes(int slots) { return 256 + (size_t)slots * (16 + 8 + 8 + 4) + 64; }
+inline void carve_control(uint8_t* cb, int slots, PersistArgs* pa) {
+  pa->queue_head = reinterpret_cast<int*>(cb);
+  pa->dparams = reinterpret_cast<int4*>(cb + 256);
+  pa->mbox = reinterpret_cast<unsigned long long*>(cb + 256 + (size_t)slots * 16);
+  pa->dtag = reinterpret_cast<unsigned long long*>(cb + 256 + (size_t)slots * 24);
+  pa->slot_fin = reinterpret_cast<unsigned int*>(cb + 256 + (size_t)slots * 32);
+}
+int max_blocks_per_sm(const Plan& pl, bool persistent, int* out);
+
+// host TopK merge (runtime.cpp)
+int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t* out_ids, float* out_d);
+
+}  // namespace algas

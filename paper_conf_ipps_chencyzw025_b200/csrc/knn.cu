@@ -1,0 +1,420 @@
+// knn.cu -- graph construction (supporting code, not the search hot path).
+//
+//  algas_knn   : exact k-NN by brute force.  Distances are computed
+//                in the DIRECT form sum_j (q_j - x_j)^2 / -sum_j q_j x_j in
+//                fp32 (no |q|^2+|x|^2-2q.x cancellation, so the result is
+//                exact up to fp32 summation order and bit-exact on the
+//                integer lattice), tile by tile into an HBM distance block,
+//                then a warp-per-row running top-k selection keyed by
+//                (dist, id) (R4).
+//  algas_prune : CAGRA-style optimisation of the kNN graph, reading R24
+//                (rank-based detour count, keep `degree`, reverse edges,
+//                merge).  The graph type is named at P:L293; the algorithm
+//                is CAGRA's (ref [25]) and not printed in the paper.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "internal.h"
+
+namespace algas {
+
+// ------------------------------------------------------------------ distance tiles
+constexpr int TQ = 128, TX = 128, TK = 16;
+
+template <int METRIC>
+__global__ void __launch_bounds__(256) dist_tile_kernel(const float* __restrict__ Q, int64_t qn,
+                                                        const float* __restrict__ X, int64_t xn, int d,
+                                                        float* __restrict__ D, int64_t ldD) {
+  __shared__ float Qs[TK][TQ + 4];
+  __shared__ float Xs[TK][TX + 4];
+  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+  const int64_t q0 = (int64_t)blockIdx.y * TQ, x0 = (int64_t)blockIdx.x * TX;
+  float acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+  for (int k0 = 0; k0 < d; k0 += TK) {
+    // 128 rows x 16 dims = 512 float4 per operand; 256 threads x 2
+    for (int t = threadIdx.x; t < TQ * TK / 4; t += 256) {
+      const int r = t >> 2, c4 = (t & 3) * 4;
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (q0 + r < qn && k0 + c4 < d) v = *reinterpret_cast<const float4*>(Q + (q0 + r) * d + k0 + c4);
+      Qs[c4 + 0][r] = v.x; Qs[c4 + 1][r] = v.y; Qs[c4 + 2][r] = v.z; Qs[c4 + 3][r] = v.w;
+      float4 u = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (x0 + r < xn && k0 + c4 < d) u = *reinterpret_cast<const float4*>(X + (x0 + r) * d + k0 + c4);
+      Xs[c4 + 0][r] = u.x; Xs[c4 + 1][r] = u.y; Xs[c4 + 2][r] = u.z; Xs[c4 + 3][r] = u.w;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < TK; ++kk) {
+      float a[8], b[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) a[i] = Qs[kk][ty * 8 + i];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) b[j] = Xs[kk][tx * 8 + j];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          if (METRIC == kL2) {
+            float t = a[i] - b[j];
+            acc[i][j] = fmaf(t, t, acc[i][j]);
+          } else {
+            acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+          }
+        }
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int64_t r = q0 + ty * 8 + i;
+    if (r >= qn) continue;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int64_t c = x0 + tx * 8 + j;
+      if (c < xn) D[r * ldD + c] = (METRIC == kL2) ? acc[i][j] : -acc[i][j];
+    }
+  }
+}
+
+// ------------------------------------------------------------------ running top-k selection
+constexpr int SEL_WARPS = 4;
+constexpr int SEL_BUF = 64;
+
+// one warp per query row; the row's sorted top-k keys live in HBM between
+// chunks and in shared memory (double buffered) while a chunk is scanned.
+__global__ void __launch_bounds__(SEL_WARPS * 32) select_kernel(const float* __restrict__ D, int64_t ldD, int rows,
+                                                                int64_t cols, int64_t col0, int64_t row0,
+                                                                int64_t self_base, int k,
+                                                                unsigned long long* __restrict__ state) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int row = blockIdx.x * SEL_WARPS + warp;
+  unsigned long long* la = reinterpret_cast<unsigned long long*>(sm) + (size_t)warp * (2 * k + SEL_BUF);
+  unsigned long long* lb = la + k;
+  unsigned long long* buf = lb + k;
+  if (row >= rows) return;
+  unsigned long long* st = state + (size_t)row * k;
+  for (int i = lane; i < k; i += 32) la[i] = st[i];
+  __syncwarp();
+  unsigned long long* cur = la;
+  unsigned long long* oth = lb;
+  int nb = 0;
+  const int64_t self = self_base >= 0 ? self_base + row0 + row : -1;
+  const float* dr = D + (size_t)row * ldD;
+  auto flush = [&]() {
+    // sort buf[0..64) (padded) with a smem bitonic network, then rank-merge
+    for (int i = nb + lane; i < SEL_BUF; i += 32) buf[i] = kKeyMax;
+    __syncwarp();
+    for (int kk = 2; kk <= SEL_BUF; kk <<= 1)
+      for (int j = kk >> 1; j > 0; j >>= 1) {
+        const int i = lane;  // SEL_BUF/2 == 32 pairs
+        const int lo = 2 * j * (i / j) + (i % j), hi = lo + j;
+        const bool up = (lo & kk) == 0;
+        unsigned long long a = buf[lo], b = buf[hi];
+        if ((a > b) == up) { buf[lo] = b; buf[hi] = a; }
+        __syncwarp();
+      }
+    for (int i = lane; i < nb; i += 32) {
+      const int pos = i + lower_bound_u64(cur, k, buf[i]);
+      if (pos < k) oth[pos] = buf[i];
+    }
+    for (int j = lane; j < k; j += 32) {
+      const int pos = j + lower_bound_u64(buf, nb, cur[j]);
+      if (pos < k) oth[pos] = cur[j];
+    }
+    __syncwarp();
+    unsigned long long* t = cur; cur = oth; oth = t;
+    nb = 0;
+  };
+  for (int64_t base = 0; base < cols; base += 32) {
+    const int64_t c = base + lane;
+    unsigned long long key = kKeyMax;
+    if (c < cols) {
+      const int64_t id = col0 + c;
+      if (id != self) key = make_key(dr[c], (uint32_t)id);
+    }
+    const unsigned long long thr = cur[k - 1];
+    const bool cand = key < thr;
+    const unsigned m = __ballot_sync(0xffffffffu, cand);
+    if (m == 0) continue;
+    const int cnt = __popc(m);
+    if (nb + cnt > SEL_BUF) flush();
+    if (cand) buf[nb + __popc(m & ((1u << lane) - 1u))] = key;
+    nb += cnt;
+    __syncwarp();
+    if (nb > SEL_BUF - 32) flush();
+  }
+  if (nb > 0) flush();
+  for (int i = lane; i < k; i += 32) st[i] = cur[i];
+}
+
+__global__ void init_state_kernel(unsigned long long* s, size_t n) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) s[i] = kKeyMax;
+}
+__global__ void decode_state_kernel(const unsigned long long* s, size_t n, uint32_t* ids, float* ds) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  unsigned long long k = s[i];
+  if (k == kKeyMax) {
+    ids[i] = kSentinel;
+    ds[i] = __int_as_float(0x7f800000);
+  } else {
+    ids[i] = key_id(k);
+    ds[i] = key_dist(k);
+  }
+}
+
+// ------------------------------------------------------------------ prune (R24)
+// step 1+2: detour counts and the pruned list (CTA per node, K <= 128)
+__global__ void detour_prune_kernel(const uint32_t* __restrict__ knn, int64_t n, int K, int R,
+                                    uint32_t* __restrict__ pruned) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  uint32_t* rows = reinterpret_cast<uint32_t*>(sm);  // K x K
+  uint32_t* cnt = rows + (size_t)K * K;               // K
+  const int64_t x = blockIdx.x;
+  const uint32_t* rx = knn + x * K;
+  for (int t = threadIdx.x; t < K * K; t += blockDim.x) {
+    const int i = t / K, c = t % K;
+    rows[t] = knn[(int64_t)rx[i] * K + c];
+  }
+  __syncthreads();
+  const int j = threadIdx.x;
+  if (j < K) {
+    const uint32_t yj = rx[j];
+    int count = 0;
+    for (int i = 0; i < j; ++i) {
+      const uint32_t* ri = rows + (size_t)i * K;
+      for (int t = 0; t < j; ++t)
+        if (ri[t] == yj) { ++count; break; }
+    }
+    cnt[j] = (uint32_t)count;
+  }
+  __syncthreads();
+  if (j < K) {
+    const uint32_t cj = cnt[j];
+    int rank = 0;
+    for (int i = 0; i < K; ++i) {
+      const uint32_t ci = cnt[i];
+      rank += (ci < cj) || (ci == cj && i < j);
+    }
+    if (rank < R) pruned[x * R + rank] = rx[j];
+  }
+}
+
+__global__ void indegree_kernel(const uint32_t* pruned, int64_t n, int R, uint32_t* indeg) {
+  int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= n * R) return;
+  atomicAdd(indeg + pruned[t], 1u);
+}
+__global__ void scatter_rev_kernel(const uint32_t* pruned, int64_t n, int R, const uint64_t* off, uint32_t* fill,
+                                   unsigned long long* rev) {
+  int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= n * R) return;
+  const uint32_t y = pruned[t];
+  const uint64_t x = (uint64_t)(t / R), r = (uint64_t)(t % R);
+  const uint64_t pos = off[y] + atomicAdd(fill + y, 1u);
+  rev[pos] = (r << 32) | x;  // ordered by (rank, source)
+}
+__global__ void merge_out_kernel(const uint32_t* pruned, const unsigned long long* rev, const uint64_t* off,
+                                 int64_t n, int R, uint32_t* out) {
+  int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (x >= n) return;
+  const uint32_t* p = pruned + x * R;
+  uint32_t* o = out + x * R;
+  int m = (int)(off[x + 1] - off[x]);
+  if (m > R) m = R;
+  const int h = R / 2;
+  int cnt = 0;
+  auto has = [&](uint32_t v) {
+    for (int t = 0; t < cnt; ++t)
+      if (o[t] == v) return true;
+    return false;
+  };
+  for (int j = 0; j < h; ++j) o[cnt++] = p[j];
+  for (int i = 0; i < m && cnt < R; ++i) {
+    const uint32_t v = (uint32_t)(rev[off[x] + i] & 0xFFFFFFFFull);
+    if (!has(v)) o[cnt++] = v;
+  }
+  for (int j = h; j < R && cnt < R; ++j)
+    if (!has(p[j])) o[cnt++] = p[j];
+  for (; cnt < R; ++cnt) o[cnt] = kSentinel;
+}
+
+struct Dev {
+  void* p = nullptr;
+  ~Dev() {
+    if (p) cudaFree(p);
+  }
+};
+
+static int to_device(const void* src, size_t bytes, Dev& holder, const void** out) {
+  if (is_device_ptr(src)) {
+    *out = src;
+    return ALGAS_OK;
+  }
+  ALGAS_CUDA_TRY(cudaMalloc(&holder.p, std::max<size_t>(bytes, 16)));
+  ALGAS_CUDA_TRY(cudaMemcpy(holder.p, src, bytes, cudaMemcpyHostToDevice));
+  *out = holder.p;
+  return ALGAS_OK;
+}
+
+}  // namespace algas
+
+using namespace algas;
+
+extern "C" {
+
+int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, int32_t dim, int32_t metric, int32_t k,
+              int64_t self_base, uint32_t* out_ids, float* out_dists) {
+  if (!base || !queries || !out_ids || !out_dists || n < 1 || n >= (1LL << 31) || nq < 0 || dim < 4 ||
+      dim % 4 != 0 || k < 1 || k > 1024 || (metric != ALGAS_L2 && metric != ALGAS_IP))
+    return set_error(ALGAS_EINVAL, "algas_knn: bad arguments");
+  if (nq == 0) return ALGAS_OK;
+  Dev hx, hq, hstate, hD, hid, hd;
+  const float *X = nullptr, *Q = nullptr;
+  int rc;
+  if ((rc = to_device(base, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
+  if ((rc = to_device(queries, (size_t)nq * dim * 4, hq, (const void**)&Q))) return rc;
+  const int64_t QB = std::min<int64_t>(nq, 4096);
+  const int64_t NB = std::min<int64_t>(n, 65536);
+  ALGAS_CUDA_TRY(cudaMalloc(&hstate.p, (size_t)QB * k * 8));
+  ALGAS_CUDA_TRY(cudaMalloc(&hD.p, (size_t)QB * NB * 4));
+  const bool dev_out = is_device_ptr(out_ids) && is_device_ptr(out_dists);
+  std::vector<uint32_t> hids;
+  std::vector<float> hds;
+  ALGAS_CUDA_TRY(cudaMalloc(&hid.p, (size_t)QB * k * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hd.p, (size_t)QB * k * 4));
+  const int sel_smem = SEL_WARPS * (2 * k + SEL_BUF) * 8;
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem));
+  auto* unsafe_D = (float*)hD.p;
+  for (int64_t q0 = 0; q0 < nq; q0 += QB) {
+    const int64_t qb = std::min<int64_t>(QB, nq - q0);
+    const size_t ns = (size_t)qb * k;
+    init_state_kernel<<<(unsigned)((ns + 255) / 256), 256>>>((unsigned long long*)hstate.p, ns);
+    for (int64_t x0 = 0; x0 < n; x0 += NB) {
+      const int64_t nb = std::min<int64_t>(NB, n - x0);
+      dim3 grid((unsigned)((nb + TX - 1) / TX), (unsigned)((qb + TQ - 1) / TQ));
+      if (metric == ALGAS_L2)
+        dist_tile_kernel<kL2><<<grid, 256>>>(Q + q0 * dim, qb, X + x0 * dim, nb, dim, unsafe_D, NB);
+      else
+        dist_tile_kernel<kIP><<<grid, 256>>>(Q + q0 * dim, qb, X + x0 * dim, nb, dim, unsafe_D, NB);
+      select_kernel<<<(unsigned)((qb + SEL_WARPS - 1) / SEL_WARPS), SEL_WARPS * 32, sel_smem>>>(
+          unsafe_D, NB, (int)qb, nb, x0, q0, self_base, k, (unsigned long long*)hstate.p);
+    }
+    decode_state_kernel<<<(unsigned)((ns + 255) / 256), 256>>>((unsigned long long*)hstate.p, ns, (uint32_t*)hid.p,
+                                                               (float*)hd.p);
+    ALGAS_CUDA_TRY(cudaGetLastError());
+    ALGAS_CUDA_TRY(cudaMemcpy(out_ids + q0 * k, hid.p, ns * 4, cudaMemcpyDefault));
+    ALGAS_CUDA_TRY(cudaMemcpy(out_dists + q0 * k, hd.p, ns * 4, cudaMemcpyDefault));
+  }
+  (void)dev_out;
+  ALGAS_CUDA_TRY(cudaDeviceSynchronize());
+  return ALGAS_OK;
+}
+
+int algas_prune(const uint32_t* knn, int64_t n, int32_t knn_degree, int32_t degree, uint32_t* out_graph) {
+  if (!knn || !out_graph || n < 1 || knn_degree < 1 || knn_degree > 128 || degree < 1 || degree > knn_degree)
+    return set_error(ALGAS_EINVAL, "algas_prune: need 1 <= degree <= knn_degree <= 128");
+  const int K = knn_degree, R = degree;
+  Dev hk, hp, hindeg, hoff, hfill, hrev, hrev2, htmp, hout;
+  const uint32_t* dk = nullptr;
+  int rc;
+  if ((rc = to_device(knn, (size_t)n * K * 4, hk, (const void**)&dk))) return rc;
+  ALGAS_CUDA_TRY(cudaMalloc(&hp.p, (size_t)n * R * 4));
+  const int threads = K <= 32 ? 32 : (K <= 64 ? 64 : 128);
+  const int smem = (K * K + K) * 4;
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(detour_prune_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  detour_prune_kernel<<<(unsigned)n, threads, smem>>>(dk, n, K, R, (uint32_t*)hp.p);
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  // reverse edges
+  ALGAS_CUDA_TRY(cudaMalloc(&hindeg.p, (size_t)(n + 1) * 4));
+  ALGAS_CUDA_TRY(cudaMemset(hindeg.p, 0, (size_t)(n + 1) * 4));
+  const int64_t E = n * R;
+  indegree_kernel<<<(unsigned)((E + 255) / 256), 256>>>((uint32_t*)hp.p, n, R, (uint32_t*)hindeg.p);
+  ALGAS_CUDA_TRY(cudaMalloc(&hoff.p, (size_t)(n + 1) * 8));
+  {
+    // exclusive scan of in-degrees (as u64) -> segment offsets
+    std::vector<uint32_t> indeg(n + 1);
+    ALGAS_CUDA_TRY(cudaMemcpy(indeg.data(), hindeg.p, (size_t)(n + 1) * 4, cudaMemcpyDeviceToHost));
+    std::vector<uint64_t> off(n + 1);
+    uint64_t acc = 0;
+    for (int64_t i = 0; i <= n; ++i) { off[i] = acc; if (i < n) acc += indeg[i]; }
+    ALGAS_CUDA_TRY(cudaMemcpy(hoff.p, off.data(), (size_t)(n + 1) * 8, cudaMemcpyHostToDevice));
+  }
+  ALGAS_CUDA_TRY(cudaMalloc(&hfill.p, (size_t)n * 4));
+  ALGAS_CUDA_TRY(cudaMemset(hfill.p, 0, (size_t)n * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hrev.p, (size_t)E * 8));
+  ALGAS_CUDA_TRY(cudaMalloc(&hrev2.p, (size_t)E * 8));
+  scatter_rev_kernel<<<(unsigned)((E + 255) / 256), 256>>>((uint32_t*)hp.p, n, R, (uint64_t*)hoff.p,
+                                                           (uint32_t*)hfill.p, (unsigned long long*)hrev.p);
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  {
+    size_t tmp = 0;
+    const uint64_t* offp = (const uint64_t*)hoff.p;
+    ALGAS_CUDA_TRY(cub::DeviceSegmentedSort::SortKeys(nullptr, tmp, (const unsigned long long*)hrev.p,
+                                                      (unsigned long long*)hrev2.p, (int)E, (int)n, offp,
+                                                      offp + 1));
+    ALGAS_CUDA_TRY(cudaMalloc(&htmp.p, std::max<size_t>(tmp, 16)));
+    ALGAS_CUDA_TRY(cub::DeviceSegmentedSort::SortKeys(htmp.p, tmp, (const unsigned long long*)hrev.p,
+                                                      (unsigned long long*)hrev2.p, (int)E, (int)n, offp,
+                                                      offp + 1));
+  }
+  uint32_t* dout = out_graph;
+  const bool dev_out = is_device_ptr(out_graph);
+  if (!dev_out) {
+    ALGAS_CUDA_TRY(cudaMalloc(&hout.p, (size_t)n * R * 4));
+    dout = (uint32_t*)hout.p;
+  }
+  merge_out_kernel<<<(unsigned)((n + 127) / 128), 128>>>((uint32_t*)hp.p, (unsigned long long*)hrev2.p,
+                                                         (uint64_t*)hoff.p, n, R, dout);
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  if (!dev_out) ALGAS_CUDA_TRY(cudaMemcpy(out_graph, dout, (size_t)n * R * 4, cudaMemcpyDeviceToHost));
+  ALGAS_CUDA_TRY(cudaDeviceSynchronize());
+  return ALGAS_OK;
+}
+
+int algas_build_graph(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t knn_degree, int32_t degree,
+                      int32_t prune, uint32_t* out_graph) {
+  if (!data || !out_graph || n < 2 || knn_degree < degree || degree < 1)
+    return set_error(ALGAS_EINVAL, "algas_build_graph: bad arguments");
+  const int K = (int)std::min<int64_t>(knn_degree, n - 1);
+  const int R = std::min(degree, K);
+  uint32_t* dk = nullptr;
+  float* dd = nullptr;
+  ALGAS_CUDA_TRY(cudaMalloc(&dk, (size_t)n * K * 4));
+  Dev guard_k;
+  guard_k.p = dk;
+  ALGAS_CUDA_TRY(cudaMalloc(&dd, (size_t)n * K * 4));
+  Dev guard_d;
+  guard_d.p = dd;
+  int rc = algas_knn(data, n, data, n, dim, metric, K, 0, dk, dd);
+  if (rc) return rc;
+  std::vector<uint32_t> tmp;
+  if (prune) {
+    if (R == degree) return algas_prune(dk, n, K, R, out_graph);
+    tmp.resize((size_t)n * R);
+    if ((rc = algas_prune(dk, n, K, R, tmp.data()))) return rc;
+  } else {
+    tmp.resize((size_t)n * R);
+    ALGAS_CUDA_TRY(cudaMemcpy2D(tmp.data(), (size_t)R * 4, dk, (size_t)K * 4, (size_t)R * 4, (size_t)n,
+                                cudaMemcpyDeviceToHost));
+    if (R == degree) {
+      ALGAS_CUDA_TRY(cudaMemcpy(out_graph, tmp.data(), tmp.size() * 4, cudaMemcpyDefault));
+      return ALGAS_OK;
+    }
+  }
+  // n - 1 < degree: pad rows with sentinels
+  std::vector<uint32_t> full((size_t)n * degree, kSentinel);
+  for (int64_t i = 0; i < n; ++i) std::copy(tmp.begin() + i * R, tmp.begin() + (i + 1) * R, full.begin() + i * degree);
+  ALGAS_CUDA_TRY(cudaMemcpy(out_graph, full.data(), full.size() * 4, cudaMemcpyDefault));
+  return ALGAS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,489 @@
+// runtime.cu -- host runtime of ALGAS:
+//   * TopK merge & filter on the host (A9): a priority queue over
+//     the T sorted per-CTA lists of one query, sentinels and repeated ids
+//     filtered out;
+//   * adaptive tuning;
+//   * the persistent server: host-mapped slot ring with per-slot state
+//     machine, one poller thread that watches the per-CTA
+//     Finish flags in host memory (local polling), merges and
+//     recycles the slot (Done -> None).
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <deque>
+#include <limits>
+#include <queue>
+#include <thread>
+#include <vector>
+
+#include "internal.h"
+
+namespace algas {
+
+// ------------------------------------------------------------------ A9 merge
+int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t* out_ids, float* out_d) {
+  // heap entry: (dist, id, cta, pos) -- min-heap on (dist, id)
+  struct H {
+    float d;
+    uint32_t id;
+    int c, p;
+  };
+  auto greater = [](const H& a, const H& b) {
+    if (a.d != b.d) return a.d > b.d;
+    return a.id > b.id;
+  };
+  std::priority_queue<H, std::vector<H>, decltype(greater)> pq(greater);
+  for (int c = 0; c < T; ++c) {
+    const ResultEntry& e = res[(size_t)c * kin];
+    if (kin > 0 && e.id != kSentinel) pq.push(H{e.dist, e.id, c, 0});
+  }
+  int n = 0;
+  while (!pq.empty() && n < k) {
+    H h = pq.top();
+    pq.pop();
+    bool dup = false;
+    for (int i = 0; i < n; ++i)
+      if (out_ids[i] == h.id) { dup = true; break; }
+    if (!dup) {
+      out_ids[n] = h.id;
+      out_d[n] = h.d;
+      ++n;
+    }
+    if (h.p + 1 < kin) {
+      const ResultEntry& e = res[(size_t)h.c * kin + h.p + 1];
+      if (e.id != kSentinel) pq.push(H{e.dist, e.id, h.c, h.p + 1});
+    }
+  }
+  for (int i = n; i < k; ++i) {
+    out_ids[i] = kSentinel;
+    out_d[i] = std::numeric_limits<float>::infinity();
+  }
+  return n;
+}
+
+}  // namespace algas
+
+using namespace algas;
+
+// ------------------------------------------------------------------ server
+struct algas_server {
+  algas_index* idx = nullptr;
+  Plan plan;
+  int slots = 0, T = 0, kmax = 0, dim = 0, d4 = 0;
+  cudaStream_t stream = nullptr;
+  // host-mapped ring (host pointer / device alias)
+  RingSlot* ring_h = nullptr;
+  RingSlot* ring_d = nullptr;
+  float* ringq_h = nullptr;
+  float4* ringq_d = nullptr;
+  ResultEntry* res_h = nullptr;
+  ResultEntry* res_d = nullptr;
+  CtaStats* st_h = nullptr;
+  CtaStats* st_d = nullptr;
+  uint32_t* done_h = nullptr;
+  uint32_t* done_d = nullptr;
+  // device mailbox
+  void* ctl = nullptr;
+  float4* qbuf = nullptr;
+  unsigned long long* gtab = nullptr;  // the server's own HBM spill tables
+  // host-side slot bookkeeping (host owns: EMPTY/claimed/in-flight)
+  std::vector<std::atomic<int>>* hstate = nullptr;  // 0 free, 1 claimed, 2 in flight
+  std::vector<uint32_t> epoch;
+  std::vector<uint64_t> tags;
+  std::vector<int> kq;
+  std::vector<std::chrono::steady_clock::time_point> t_submit;
+  std::atomic<int> next_slot{0};
+  std::thread poller;
+  std::atomic<bool> stop{false};
+  std::atomic<bool> kernel_ok{true};
+  std::mutex cq_mu;
+  struct Done {
+    uint64_t tag;
+    std::vector<uint32_t> ids;
+    std::vector<float> d;
+    algas_query_stats st;
+  };
+  std::deque<Done> cq;
+  std::atomic<int64_t> inflight{0};
+};
+
+static void poller_main(algas_server* s) {
+  const int T = s->T;
+  std::vector<uint32_t> ids(s->kmax);
+  std::vector<float> ds(s->kmax);
+  int idle = 0;
+  while (!s->stop.load(std::memory_order_acquire)) {
+    bool any = false;
+    for (int q = 0; q < s->slots; ++q) {
+      if ((*s->hstate)[q].load(std::memory_order_acquire) != 2) continue;
+      const uint32_t ep = s->epoch[q];
+      bool all = true;
+      for (int c = 0; c < T; ++c) {
+        // local polling of host memory: no PCIe traffic
+        uint32_t v = __atomic_load_n(&s->done_h[(size_t)q * T + c], __ATOMIC_ACQUIRE);
+        if (v != ep) { all = false; break; }
+      }
+      if (!all) continue;
+      any = true;
+      algas_server::Done d;
+      d.tag = s->tags[q];
+      const int k = s->kq[q];
+      const ResultEntry* r = s->res_h + (size_t)q * T * s->kmax;
+      d.ids.assign(s->kmax, kSentinel);
+      d.d.assign(s->kmax, std::numeric_limits<float>::infinity());
+      if (T == 1) {
+        for (int i = 0; i < k; ++i) { d.ids[i] = r[i].id; d.d[i] = r[i].dist; }
+      } else {
+        merge_cta_lists(r, T, s->kmax, k, d.ids.data(), d.d.data());
+      }
+      memset(&d.st, 0, sizeof(d.st));
+      d.st.ctas = (uint32_t)T;
+      uint64_t t0 = ~0ull, t1 = 0;
+      for (int c = 0; c < T; ++c) {
+        const CtaStats& cs = s->st_h[(size_t)q * T + c];
+        d.st.iters += cs.iters;
+        d.st.max_iters = std::max(d.st.max_iters, cs.iters);
+        d.st.parents += cs.parents;
+        d.st.dist_evals += cs.dist_evals;
+        d.st.cap_hits += cs.cap_hit;
+        d.st.spills += cs.spilled;
+        d.st.overflows += cs.overflow;
+        t0 = std::min<uint64_t>(t0, cs.t_start);
+        t1 = std::max<uint64_t>(t1, cs.t_end);
+      }
+      d.st.t_start_ns = t0;
+      d.st.t_end_ns = t1;
+      d.st.latency_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+                            std::chrono::steady_clock::now() - s->t_submit[q])
+                            .count();
+      {
+        std::lock_guard<std::mutex> lk(s->cq_mu);
+        s->cq.push_back(std::move(d));
+      }
+      // Done -> None: host owns the slot again
+      __atomic_store_n(&s->ring_h[q].state, (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
+      (*s->hstate)[q].store(0, std::memory_order_release);
+    }
+    if (!any) {
+      if (++idle > 64) {
+        std::this_thread::yield();
+        idle = 0;
+      }
+    } else {
+      idle = 0;
+    }
+  }
+}
+
+extern "C" {
+
+int algas_server_create(const algas_index* cidx, const algas_params* params, algas_server** out) {
+  if (!out) return set_error(ALGAS_EINVAL, "null out");
+  *out = nullptr;
+  algas_index* idx = const_cast<algas_index*>(cidx);
+  if (!idx || !params) return set_error(ALGAS_EINVAL, "null argument");
+  if (params->visited_mode != ALGAS_VISITED_PRIVATE)
+    return set_error(ALGAS_EINVAL, "server: SHARED visited mode not implemented yet");
+  const int slots = params->slots > 0 ? params->slots : 32;
+  algas_server* s = new algas_server();
+  s->idx = idx;
+  int rc = make_plan(idx, params, slots, &s->plan, true);
+  if (rc) { delete s; return rc; }
+  s->slots = slots;
+  s->T = s->plan.T;
+  s->kmax = s->plan.k;
+  s->dim = idx->dim;
+  s->d4 = idx->d4;
+  int nsm = 0, dev = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  if ((int64_t)slots * s->T > (int64_t)s->plan.blocks_per_sm * nsm) {
+    delete s;
+    return set_error(ALGAS_EINVAL, "%d slots x %d CTAs exceed co-resident capacity %d x %d SMs (P:L231)", slots,
+                     s->plan.T, s->plan.blocks_per_sm, nsm);
+  }
+  auto cleanup = [&](int code) {
+    algas_server_destroy(s);
+    return code;
+  };
+  const unsigned fl = cudaHostAllocMapped | cudaHostAllocPortable;
+  cudaError_t e;
+#define SRV_ALLOC(hp, dp, bytes)                                                       \
+  if ((e = cudaHostAlloc((void**)&hp, (bytes), fl)) != cudaSuccess)                    \
+    return cleanup(set_error(ALGAS_ENOMEM, "cudaHostAlloc: %s", cudaGetErrorString(e))); \
+  memset(hp, 0, (bytes));                                                              \
+  if ((e = cudaHostGetDevicePointer((void**)&dp, hp, 0)) != cudaSuccess)               \
+    return cleanup(set_error(ALGAS_ECUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(e)));
+  SRV_ALLOC(s->ring_h, s->ring_d, sizeof(RingSlot) * slots);
+  SRV_ALLOC(s->ringq_h, s->ringq_d, (size_t)slots * s->dim * 4);
+  SRV_ALLOC(s->res_h, s->res_d, sizeof(ResultEntry) * (size_t)slots * s->T * s->kmax);
+  SRV_ALLOC(s->st_h, s->st_d, sizeof(CtaStats) * (size_t)slots * s->T);
+  SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)slots * s->T);
+#undef SRV_ALLOC
+  s->hstate = new std::vector<std::atomic<int>>(slots);
+  for (auto& a : *s->hstate) a.store(0);
+  s->epoch.assign(slots, 0);
+  s->tags.assign(slots, 0);
+  s->kq.assign(slots, s->kmax);
+  s->t_submit.resize(slots);
+  const size_t ctl_bytes = control_bytes(slots);
+  if ((e = cudaMalloc(&s->ctl, ctl_bytes)) != cudaSuccess)
+    return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc: %s", cudaGetErrorString(e)));
+  cudaMemset(s->ctl, 0, ctl_bytes);
+  if ((e = cudaMalloc(&s->qbuf, (size_t)slots * s->dim * 4)) != cudaSuccess)
+    return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc: %s", cudaGetErrorString(e)));
+  if ((e = cudaStreamCreateWithFlags(&s->stream, cudaStreamNonBlocking)) != cudaSuccess)
+    return cleanup(set_error(ALGAS_ECUDA, "stream: %s", cudaGetErrorString(e)));
+  // a server owns its spill tables (the index workspace serves batch searches)
+  const size_t gent = ((size_t)slots * s->T) << s->plan.cfg.gtab_bits;
+  if ((e = cudaMalloc(&s->gtab, gent * 8)) != cudaSuccess)
+    return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc spill tables: %s", cudaGetErrorString(e)));
+  cudaMemset(s->gtab, 0, gent * 8);
+  uint8_t* cb = (uint8_t*)s->ctl;
+  PersistArgs pa;
+  memset(&pa, 0, sizeof(pa));
+  pa.mode = 0;
+  pa.slots = slots;
+  pa.T = s->T;
+  pa.kmax = s->kmax;
+  pa.ring = s->ring_d;
+  pa.ring_q = s->ringq_d;
+  pa.ring_res = s->res_d;
+  pa.ring_stats = s->st_d;
+  pa.ring_done = s->done_d;
+  carve_control(cb, slots, &pa);
+  pa.qbuf = s->qbuf;
+  pa.gtab = s->gtab;
+  pa.epoch_base = 1;
+  cudaDeviceSynchronize();
+  rc = launch_persistent(s->plan, pa, s->stream);
+  if (rc) return cleanup(rc);
+  s->poller = std::thread(poller_main, s);
+  *out = s;
+  return ALGAS_OK;
+}
+
+int algas_submit(algas_server* s, const float* query, uint64_t tag, int32_t k, int32_t itopk, int32_t width) {
+  if (!s || !query) return set_error(ALGAS_EINVAL, "null argument");
+  if (s->stop.load()) return set_error(ALGAS_ESTATE, "server is shutting down");
+  if (k <= 0) k = s->kmax;
+  if (itopk <= 0) itopk = s->plan.cfg.L;
+  if (width <= 0) width = s->plan.cfg.w;
+  if (k > s->kmax || itopk > s->plan.cfg.L || k > itopk || width > s->plan.cfg.w)
+    return set_error(ALGAS_EINVAL, "submit: k=%d itopk=%d width=%d exceed server limits (%d,%d,%d)", k, itopk, width,
+                     s->kmax, s->plan.cfg.L, s->plan.cfg.w);
+  const int start = s->next_slot.fetch_add(1, std::memory_order_relaxed);
+  for (int i = 0; i < s->slots; ++i) {
+    const int q = (start + i) % s->slots;
+    int expect = 0;
+    if (!(*s->hstate)[q].compare_exchange_strong(expect, 1, std::memory_order_acq_rel)) continue;
+    // None -> Work: payload first, state word last (release)
+    memcpy(s->ringq_h + (size_t)q * s->dim, query, (size_t)s->dim * 4);
+    RingSlot* rs = &s->ring_h[q];
+    rs->k = k;
+    rs->L = itopk;
+    rs->w = width;
+    rs->tag = tag;
+    s->tags[q] = tag;
+    s->kq[q] = k;
+    const uint32_t ep = (s->epoch[q] + 1) & 0xFFFFFFu;
+    s->epoch[q] = ep == 0 ? 1 : ep;
+    s->t_submit[q] = std::chrono::steady_clock::now();
+    s->inflight.fetch_add(1);
+    (*s->hstate)[q].store(2, std::memory_order_release);
+    __atomic_store_n(&rs->state, (s->epoch[q] << 8) | kSlotReady, __ATOMIC_RELEASE);
+    return ALGAS_OK;
+  }
+  return ALGAS_EAGAIN;
+}
+
+int algas_poll(algas_server* s, uint64_t* tags, uint32_t* ids, float* dists, algas_query_stats* stats,
+               int32_t max_results, int32_t* n_out) {
+  if (!s || !n_out) return set_error(ALGAS_EINVAL, "null argument");
+  *n_out = 0;
+  if (max_results <= 0) return ALGAS_OK;
+  // a persistent kernel that died is reported, not silently waited on
+  cudaError_t e = cudaStreamQuery(s->stream);
+  if (e != cudaSuccess && e != cudaErrorNotReady)
+    return set_error(ALGAS_ECUDA, "persistent kernel failed: %s", cudaGetErrorString(e));
+  std::lock_guard<std::mutex> lk(s->cq_mu);
+  int n = 0;
+  while (n < max_results && !s->cq.empty()) {
+    algas_server::Done& d = s->cq.front();
+    if (tags) tags[n] = d.tag;
+    if (ids) memcpy(ids + (size_t)n * s->kmax, d.ids.data(), sizeof(uint32_t) * s->kmax);
+    if (dists) memcpy(dists + (size_t)n * s->kmax, d.d.data(), sizeof(float) * s->kmax);
+    if (stats) stats[n] = d.st;
+    s->cq.pop_front();
+    ++n;
+  }
+  s->inflight.fetch_sub(n);
+  *n_out = n;
+  return ALGAS_OK;
+}
+
+int algas_server_inflight(const algas_server* s, int64_t* n) {
+  if (!s || !n) return set_error(ALGAS_EINVAL, "null argument");
+  *n = s->inflight.load();
+  return ALGAS_OK;
+}
+
+int algas_server_destroy(algas_server* s) {
+  if (!s) return ALGAS_OK;
+  int rc = ALGAS_OK;
+  if (s->ring_h && s->stream) {
+    // Quit: every slot, then wait for the kernel to exit
+    for (int q = 0; q < s->slots; ++q) __atomic_store_n(&s->ring_h[q].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+    auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+      cudaError_t e = cudaStreamQuery(s->stream);
+      if (e == cudaSuccess) break;
+      if (e != cudaErrorNotReady) {
+        rc = set_error(ALGAS_ECUDA, "persistent kernel failed: %s", cudaGetErrorString(e));
+        break;
+      }
+      if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(30)) {
+        rc = set_error(ALGAS_ESTATE, "persistent kernel did not quit within 30 s");
+        break;
+      }
+      std::this_thread::sleep_for(std::chrono::microseconds(50));
+    }
+  }
+  s->stop.store(true);
+  if (s->poller.joinable()) s->poller.join();
+  if (rc == ALGAS_OK) {
+    if (s->gtab) cudaFree(s->gtab);
+    if (s->ctl) cudaFree(s->ctl);
+    if (s->qbuf) cudaFree(s->qbuf);
+    if (s->ring_h) cudaFreeHost(s->ring_h);
+    if (s->ringq_h) cudaFreeHost(s->ringq_h);
+    if (s->res_h) cudaFreeHost(s->res_h);
+    if (s->st_h) cudaFreeHost(s->st_h);
+    if (s->done_h) cudaFreeHost(s->done_h);
+    if (s->stream) cudaStreamDestroy(s->stream);
+    delete s->hstate;
+    delete s;
+  }
+  return rc;
+}
+
+int32_t algas_merge_topk(const uint32_t* ids, const float* dists, int32_t m, int32_t k, uint32_t* out_ids,
+                         float* out_dists) {
+  if (m < 0 || k < 1 || (m > 0 && (!ids || !dists)) || !out_ids || !out_dists)
+    return set_error(ALGAS_EINVAL, "algas_merge_topk: bad arguments");
+  std::vector<ResultEntry> all;
+  all.reserve(m);
+  for (int i = 0; i < m; ++i)
+    if (ids[i] != kSentinel) all.push_back(ResultEntry{ids[i], dists[i]});
+  std::sort(all.begin(), all.end(), [](const ResultEntry& a, const ResultEntry& b) {
+    if (a.dist != b.dist) return a.dist < b.dist;
+    return a.id < b.id;
+  });
+  // one sorted list; reuse the T-way merge with T = 1 for the filtering rule
+  std::vector<ResultEntry> one(all.size() + 1, ResultEntry{kSentinel, 0.f});
+  std::copy(all.begin(), all.end(), one.begin());
+  return merge_cta_lists(one.data(), 1, (int)all.size() + 1, k, out_ids, out_dists);
+}
+
+// ------------------------------------------------------------------ tuner
+int32_t algas_tuner_max_parallel(int32_t slots, int32_t n_sm, int32_t max_blocks_per_sm) {
+  if (slots < 1) return 0;
+  return (int32_t)(((int64_t)n_sm * max_blocks_per_sm) / slots);
+}
+int32_t algas_tuner_blocks_per_sm(int32_t n_parallel, int32_t slots, int32_t n_sm) {
+  if (n_sm < 1) return 0;
+  const int64_t t = (int64_t)n_parallel * slots;
+  return (int32_t)((t + n_sm - 1) / n_sm);  // P:L235, align() = ceil (R13)
+}
+int64_t algas_tuner_smem_per_block(int64_t smem_per_sm, int32_t blocks_per_sm, int64_t smem_reserved_per_block) {
+  if (blocks_per_sm < 1) return 0;
+  return smem_per_sm / blocks_per_sm - smem_reserved_per_block;
+}
+
+int algas_device_query(algas_device_props* out) {
+  if (!out) return set_error(ALGAS_EINVAL, "null out");
+  int dev = 0;
+  ALGAS_CUDA_TRY(cudaGetDevice(&dev));
+  int v = 0;
+  memset(out, 0, sizeof(*out));
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev));
+  out->n_sm = v;
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrMaxBlocksPerMultiprocessor, dev));
+  out->max_blocks_per_sm = v;
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+  out->smem_per_sm = v;
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrReservedSharedMemoryPerBlock, dev));
+  out->smem_reserved_per_block = v;
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  out->smem_per_block_optin = v;
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrMaxThreadsPerMultiProcessor, dev));
+  out->max_threads_per_sm = v;
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&v, cudaDevAttrMaxRegistersPerMultiprocessor, dev));
+  out->regs_per_sm = v;
+  return ALGAS_OK;
+}
+
+// Full tuner.  Policy ("tuner"):
+//  * threads/CTA: the paper fixes one warp; on B200 the distance
+//    gathers need more loads in flight per query, so 64 threads for d <= 128,
+//    128 above (one 16-B chunk per lane per vector row at 512 B rows).
+//  * N_parallel: the largest T allowed by P:L231 whose per-block shared memory
+//    fits P:L245 (with M_reserved grown for wide vectors), capped at
+//    T_cap = 8 beyond which extra CTAs mostly repeat work (measured in
+//    profiles/); small batches get the most CTAs per query.
+//  * width / offset_beam: beam extend in the diffusing phase:
+//    w = 1 for L <= 32, 2 for L <= 64, 4 above; off = L/4 (R6).
+int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int32_t degree, int32_t itopk, int32_t k,
+               algas_tuning* out) {
+  if (!out || slots < 1 || dim < 4 || degree < 1 || itopk < 1 || k < 1)
+    return set_error(ALGAS_EINVAL, "algas_tune: bad arguments");
+  algas_device_props dp;
+  if (!props) {
+    int rc = algas_device_query(&dp);
+    if (rc) return rc;
+    props = &dp;
+  }
+  const int nt = dim <= 128 ? 64 : 128;
+  const int w = itopk <= 32 ? 1 : (itopk <= 64 ? 2 : 4);
+  const int Rp = (degree + 3) / 4 * 4;
+  const int S = 32;
+  int ncap = 1;
+  while (ncap < std::max(S, w * Rp)) ncap <<= 1;
+  long long need = 8LL * itopk + 2LL * (S + w * Rp);
+  int hb = 10;
+  while ((1LL << hb) < need && hb < 15) ++hb;
+  const int d4 = dim / 4;
+  const int64_t smem = smem_layout(d4, itopk, ncap, hb).total;
+  // M_reserved_per_block: driver reservation + extra L1 for wide rows
+  const int64_t reserved = props->smem_reserved_per_block + (dim > 256 ? 8 * 1024 : 0);
+  const int tmax_eq = algas_tuner_max_parallel(slots, props->n_sm, props->max_blocks_per_sm);
+  const int tcap = std::min(8, ALGAS_MAX_CTAS);
+  int best = 0, best_bps = 0;
+  int64_t best_avail = 0;
+  for (int T = std::min(tmax_eq, tcap); T >= 1; --T) {
+    const int bps = algas_tuner_blocks_per_sm(T, slots, props->n_sm);
+    if (bps > props->max_blocks_per_sm) continue;
+    if ((int64_t)bps * nt > props->max_threads_per_sm) continue;
+    const int64_t avail = algas_tuner_smem_per_block(props->smem_per_sm, bps, reserved);
+    if (smem <= avail) {
+      best = T;
+      best_bps = bps;
+      best_avail = avail;
+      break;
+    }
+  }
+  if (best == 0) return set_error(ALGAS_EINVAL, "algas_tune: no N_parallel fits %d slots (smem %lld B)", slots, (long long)smem);
+  memset(out, 0, sizeof(*out));
+  out->ctas_per_query = best;
+  out->blocks_per_sm = best_bps;
+  out->smem_avail_per_block = best_avail;
+  out->smem_per_block = smem;
+  out->threads_per_cta = nt;
+  out->width = w;
+  out->offset_beam = std::max(1, itopk / 4);
+  out->hash_bits = hb;
+  (void)k;
+  return ALGAS_OK;
+}
+
+}  // extern "C"

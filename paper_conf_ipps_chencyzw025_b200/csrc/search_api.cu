@@ -1,0 +1,505 @@
+// search_api.cu -- C-ABI: errors, index lifetime, planning, batch search
+// (algas_search / algas_search_ex) and dynamic batching from an HBM queue
+// (algas_search_dynamic).  The host merge of per-CTA results is in
+// runtime.cu; graph construction in knn.cu.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <vector>
+
+#include "internal.h"
+
+namespace algas {
+
+static thread_local std::string g_err = "no error";
+
+int set_error(int code, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+static int ilog2_ceil(long long x) {
+  int b = 0;
+  while ((1LL << b) < x) ++b;
+  return b;
+}
+
+int ensure_gtab(algas_index* idx, size_t entries) {
+  Workspace* ws = idx->ws;
+  if (ws->gtab_entries >= entries) return ALGAS_OK;
+  if (ws->gtab) cudaFree(ws->gtab);
+  ws->gtab = nullptr;
+  ws->gtab_entries = 0;
+  ALGAS_CUDA_TRY(cudaMalloc(&ws->gtab, entries * sizeof(unsigned long long)));
+  ALGAS_CUDA_TRY(cudaMemset(ws->gtab, 0, entries * sizeof(unsigned long long)));
+  ws->gtab_entries = entries;
+  ws->epoch = 1;
+  return ALGAS_OK;
+}
+
+// Reserve `count` consecutive spill-table epochs; clears the tables on wrap.
+static int take_epochs(algas_index* idx, uint64_t count, uint32_t* base, cudaStream_t st) {
+  Workspace* ws = idx->ws;
+  if ((uint64_t)ws->epoch + count >= 0xFFFFFFF0ull) {
+    if (ws->gtab) ALGAS_CUDA_TRY(cudaMemsetAsync(ws->gtab, 0, ws->gtab_entries * 8, st));
+    ws->epoch = 1;
+  }
+  *base = ws->epoch;
+  ws->epoch += (uint32_t)count;
+  return ALGAS_OK;
+}
+
+int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent) {
+  Plan pl;
+  memset(&pl, 0, sizeof(pl));
+  const int L = p->itopk, k = p->k, w = p->width;
+  if (k < 1 || L < k || L > ALGAS_MAX_ITOPK)
+    return set_error(ALGAS_EINVAL, "need 1 <= k (%d) <= itopk (%d) <= %d", k, L, ALGAS_MAX_ITOPK);
+  if (w < 1 || w > ALGAS_MAX_WIDTH) return set_error(ALGAS_EINVAL, "width %d not in [1,%d]", w, ALGAS_MAX_WIDTH);
+  if (p->visited_mode != ALGAS_VISITED_PRIVATE && p->visited_mode != ALGAS_VISITED_SHARED)
+    return set_error(ALGAS_EINVAL, "bad visited_mode %d", p->visited_mode);
+  int S = p->n_seeds > 0 ? p->n_seeds : 32;
+  if (S > ALGAS_MAX_SEEDS) return set_error(ALGAS_EINVAL, "n_seeds %d > %d", S, ALGAS_MAX_SEEDS);
+  int T = p->ctas_per_query;
+  int nt = p->threads_per_cta;
+  if (T == 0 || nt == 0) {
+    algas_tuning tu;
+    int rc = algas_tune(nullptr, slots, idx->dim, idx->degree, L, k, &tu);
+    if (rc != ALGAS_OK) return rc;
+    if (T == 0) T = tu.ctas_per_query;
+    if (nt == 0) nt = tu.threads_per_cta;
+  }
+  if (T < 1 || T > ALGAS_MAX_CTAS) return set_error(ALGAS_EINVAL, "ctas_per_query %d not in [1,%d]", T, ALGAS_MAX_CTAS);
+  if (nt != 32 && nt != 64 && nt != 128 && nt != 256)
+    return set_error(ALGAS_EINVAL, "threads_per_cta %d not in {32,64,128,256}", nt);
+  const int cc = chunk_config_for(idx->d4);
+  if (cc < 0) return set_error(ALGAS_EINVAL, "dim %d unsupported", idx->dim);
+  const int Rp = idx->rp4 * 4;
+  int ncap = 1;
+  while (ncap < std::max(S, w * Rp)) ncap <<= 1;
+  int hb = p->hash_bits;
+  if (hb <= 0) {
+    long long need = 8LL * L + 2LL * (S + w * Rp);
+    hb = std::min(15, std::max(10, ilog2_ceil(need)));
+  }
+  if (hb < 6 || hb > 16) return set_error(ALGAS_EINVAL, "hash_bits %d not in [6,16]", hb);
+  if ((1 << hb) < 2 * (S + w * Rp))
+    return set_error(ALGAS_EINVAL, "visited hash 2^%d too small for seeds + one step (%d)", hb, S + w * Rp);
+  SmemLayout lay = smem_layout(idx->d4, L, ncap, hb);
+  int optin = 0, dev = 0;
+  ALGAS_CUDA_TRY(cudaGetDevice(&dev));
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  if (lay.total + 1024 > optin)
+    return set_error(ALGAS_EINVAL, "search needs %d B shared memory per CTA, device allows %d", lay.total, optin);
+
+  pl.nt = nt;
+  pl.ccfg = cc;
+  pl.T = T;
+  pl.k = k;
+  pl.smem = lay.total;
+  pl.visited_mode = p->visited_mode;
+  pl.metric = idx->metric;
+  SearchCfg& c = pl.cfg;
+  c.data = reinterpret_cast<const float4*>(idx->d_data);
+  c.graph = reinterpret_cast<const uint4*>(idx->d_graph);
+  c.n = (uint64_t)idx->n;
+  c.d4 = idx->d4;
+  c.R = idx->degree;
+  c.rp4 = idx->rp4;
+  c.L = L;
+  c.w = w;
+  c.off = p->offset_beam < 0 ? std::max(1, L / 4) : std::min(p->offset_beam, L);
+  c.S = S;
+  c.max_iter = p->max_iter > 0 ? p->max_iter : 4 * L + 256;
+  c.hash_bits = hb;
+  c.gtab_bits = std::min(20, hb + 2);
+  c.ncap = ncap;
+  c.seed = p->seed;
+  int nb = 0;
+  int rc = max_blocks_per_sm(pl, persistent, &nb);
+  if (rc != ALGAS_OK) return rc;
+  if (nb < 1) return set_error(ALGAS_EINVAL, "search kernel does not fit on an SM (smem %d)", pl.smem);
+  pl.blocks_per_sm = nb;
+  (void)slots;
+  *out = pl;
+  return ALGAS_OK;
+}
+
+static int num_sms() {
+  int dev = 0, n = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+  return n;
+}
+
+// RAII device buffer on a stream
+struct DevBuf {
+  void* p = nullptr;
+  cudaStream_t st = nullptr;
+  ~DevBuf() {
+    if (p) cudaFreeAsync(p, st);
+  }
+  int alloc(size_t bytes, cudaStream_t s) {
+    st = s;
+    ALGAS_CUDA_TRY(cudaMallocAsync(&p, std::max<size_t>(bytes, 16), s));
+    return ALGAS_OK;
+  }
+};
+
+static void aggregate_stats(const CtaStats* cs, int T, algas_query_stats* q) {
+  memset(q, 0, sizeof(*q));
+  q->ctas = (uint32_t)T;
+  uint64_t t0 = ~0ull, t1 = 0;
+  for (int c = 0; c < T; ++c) {
+    q->iters += cs[c].iters;
+    q->max_iters = std::max(q->max_iters, cs[c].iters);
+    q->parents += cs[c].parents;
+    q->dist_evals += cs[c].dist_evals;
+    q->cap_hits += cs[c].cap_hit;
+    q->spills += cs[c].spilled;
+    q->overflows += cs[c].overflow;
+    t0 = std::min<uint64_t>(t0, cs[c].t_start);
+    t1 = std::max<uint64_t>(t1, cs[c].t_end);
+  }
+  q->t_start_ns = t0 == ~0ull ? 0 : t0;
+  q->t_end_ns = t1;
+}
+
+// Host merge of nq x T x k per-CTA lists into the caller's outputs.
+static int finish_outputs(const std::vector<ResultEntry>& res, const std::vector<CtaStats>& cst, int64_t nq,
+                          int T, int kin, int k, uint32_t* out_ids, float* out_dists, uint32_t* out_cta_ids,
+                          float* out_cta_dists, algas_query_stats* out_stats, bool* overflow) {
+  const bool dev_ids = is_device_ptr(out_ids), dev_d = is_device_ptr(out_dists);
+  std::vector<uint32_t> hid;
+  std::vector<float> hd;
+  uint32_t* ids = out_ids;
+  float* ds = out_dists;
+  if (dev_ids) { hid.resize((size_t)nq * k); ids = hid.data(); }
+  if (dev_d) { hd.resize((size_t)nq * k); ds = hd.data(); }
+  for (int64_t q = 0; q < nq; ++q) {
+    const ResultEntry* r = res.data() + (size_t)q * T * kin;
+    if (T == 1) {
+      for (int i = 0; i < k; ++i) { ids[q * k + i] = r[i].id; ds[q * k + i] = r[i].dist; }
+    } else {
+      merge_cta_lists(r, T, kin, k, ids + q * k, ds + q * k);
+    }
+  }
+  if (dev_ids) ALGAS_CUDA_TRY(cudaMemcpy(out_ids, hid.data(), hid.size() * 4, cudaMemcpyHostToDevice));
+  if (dev_d) ALGAS_CUDA_TRY(cudaMemcpy(out_dists, hd.data(), hd.size() * 4, cudaMemcpyHostToDevice));
+  if (out_cta_ids || out_cta_dists) {
+    std::vector<uint32_t> ci((size_t)nq * T * kin);
+    std::vector<float> cd((size_t)nq * T * kin);
+    for (size_t i = 0; i < ci.size(); ++i) { ci[i] = res[i].id; cd[i] = res[i].dist; }
+    if (out_cta_ids) ALGAS_CUDA_TRY(cudaMemcpy(out_cta_ids, ci.data(), ci.size() * 4, cudaMemcpyDefault));
+    if (out_cta_dists) ALGAS_CUDA_TRY(cudaMemcpy(out_cta_dists, cd.data(), cd.size() * 4, cudaMemcpyDefault));
+  }
+  *overflow = false;
+  for (int64_t q = 0; q < nq; ++q) {
+    algas_query_stats qs;
+    aggregate_stats(cst.data() + q * T, T, &qs);
+    if (qs.overflows) *overflow = true;
+    if (out_stats) out_stats[q] = qs;
+  }
+  return ALGAS_OK;
+}
+
+// queries -> device (copy if host); returns pointer usable by kernels
+static int stage_queries(const algas_index* idx, const float* q, int64_t nq, DevBuf& buf, cudaStream_t st,
+                         const float4** out) {
+  if (is_device_ptr(q)) {
+    if (((uintptr_t)q & 15u) != 0) return set_error(ALGAS_EINVAL, "device queries must be 16-B aligned");
+    *out = reinterpret_cast<const float4*>(q);
+    return ALGAS_OK;
+  }
+  size_t bytes = (size_t)nq * idx->dim * 4;
+  int rc = buf.alloc(bytes, st);
+  if (rc) return rc;
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(buf.p, q, bytes, cudaMemcpyHostToDevice, st));
+  *out = reinterpret_cast<const float4*>(buf.p);
+  return ALGAS_OK;
+}
+
+struct EventTimer {
+  cudaStream_t st;
+  cudaEvent_t a = nullptr, b = nullptr;
+  explicit EventTimer(cudaStream_t s) : st(s) {}
+  ~EventTimer() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+  }
+  int start() {
+    ALGAS_CUDA_TRY(cudaEventCreate(&a));
+    ALGAS_CUDA_TRY(cudaEventCreate(&b));
+    ALGAS_CUDA_TRY(cudaEventRecord(a, st));
+    return ALGAS_OK;
+  }
+  int stop() {
+    ALGAS_CUDA_TRY(cudaEventRecord(b, st));
+    return ALGAS_OK;
+  }
+  float ms() {
+    float m = 0.f;
+    if (cudaEventElapsedTime(&m, a, b) != cudaSuccess) (void)cudaGetLastError();
+    return m;
+  }
+};
+
+static void fill_info(algas_run_info* info, const Plan& pl, int grid, float ms) {
+  memset(info, 0, sizeof(*info));
+  info->kernel_ms = ms;
+  info->grid = grid;
+  info->threads_per_cta = pl.nt;
+  info->ctas_per_query = pl.T;
+  info->smem_per_cta = pl.smem;
+  info->blocks_per_sm = pl.blocks_per_sm;
+  info->hash_bits = pl.cfg.hash_bits;
+}
+
+}  // namespace algas
+
+using namespace algas;
+
+extern "C" {
+
+void algas_params_default(algas_params* p) {
+  memset(p, 0, sizeof(*p));
+  p->k = 10;
+  p->itopk = 64;
+  p->width = 1;
+  p->offset_beam = -1;
+  p->ctas_per_query = 1;
+  p->threads_per_cta = 0;
+  p->n_seeds = 32;
+  p->max_iter = 0;
+  p->visited_mode = ALGAS_VISITED_PRIVATE;
+  p->slots = 32;
+  p->hash_bits = 0;
+  p->seed = 0;
+}
+
+const char* algas_last_error(void) { return g_err.c_str(); }
+const char* algas_version(void) { return "algas-b200 0.1 (sm_100a)"; }
+
+algas_index* algas_index_create(const float* data, int64_t n, int32_t dim, int32_t metric, const uint32_t* graph,
+                                int32_t degree) {
+  if (!data || n < 1 || n >= (1LL << 31) || dim < 4 || dim % 4 != 0 || dim > ALGAS_MAX_DIM || degree < 1 ||
+      degree > ALGAS_MAX_DEGREE || (metric != ALGAS_L2 && metric != ALGAS_IP)) {
+    set_error(ALGAS_EINVAL, "algas_index_create: bad arguments (n=%lld dim=%d degree=%d metric=%d)", (long long)n,
+              dim, degree, metric);
+    return nullptr;
+  }
+  algas_index* idx = new algas_index();
+  idx->n = n;
+  idx->dim = dim;
+  idx->d4 = dim / 4;
+  idx->metric = metric;
+  idx->degree = degree;
+  idx->rp4 = (degree + 3) / 4;
+  idx->ws = new Workspace();
+  cudaGetDevice(&idx->device);
+  const size_t dbytes = (size_t)n * dim * 4, gpitch = (size_t)idx->rp4 * 16;
+  auto fail = [&](const char* what, cudaError_t e) -> algas_index* {
+    set_error(e == cudaErrorMemoryAllocation ? ALGAS_ENOMEM : ALGAS_ECUDA, "algas_index_create: %s: %s", what,
+              cudaGetErrorString(e));
+    algas_index_destroy(idx);
+    return nullptr;
+  };
+  cudaError_t e;
+  if ((e = cudaMalloc(&idx->d_data, dbytes)) != cudaSuccess) return fail("cudaMalloc data", e);
+  if ((e = cudaMemcpy(idx->d_data, data, dbytes, cudaMemcpyDefault)) != cudaSuccess) return fail("copy data", e);
+  if ((e = cudaMalloc(&idx->d_graph, (size_t)n * gpitch)) != cudaSuccess) return fail("cudaMalloc graph", e);
+  if ((e = cudaMemset(idx->d_graph, 0xFF, (size_t)n * gpitch)) != cudaSuccess) return fail("memset graph", e);
+  std::vector<uint32_t> built;
+  const uint32_t* g = graph;
+  if (!g) {
+    built.resize((size_t)n * degree);
+    int rc = algas_build_graph(idx->d_data, n, dim, metric, std::min<int64_t>(2 * degree, std::max<int64_t>(1, n - 1)),
+                               degree, 1, built.data());
+    if (rc != ALGAS_OK) {
+      algas_index_destroy(idx);
+      return nullptr;
+    }
+    g = built.data();
+  }
+  if ((e = cudaMemcpy2D(idx->d_graph, gpitch, g, (size_t)degree * 4, (size_t)degree * 4, (size_t)n,
+                        cudaMemcpyDefault)) != cudaSuccess)
+    return fail("copy graph", e);
+  return idx;
+}
+
+int algas_index_destroy(algas_index* idx) {
+  if (!idx) return ALGAS_OK;
+  if (idx->d_data) cudaFree(idx->d_data);
+  if (idx->d_graph) cudaFree(idx->d_graph);
+  if (idx->ws) {
+    if (idx->ws->gtab) cudaFree(idx->ws->gtab);
+    if (idx->ws->counters) cudaFree(idx->ws->counters);
+    delete idx->ws;
+  }
+  delete idx;
+  return ALGAS_OK;
+}
+
+int algas_index_info(const algas_index* idx, int64_t* n, int32_t* dim, int32_t* metric, int32_t* degree,
+                     int32_t* graph_stride, const float** dev_data, const uint32_t** dev_graph) {
+  if (!idx) return set_error(ALGAS_EINVAL, "null index");
+  if (n) *n = idx->n;
+  if (dim) *dim = idx->dim;
+  if (metric) *metric = idx->metric;
+  if (degree) *degree = idx->degree;
+  if (graph_stride) *graph_stride = idx->rp4 * 4;
+  if (dev_data) *dev_data = idx->d_data;
+  if (dev_graph) *dev_graph = idx->d_graph;
+  return ALGAS_OK;
+}
+
+int algas_search(const algas_index* idx, const float* queries, int64_t nq, int32_t k, int32_t itopk, int32_t width,
+                 uint32_t* out_ids, float* out_dists) {
+  algas_params p;
+  algas_params_default(&p);
+  p.k = k;
+  p.itopk = itopk;
+  p.width = width;
+  return algas_search_ex(idx, queries, nq, &p, 0, out_ids, out_dists, nullptr, nullptr, nullptr, nullptr, nullptr);
+}
+
+int algas_search_ex(const algas_index* cidx, const float* queries, int64_t nq, const algas_params* params,
+                    uint64_t tag0, uint32_t* out_ids, float* out_dists, uint32_t* out_cta_ids, float* out_cta_dists,
+                    algas_query_stats* out_stats, void* stream, algas_run_info* info) {
+  algas_index* idx = const_cast<algas_index*>(cidx);
+  if (!idx || !params || !queries || !out_ids || !out_dists || nq < 0)
+    return set_error(ALGAS_EINVAL, "algas_search_ex: null argument");
+  if (nq == 0) return ALGAS_OK;
+  if (params->visited_mode != ALGAS_VISITED_PRIVATE)
+    return set_error(ALGAS_EINVAL, "algas_search_ex: SHARED visited mode is served by the persistent paths only");
+  Plan pl;
+  int rc = make_plan(idx, params, 1, &pl, false);
+  if (rc) return rc;
+  if (nq * pl.T >= (1LL << 31)) return set_error(ALGAS_EINVAL, "nq * T too large");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const int64_t items = nq * pl.T;
+  const int grid = (int)std::min<int64_t>(items, (int64_t)pl.blocks_per_sm * num_sms());
+
+  std::lock_guard<std::mutex> lk(idx->ws->mu);
+  if ((rc = ensure_gtab(idx, (size_t)grid << pl.cfg.gtab_bits))) return rc;
+  if (!idx->ws->counters) ALGAS_CUDA_TRY(cudaMalloc(&idx->ws->counters, 4096));
+  uint32_t epoch_base = 1;
+  if ((rc = take_epochs(idx, (uint64_t)items + 1, &epoch_base, st))) return rc;
+
+  DevBuf qb, rb, sb;
+  const float4* dq = nullptr;
+  if ((rc = stage_queries(idx, queries, nq, qb, st, &dq))) return rc;
+  if ((rc = rb.alloc((size_t)items * pl.k * sizeof(ResultEntry), st))) return rc;
+  if ((rc = sb.alloc((size_t)items * sizeof(CtaStats), st))) return rc;
+  ALGAS_CUDA_TRY(cudaMemsetAsync(sb.p, 0, (size_t)items * sizeof(CtaStats), st));
+  BatchLaunch bl;
+  bl.queries = dq;
+  bl.nq = nq;
+  bl.tag0 = tag0;
+  bl.res = (ResultEntry*)rb.p;
+  bl.stats = (CtaStats*)sb.p;
+  bl.gtab = idx->ws->gtab;
+  bl.epoch_base = epoch_base;
+  bl.work_counter = idx->ws->counters;
+  bl.grid = grid;
+  EventTimer tm(st);
+  if ((rc = tm.start())) return rc;
+  if ((rc = launch_batch(pl, bl, st))) return rc;
+  if ((rc = tm.stop())) return rc;
+  std::vector<ResultEntry> res((size_t)items * pl.k);
+  std::vector<CtaStats> cst((size_t)items);
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(res.data(), rb.p, res.size() * sizeof(ResultEntry), cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst.data(), sb.p, cst.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaStreamSynchronize(st));
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  if (info) fill_info(info, pl, grid, tm.ms());
+  bool ovf = false;
+  if ((rc = finish_outputs(res, cst, nq, pl.T, pl.k, pl.k, out_ids, out_dists, out_cta_ids, out_cta_dists, out_stats,
+                           &ovf)))
+    return rc;
+  return ovf ? set_error(ALGAS_EOVERFLOW, "a visited table overflowed") : ALGAS_OK;
+}
+
+int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int64_t nq, const algas_params* params,
+                         uint64_t tag0, uint32_t* out_ids, float* out_dists, algas_query_stats* out_stats,
+                         void* stream, algas_run_info* info) {
+  algas_index* idx = const_cast<algas_index*>(cidx);
+  if (!idx || !params || !queries_dev || !out_ids || !out_dists || nq < 0)
+    return set_error(ALGAS_EINVAL, "algas_search_dynamic: null argument");
+  if (!is_device_ptr(queries_dev)) return set_error(ALGAS_EINVAL, "algas_search_dynamic: queries must be device memory");
+  if (nq == 0) return ALGAS_OK;
+  if (nq >= (1LL << 31)) return set_error(ALGAS_EINVAL, "nq too large");
+  if (params->visited_mode != ALGAS_VISITED_PRIVATE)
+    return set_error(ALGAS_EINVAL, "algas_search_dynamic: SHARED visited mode not implemented yet");
+  const int slots = params->slots > 0 ? params->slots : 32;
+  Plan pl;
+  int rc = make_plan(idx, params, slots, &pl, true);
+  if (rc) return rc;
+  if ((int64_t)slots * pl.T > (int64_t)pl.blocks_per_sm * num_sms())
+    return set_error(ALGAS_EINVAL, "%d slots x %d CTAs exceed co-resident capacity %d x %d SMs (P:L231)", slots, pl.T,
+                     pl.blocks_per_sm, num_sms());
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const int ctas = slots * pl.T;
+  const int64_t items = nq * pl.T;
+
+  std::lock_guard<std::mutex> lk(idx->ws->mu);
+  if ((rc = ensure_gtab(idx, (size_t)ctas << pl.cfg.gtab_bits))) return rc;
+  // per-CTA tables restart at epoch 1 for this launch: clear the used region
+  ALGAS_CUDA_TRY(cudaMemsetAsync(idx->ws->gtab, 0, ((size_t)ctas << pl.cfg.gtab_bits) * 8, st));
+  idx->ws->epoch = 1;
+
+  DevBuf rb, sb, ctl;
+  if ((rc = rb.alloc((size_t)items * pl.k * sizeof(ResultEntry), st))) return rc;
+  if ((rc = sb.alloc((size_t)items * sizeof(CtaStats), st))) return rc;
+  // control block: queue head | mbox[slots] | dparams[slots] | dtag[slots] | slot_fin[slots] | qbuf unused
+  const size_t ctl_bytes = control_bytes(slots);
+  if ((rc = ctl.alloc(ctl_bytes, st))) return rc;
+  ALGAS_CUDA_TRY(cudaMemsetAsync(ctl.p, 0, ctl_bytes, st));
+  uint8_t* cb = (uint8_t*)ctl.p;
+  PersistArgs pa;
+  memset(&pa, 0, sizeof(pa));
+  pa.mode = 1;
+  pa.slots = slots;
+  pa.T = pl.T;
+  pa.kmax = pl.k;
+  pa.queries = reinterpret_cast<const float4*>(queries_dev);
+  pa.nq = nq;
+  pa.tag0 = tag0;
+  carve_control(cb, slots, &pa);
+  pa.dq_res = (ResultEntry*)rb.p;
+  pa.dq_stats = (CtaStats*)sb.p;
+  pa.gtab = idx->ws->gtab;
+  pa.epoch_base = 1;
+  EventTimer tm(st);
+  if ((rc = tm.start())) return rc;
+  if ((rc = launch_persistent(pl, pa, st))) return rc;
+  if ((rc = tm.stop())) return rc;
+  std::vector<ResultEntry> res((size_t)items * pl.k);
+  std::vector<CtaStats> cst((size_t)items);
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(res.data(), rb.p, res.size() * sizeof(ResultEntry), cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst.data(), sb.p, cst.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaStreamSynchronize(st));
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  if (info) fill_info(info, pl, ctas, tm.ms());
+  bool ovf = false;
+  if ((rc = finish_outputs(res, cst, nq, pl.T, pl.k, pl.k, out_ids, out_dists, nullptr, nullptr, out_stats, &ovf)))
+    return rc;
+  return ovf ? set_error(ALGAS_EOVERFLOW, "a visited table overflowed") : ALGAS_OK;
+}
+
+}  // extern "C"

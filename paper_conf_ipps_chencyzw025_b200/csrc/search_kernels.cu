@@ -1,0 +1,341 @@
+// search_kernels.cu -- the batch (static) and persistent (dynamic batching)
+// search kernels and their launchers.
+//
+//  batch_kernel      : static batching -- one launch over nq queries,
+//                      each CTA pulls (query, cta_rank) work items from an
+//                      atomic counter until the batch is drained.
+//  persistent_kernel : dynamic batching -- grid = slots x T
+//                      CTAs that never exit; each slot's rank-0 CTA polls for
+//                      work (host-mapped ring: "The CTAs in the slot
+//                      poll the state", or an HBM query queue), publishes it
+//                      through a device mailbox to the slot's other CTAs,
+//                      and every CTA publishes its own top-k + a Finish flag
+//                      (P:L170).
+#include <cooperative_groups.h>
+
+#include "internal.h"
+
+namespace algas {
+
+// ------------------------------------------------------------------ memory-order helpers
+__device__ __forceinline__ uint32_t ld_acquire_sys(const volatile uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_gpu64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned int ld_acquire_gpu32(const unsigned int* p) {
+  unsigned int v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ float4 ld_volatile_f4(const float4* p) {
+  float4 r;
+  asm volatile("ld.volatile.global.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p)
+               : "memory");
+  return r;
+}
+
+// ------------------------------------------------------------------ static batch kernel
+struct BatchArgs {
+  SearchCfg cfg;
+  const float4* queries;
+  int64_t nq;
+  int32_t T, k;
+  uint64_t tag0;
+  int* work_counter;
+  ResultEntry* res;
+  CtaStats* stats;
+  unsigned long long* gtab;
+  uint32_t epoch_base;
+};
+
+template <int NT, int TL, int CPL, int METRIC>
+__global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  const SmemLayout lay = smem_layout(a.cfg.d4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits);
+  const Smem s = carve(smem_raw, lay);
+  __shared__ int s_item;
+  const int64_t total = a.nq * a.T;
+  unsigned long long* gt = a.gtab ? a.gtab + ((uint64_t)blockIdx.x << a.cfg.gtab_bits) : nullptr;
+  for (;;) {
+    if (threadIdx.x == 0) s_item = atomicAdd(a.work_counter, 1);
+    __syncthreads();
+    const int64_t item = s_item;
+    if (item >= total) break;
+    const int64_t qi = item / a.T;
+    const int c = (int)(item - qi * a.T);
+    const float4* qsrc = a.queries + qi * a.cfg.d4;
+    for (int i = threadIdx.x; i < a.cfg.d4; i += NT) s.q[i] = qsrc[i];
+    __syncthreads();
+    CtaStats* st = a.stats ? a.stats + item : nullptr;
+    search_cta<NT, TL, CPL, METRIC>(a.cfg, s, a.tag0 + (uint64_t)qi, (uint32_t)c, a.k, gt,
+                                    a.epoch_base + (uint32_t)item, a.res + item * a.k, st);
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------------ persistent kernel
+struct PKArgs {
+  SearchCfg cfg;
+  PersistArgs p;
+};
+
+constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
+
+template <int NT, int TL, int CPL, int METRIC>
+__global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  const SmemLayout lay = smem_layout(A.cfg.d4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits);
+  const Smem s = carve(smem_raw, lay);
+  const PersistArgs& P = A.p;
+  const int slot = blockIdx.x / P.T;
+  const int rank = blockIdx.x % P.T;
+  const int tid = threadIdx.x;
+  unsigned long long* gt = P.gtab ? P.gtab + ((uint64_t)blockIdx.x << A.cfg.gtab_bits) : nullptr;
+  __shared__ unsigned long long s_mbox;
+  __shared__ int4 s_par;
+  __shared__ unsigned long long s_tag, s_t0;
+  uint32_t served = 0;  // queries this CTA has finished (= last epoch in devq mode)
+  uint32_t last_epoch = 0;
+
+  for (;;) {
+    // ---------------- acquire work (rank 0) and publish it to the slot's CTAs
+    if (rank == 0) {
+      if (tid == 0) {
+        unsigned long long mb;
+        if (P.mode == 0) {
+          // host ring: poll the slot state in host memory
+          uint32_t st;
+          unsigned ns = 64;
+          for (;;) {
+            st = ld_acquire_sys(&P.ring[slot].state);
+            uint32_t kind = st & 0xFFu, ep = st >> 8;
+            if (kind == kSlotQuit) break;
+            if (kind == kSlotReady && ep != last_epoch) break;
+            __nanosleep(ns);
+            if (ns < 1024) ns <<= 1;
+          }
+          if ((st & 0xFFu) == kSlotQuit) {
+            mb = kMboxQuit;
+          } else {
+            const uint32_t ep = st >> 8;
+            // payload: params + query from mapped memory (volatile: never a stale line)
+            const volatile RingSlot* rs = &P.ring[slot];
+            int4 par = make_int4(rs->k, rs->L, rs->w, 0);
+            unsigned long long tag = rs->tag;
+            P.dparams[slot] = par;
+            P.dtag[slot] = tag;
+            mb = ((unsigned long long)ep << 32) | (unsigned long long)slot;
+          }
+        } else {
+          // device queue: wait until every CTA of the slot finished the previous query
+          while (ld_acquire_gpu32(P.slot_fin + slot) < (unsigned)(served * P.T)) __nanosleep(32);
+          int item = atomicAdd(P.queue_head, 1);
+          if (item >= P.nq) {
+            mb = kMboxQuit;
+          } else {
+            const uint32_t ep = served + 1;
+            P.dparams[slot] = make_int4(P.kmax, A.cfg.L, A.cfg.w, 0);
+            P.dtag[slot] = P.tag0 + (uint64_t)item;
+            mb = ((unsigned long long)ep << 32) | (unsigned long long)(uint32_t)item;
+          }
+        }
+        s_mbox = mb;
+        s_t0 = globaltimer();
+      }
+      __syncthreads();
+      if (s_mbox != kMboxQuit && P.mode == 0) {
+        // stage the query from host memory into the slot's HBM buffer (one PCIe read)
+        const float4* src = P.ring_q + (uint64_t)slot * A.cfg.d4;
+        float4* dst = P.qbuf + (uint64_t)slot * A.cfg.d4;
+        for (int i = tid; i < A.cfg.d4; i += NT) dst[i] = ld_volatile_f4(src + i);
+      }
+      __syncthreads();
+      if (tid == 0) {
+        __threadfence();
+        st_release_gpu64(P.mbox + slot, s_mbox);
+      }
+    } else {
+      if (tid == 0) {
+        unsigned long long mb;
+        for (;;) {
+          mb = ld_acquire_gpu64(P.mbox + slot);
+          if (mb == kMboxQuit) break;
+          if ((uint32_t)(mb >> 32) != last_epoch && (uint32_t)(mb >> 32) != 0u) break;
+          __nanosleep(32);
+        }
+        s_mbox = mb;
+        s_t0 = globaltimer();
+      }
+      __syncthreads();
+    }
+    const unsigned long long mb = s_mbox;
+    if (mb == kMboxQuit) break;
+    const uint32_t epoch = (uint32_t)(mb >> 32);
+    const uint32_t item = (uint32_t)mb;
+    if (tid == 0) {
+      const volatile int* vp = reinterpret_cast<const volatile int*>(P.dparams + slot);
+      s_par = make_int4(vp[0], vp[1], vp[2], vp[3]);
+      s_tag = *((volatile unsigned long long*)(P.dtag + slot));
+    }
+    __syncthreads();
+    const int4 par = s_par;
+    const uint64_t tag = s_tag;
+
+    // ---------------- stage the query into shared memory
+    const float4* qsrc = (P.mode == 0) ? P.qbuf + (uint64_t)slot * A.cfg.d4
+                                       : P.queries + (uint64_t)item * A.cfg.d4;
+    for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = (P.mode == 0) ? ld_volatile_f4(qsrc + i) : qsrc[i];
+    __syncthreads();
+
+    SearchCfg cfg = A.cfg;
+    cfg.L = par.y;
+    cfg.w = par.z;
+    if (cfg.off > cfg.L) cfg.off = cfg.L;
+    const int k = par.x;
+    ResultEntry* out;
+    CtaStats* stp;
+    if (P.mode == 0) {
+      out = P.ring_res + ((uint64_t)slot * P.T + rank) * P.kmax;
+      stp = P.ring_stats + (uint64_t)slot * P.T + rank;
+    } else {
+      out = P.dq_res + ((uint64_t)item * P.T + rank) * P.kmax;
+      stp = P.dq_stats + (uint64_t)item * P.T + rank;
+    }
+    CtaStats local;
+    search_cta<NT, TL, CPL, METRIC>(cfg, s, tag, (uint32_t)rank, k, gt,
+                                    P.epoch_base + served, out, &local);
+    __syncthreads();
+    if (tid == 0) {
+      local.t_start = s_t0;
+      local.t_end = globaltimer();
+      *stp = local;
+    }
+    served++;
+    last_epoch = epoch;
+    __syncthreads();
+    // ---------------- Finish
+    if (tid == 0) {
+      if (P.mode == 0) {
+        __threadfence_system();
+        st_release_sys(P.ring_done + (uint64_t)slot * P.T + rank, epoch);
+      } else {
+        __threadfence();
+        atomicAdd(P.slot_fin + slot, 1u);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ dispatch
+template <int NT, int TL, int CPL, int M>
+struct KSel {
+  static void* batch() { return (void*)batch_kernel<NT, TL, CPL, M>; }
+  static void* persist() { return (void*)persistent_kernel<NT, TL, CPL, M>; }
+};
+
+// chunk configs: (TL lanes per vector, CPL float4 chunks per lane)
+//   0:(8,3) d4<=24   1:(8,4) d4<=32   2:(16,4) d4<=64
+//   3:(32,4) d4<=128 4:(32,8) d4<=256 5:(32,16) d4<=512
+int chunk_config_for(int d4) {
+  if (d4 <= 24) return 0;
+  if (d4 <= 32) return 1;
+  if (d4 <= 64) return 2;
+  if (d4 <= 128) return 3;
+  if (d4 <= 256) return 4;
+  if (d4 <= 512) return 5;
+  return -1;
+}
+
+template <int NT, int M>
+static void* pick_cc(int cc, bool persist) {
+  switch (cc) {
+    case 0: return persist ? KSel<NT, 8, 3, M>::persist() : KSel<NT, 8, 3, M>::batch();
+    case 1: return persist ? KSel<NT, 8, 4, M>::persist() : KSel<NT, 8, 4, M>::batch();
+    case 2: return persist ? KSel<NT, 16, 4, M>::persist() : KSel<NT, 16, 4, M>::batch();
+    case 3: return persist ? KSel<NT, 32, 4, M>::persist() : KSel<NT, 32, 4, M>::batch();
+    case 4: return persist ? KSel<NT, 32, 8, M>::persist() : KSel<NT, 32, 8, M>::batch();
+    case 5: return persist ? KSel<NT, 32, 16, M>::persist() : KSel<NT, 32, 16, M>::batch();
+  }
+  return nullptr;
+}
+template <int NT>
+static void* pick_metric(int metric, int cc, bool persist) {
+  return metric == kL2 ? pick_cc<NT, kL2>(cc, persist) : pick_cc<NT, kIP>(cc, persist);
+}
+static void* kernel_for(const Plan& pl, int metric, bool persist) {
+  switch (pl.nt) {
+    case 32: return pick_metric<32>(metric, pl.ccfg, persist);
+    case 64: return pick_metric<64>(metric, pl.ccfg, persist);
+    case 128: return pick_metric<128>(metric, pl.ccfg, persist);
+    case 256: return pick_metric<256>(metric, pl.ccfg, persist);
+  }
+  return nullptr;
+}
+
+int max_blocks_per_sm(const Plan& pl, bool persistent, int* out) {
+  void* fn = kernel_for(pl, pl.metric, persistent);
+  if (!fn) return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d", pl.nt, pl.ccfg);
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
+  int nb = 0;
+  ALGAS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, pl.nt, pl.smem));
+  *out = nb;
+  return ALGAS_OK;
+}
+
+int launch_batch(const Plan& pl, const BatchLaunch& bl, cudaStream_t st) {
+  void* fn = kernel_for(pl, pl.metric, false);
+  if (!fn) return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d", pl.nt, pl.ccfg);
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
+  BatchArgs a;
+  a.cfg = pl.cfg;
+  a.queries = bl.queries;
+  a.nq = bl.nq;
+  a.T = pl.T;
+  a.k = pl.k;
+  a.tag0 = bl.tag0;
+  a.work_counter = bl.work_counter;
+  a.res = bl.res;
+  a.stats = bl.stats;
+  a.gtab = bl.gtab;
+  a.epoch_base = bl.epoch_base;
+  ALGAS_CUDA_TRY(cudaMemsetAsync(bl.work_counter, 0, sizeof(int), st));
+  void* args[] = {&a};
+  ALGAS_CUDA_TRY(cudaLaunchKernel(fn, dim3(bl.grid), dim3(pl.nt), args, pl.smem, st));
+  return ALGAS_OK;
+}
+
+int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st) {
+  void* fn = kernel_for(pl, pl.metric, true);
+  if (!fn) return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d", pl.nt, pl.ccfg);
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
+  PKArgs A;
+  A.cfg = pl.cfg;
+  A.p = pa;
+  void* args[] = {&A};
+  // cooperative launch: the runtime refuses a grid that cannot be fully
+  // co-resident, which a persistent kernel needs for forward progress
+  cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(pa.slots * pa.T), dim3(pl.nt), args, pl.smem, st);
+  if (e != cudaSuccess) {
+    (void)cudaGetLastError();
+    return set_error(e == cudaErrorCooperativeLaunchTooLarge ? ALGAS_EINVAL : ALGAS_ECUDA,
+                     "persistent launch (%d slots x %d CTAs x %d threads, %d B smem) failed: %s", pa.slots,
+                     pa.T, pl.nt, pl.smem, cudaGetErrorString(e));
+  }
+  return ALGAS_OK;
+}
+
+}  // namespace algas

@@ -1,0 +1,119 @@
+"""CPU-side checks of the C-ABI library: it loads without a GPU, exports every
+symbol include/algas.h declares, and its host-only logic (host TopK merge,
+tuning equations, tuner policy, argument validation) matches the oracle /
+the paper's closed forms.  No compute calls that need a GPU."""
+import json
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_chencyzw025_b200 as algas
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared_functions():
+    src = open(os.path.join(ROOT, "include", "algas.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(algas_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    L = algas.lib()
+    declared = _declared_functions()
+    assert len(declared) >= 20
+    for name in declared:
+        assert hasattr(L, name), f"{name} declared in algas.h but not exported"
+    assert sorted(algas.EXPORTS) == declared
+
+
+def test_version_and_defaults():
+    assert b"sm_100a" in algas.lib().algas_version()
+    p = algas.default_params()
+    assert (p.k, p.itopk, p.width, p.offset_beam, p.n_seeds, p.slots) == (10, 64, 1, -1, 32, 32)
+
+
+def test_host_merge_matches_oracle_merge():
+    rng = np.random.default_rng(3)
+    for _ in range(200):
+        m = int(rng.integers(0, 80))
+        ids = rng.integers(0, 40, size=m).astype(np.uint32)
+        ids[rng.random(m) < 0.1] = algas.SENTINEL
+        table = rng.integers(0, 8, size=40).astype(np.float32)
+        ds = np.where(ids == algas.SENTINEL, np.float32(np.inf), table[np.minimum(ids, 39)]).astype(np.float32)
+        k = int(rng.integers(1, 16))
+        a = algas.merge_topk(ids, ds, k)
+        b = oracle.merge_topk(ids, ds, k)
+        np.testing.assert_array_equal(a[0], b[0])
+        np.testing.assert_array_equal(a[1], b[1])
+        assert a[2] == b[2]
+
+
+def test_tuner_equations_match_oracle_and_table2():
+    L = algas.lib()
+    g = json.load(open(os.path.join(ROOT, "tests", "golden", "table2_tuner.json")))
+    a = g["a6000"]
+    for w in g["worked"]:
+        if "expect_max_parallel" in w:
+            assert L.algas_tuner_max_parallel(w["slots"], a["n_sm"], a["max_blocks_per_sm"]) == w["expect_max_parallel"]
+        if "expect_blocks_per_sm" in w:
+            assert L.algas_tuner_blocks_per_sm(w["n_parallel"], w["slots"], a["n_sm"]) == w["expect_blocks_per_sm"]
+        if "expect_smem_per_block" in w:
+            assert L.algas_tuner_smem_per_block(a["shared_mem_per_sm_bytes"], w["blocks_per_sm"],
+                                                a["reserved_shared_mem_per_block_bytes"]) == w["expect_smem_per_block"]
+    rng = np.random.default_rng(0)
+    for _ in range(300):
+        slots, nsm, mb = int(rng.integers(1, 64)), int(rng.integers(1, 200)), int(rng.integers(1, 33))
+        assert L.algas_tuner_max_parallel(slots, nsm, mb) == oracle.tuner_max_parallel(slots, nsm, mb)
+        npar = int(rng.integers(1, 64))
+        assert L.algas_tuner_blocks_per_sm(npar, slots, nsm) == oracle.tuner_blocks_per_sm(npar, slots, nsm)
+        m, b, r = int(rng.integers(1, 300000)), int(rng.integers(1, 33)), int(rng.integers(0, 4096))
+        assert L.algas_tuner_smem_per_block(m, b, r) == oracle.tuner_smem_per_block(m, b, r)
+
+
+def _b200_props():
+    p = algas.DeviceProps()
+    p.n_sm, p.max_blocks_per_sm = 148, 32
+    p.smem_per_sm, p.smem_reserved_per_block, p.smem_per_block_optin = 233472, 1024, 232448
+    p.max_threads_per_sm, p.regs_per_sm = 2048, 65536
+    return p
+
+
+def _a6000_props():
+    p = algas.DeviceProps()
+    p.n_sm, p.max_blocks_per_sm = 84, 16
+    p.smem_per_sm, p.smem_reserved_per_block, p.smem_per_block_optin = 102400, 1024, 101376
+    p.max_threads_per_sm, p.regs_per_sm = 1536, 65536
+    return p
+
+
+@pytest.mark.parametrize("props", [_b200_props(), _a6000_props()])
+@pytest.mark.parametrize("slots", [1, 8, 16, 32])
+def test_tuner_policy_respects_paper_constraints(props, slots):
+    for dim, L in [(128, 64), (960, 128), (100, 256), (96, 64)]:
+        t = algas.tune(slots, dim, 64, L, 10, props=props)
+        # all slots' CTAs co-resident
+        assert t.ctas_per_query * slots <= props.n_sm * props.max_blocks_per_sm
+        # P:L235
+        assert t.blocks_per_sm == oracle.tuner_blocks_per_sm(t.ctas_per_query, slots, props.n_sm)
+        # P:L245 with M_reserved >= the driver reservation
+        assert t.smem_per_block <= t.smem_avail_per_block
+        assert t.smem_avail_per_block <= oracle.tuner_smem_per_block(props.smem_per_sm, t.blocks_per_sm,
+                                                                     props.smem_reserved_per_block)
+        assert t.threads_per_cta in (32, 64, 128, 256)
+        assert 1 <= t.width <= 32 and 1 <= t.offset_beam <= L
+
+
+def test_tuner_small_batch_gets_more_ctas():
+    props = _b200_props()
+    t1 = algas.tune(1, 128, 64, 64, 10, props=props)
+    t32 = algas.tune(32, 128, 64, 64, 10, props=props)
+    assert t1.ctas_per_query >= t32.ctas_per_query
+
+
+def test_merge_rejects_bad_arguments():
+    with pytest.raises(algas.AlgasError):
+        algas.merge_topk(np.zeros(3, np.uint32), np.zeros(3, np.float32), 0)

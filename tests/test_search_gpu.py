@@ -1,0 +1,302 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle on the
+same seeded inputs.
+
+  * integer-lattice data: fp32 sums are exact in any order, so the GPU must
+    reproduce the oracle bit for bit -- ids, distance bits, and the per-query
+    step / parent / distance-evaluation counters (exact-trajectory parity)
+  * float data: recall@k no lower than the oracle's minus 0.005 at identical
+    parameters (BASELINE.json north_star), every returned distance within
+    1e-5 (magnitude-scaled for IP) of an fp64 recomputation, sorted, unique
+  * batch invariance: static batch == dynamic (HBM queue) == persistent
+    server, bitwise, for any slot count / arrival order
+"""
+import time
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_chencyzw025_b200 as algas
+import synth
+
+pytestmark = pytest.mark.gpu
+SENT = algas.SENTINEL
+
+
+def _bits(a):
+    """fp32 bit pattern with -0.0 folded onto +0.0 (the two compare equal, R4)."""
+    return (np.asarray(a, np.float32) + np.float32(0.0)).view(np.uint32)
+
+
+def _torch_cuda(a):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+# ------------------------------------------------------------------ fixtures
+_cache = {}
+
+
+def lattice_case(n, d, metric, R, seed):
+    key = ("lat", n, d, metric, R, seed)
+    if key not in _cache:
+        X = synth.lattice(n, d, seed=seed, metric=metric)
+        Q = synth.lattice(37, d, seed=seed + 1, metric=metric)
+        G, _ = oracle.knn_graph(X, R, metric)
+        _cache[key] = (X, Q, G)
+    return _cache[key]
+
+
+def float_case():
+    key = "C1"
+    if key not in _cache:
+        w = synth.WORKLOADS["C1"]
+        X = synth.base_vectors(w)
+        Q = synth.query_vectors(w)
+        G, _ = oracle.knn_graph(X, w.degree)
+        ti, td = oracle.brute_force(X, Q, 10)
+        _cache[key] = (X, Q, G, ti, td)
+    return _cache[key]
+
+
+def _oracle_params(p: algas.Params):
+    L = p.itopk
+    off = p.offset_beam if p.offset_beam >= 0 else max(1, L // 4)
+    return oracle.make_params(k=p.k, L=L, w=p.width, off=min(off, L), T=p.ctas_per_query,
+                              S=p.n_seeds, max_iter=p.max_iter if p.max_iter > 0 else 4 * L + 256,
+                              shared_visited=0, seed=p.seed)
+
+
+def _check_invariants(X, Q, ids, ds, metric, k):
+    for t in range(Q.shape[0]):
+        real = [int(i) for i in ids[t] if i != SENT]
+        assert len(real) == len(set(real)), "duplicate ids"
+        assert all(0 <= i < X.shape[0] for i in real)
+        n = len(real)
+        assert np.all(ids[t, n:] == SENT) and np.all(np.isinf(ds[t, n:]))
+        assert np.all(np.diff(ds[t, :n]) >= 0), "not sorted"
+        x = X[real].astype(np.float64)
+        q = Q[t].astype(np.float64)
+        if metric == algas.L2:
+            ref = ((x - q) ** 2).sum(1)
+            scale = ref
+        else:
+            ref = -(x * q).sum(1)
+            scale = np.abs(x * q).sum(1)
+        assert np.all(np.abs(ds[t, :n] - ref) <= 1e-5 * scale + 1e-30), "distance tolerance"
+
+
+# ------------------------------------------------------------------ K9 brute force
+@pytest.mark.parametrize("metric", [algas.L2, algas.IP])
+@pytest.mark.parametrize("d", [16, 128])
+def test_knn_lattice_bit_exact(metric, d):
+    X = synth.lattice(3001, d, seed=5, metric=metric)
+    Q = synth.lattice(77, d, seed=6, metric=metric)
+    gi, gd = algas.knn(X, Q, 33, metric)
+    oi, od = oracle.brute_force(X, Q, 33, metric)
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(_bits(gd), _bits(od))
+
+
+def test_knn_self_exclusion_and_chunking():
+    # more base points than one 65536-column chunk, rows not a multiple of any tile
+    X = synth.lattice(70001, 8, seed=7)
+    gi, gd = algas.knn(X, X[:50], 10, algas.L2, self_base=0)
+    oi, od = oracle.brute_force(X, X[:50], 10, oracle.L2, self_base=0)
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(gd, od)
+
+
+def test_knn_float_modulo_ties():
+    X = synth.uniform(5000, 100, seed=8)
+    Q = synth.uniform(64, 100, seed=9)
+    gi, gd = algas.knn(X, Q, 20, algas.L2)
+    oi, od = oracle.brute_force(X, Q, 20, oracle.L2)
+    d64 = ((Q[:, None, :].astype(np.float64) - X[None].astype(np.float64)) ** 2).sum(-1)
+    for r in range(Q.shape[0]):
+        kth = d64[r, oi[r, -1]]
+        if set(gi[r].tolist()) != set(oi[r].tolist()):
+            # only points within the tolerance of the k-th distance may differ
+            for i in set(gi[r].tolist()) ^ set(oi[r].tolist()):
+                assert abs(d64[r, i] - kth) <= 1e-5 * kth
+        np.testing.assert_allclose(gd[r], d64[r, gi[r]], rtol=1e-5)
+
+
+def test_knn_k_exceeds_n_padding():
+    X = synth.uniform(7, 8, seed=1)
+    gi, gd = algas.knn(X, X[:2], 9, algas.L2, self_base=0)
+    assert np.all(gi[:, 6:] == SENT) and np.all(np.isinf(gd[:, 6:]))
+
+
+# ------------------------------------------------------------------ K10 prune
+@pytest.mark.parametrize("K,R", [(32, 16), (64, 32), (16, 16), (24, 7)])
+def test_prune_bit_exact(K, R):
+    X = synth.lattice(1500, 16, seed=11)
+    knn, _ = oracle.knn_graph(X, K)
+    np.testing.assert_array_equal(algas.prune(knn, R), oracle.prune(knn, R))
+
+
+def test_build_graph_matches_oracle_pipeline():
+    X = synth.lattice(1200, 32, seed=12)
+    g = algas.build_graph(X, 16, knn_degree=32, prune=True)
+    knn, _ = oracle.knn_graph(X, 32)
+    np.testing.assert_array_equal(g, oracle.prune(knn, 16))
+    g2 = algas.build_graph(X, 16, knn_degree=32, prune=False)
+    np.testing.assert_array_equal(g2, knn[:, :16])
+
+
+# ------------------------------------------------------------------ search: exact trajectory
+LATTICE_CASES = [
+    # n, d, metric, R, params
+    (2000, 32, algas.L2, 16, dict(k=10, itopk=16, width=1, n_seeds=4, ctas_per_query=1)),
+    (2000, 32, algas.L2, 16, dict(k=10, itopk=32, width=4, offset_beam=8, n_seeds=8, ctas_per_query=1)),
+    (2000, 128, algas.L2, 32, dict(k=10, itopk=64, width=2, offset_beam=16, n_seeds=32, ctas_per_query=1)),
+    (2000, 128, algas.L2, 32, dict(k=10, itopk=64, width=4, offset_beam=0, n_seeds=32, ctas_per_query=3)),
+    (2000, 96, algas.L2, 32, dict(k=16, itopk=128, width=8, offset_beam=32, n_seeds=16, ctas_per_query=2)),
+    (2000, 100, algas.IP, 32, dict(k=10, itopk=48, width=2, offset_beam=12, n_seeds=32, ctas_per_query=1)),
+    (2000, 960, algas.L2, 20, dict(k=10, itopk=32, width=2, offset_beam=8, n_seeds=8, ctas_per_query=1)),
+    (1500, 256, algas.IP, 24, dict(k=5, itopk=5, width=1, n_seeds=1, ctas_per_query=4)),
+]
+
+
+@pytest.mark.parametrize("case", range(len(LATTICE_CASES)))
+@pytest.mark.parametrize("threads", [32, 64, 128, 256])
+def test_search_lattice_exact_trajectory(case, threads):
+    n, d, metric, R, kw = LATTICE_CASES[case]
+    X, Q, G = lattice_case(n, d, metric, R, seed=100 + case)
+    p = algas.default_params(threads_per_cta=threads, seed=7, **kw)
+    idx = algas.Index(X, G, metric)
+    r = idx.search(Q, params=p, tag0=11, want_cta=True)
+    oi, od, ost, oci, ocd = oracle.search(X, G, Q, _oracle_params(p), metric=metric, tag0=11, want_cta=True)
+    np.testing.assert_array_equal(r["cta_ids"], oci)
+    np.testing.assert_array_equal(_bits(r["cta_dists"]), _bits(ocd))
+    np.testing.assert_array_equal(r["ids"], oi)
+    np.testing.assert_array_equal(_bits(r["dists"]), _bits(od))
+    st = r["stats"]
+    np.testing.assert_array_equal(st["iters"].astype(np.int64), ost["iters"])
+    np.testing.assert_array_equal(st["parents"].astype(np.int64), ost["parents"])
+    np.testing.assert_array_equal(st["dist_evals"].astype(np.int64), ost["dist_evals"])
+    np.testing.assert_array_equal(st["max_iters"].astype(np.int64), ost["max_iters"])
+    assert (st["cap_hits"] == 0).all() and (st["overflows"] == 0).all()
+    _check_invariants(X, Q, r["ids"], r["dists"], metric, p.k)
+
+
+def test_search_spill_to_hbm_is_exact():
+    """A tiny shared-memory hash forces the HBM spill table; results stay exact."""
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=200)
+    p = algas.default_params(k=10, itopk=128, width=4, offset_beam=16, n_seeds=8, ctas_per_query=1,
+                             threads_per_cta=64, hash_bits=8)
+    r = algas.Index(X, G).search(Q, params=p)
+    assert (r["stats"]["spills"] > 0).any()
+    oi, od, ost = oracle.search(X, G, Q, _oracle_params(p))
+    np.testing.assert_array_equal(r["ids"], oi)
+    np.testing.assert_array_equal(r["stats"]["dist_evals"].astype(np.int64), ost["dist_evals"])
+
+
+def test_search_max_iter_cap_counted():
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=201)
+    p = algas.default_params(k=10, itopk=32, n_seeds=4, ctas_per_query=1, max_iter=3, threads_per_cta=64)
+    r = algas.Index(X, G).search(Q, params=p)
+    oi, od, ost = oracle.search(X, G, Q, _oracle_params(p))
+    np.testing.assert_array_equal(r["ids"], oi)
+    assert (r["stats"]["iters"] == 3).all() and (r["stats"]["cap_hits"] == ost["cap_hits"]).all()
+
+
+def test_search_degenerate_inputs():
+    # n smaller than k and the seed count; graph rows full of sentinels
+    X = synth.lattice(6, 8, seed=3)
+    G = np.full((6, 4), SENT, np.uint32)
+    G[0, :2] = [1, 2]
+    Q = synth.lattice(5, 8, seed=4)
+    p = algas.default_params(k=8, itopk=8, n_seeds=32, ctas_per_query=2, threads_per_cta=32)
+    r = algas.Index(X, G).search(Q, params=p)
+    oi, od, ost = oracle.search(X, G, Q, _oracle_params(p))
+    np.testing.assert_array_equal(r["ids"], oi)
+    np.testing.assert_array_equal(r["dists"], od)
+    # empty batch
+    e = algas.Index(X, G).search(Q[:0], params=p)
+    assert e["ids"].shape == (0, 8)
+
+
+def test_search_rejects_bad_params():
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=202)
+    idx = algas.Index(X, G)
+    for kw in (dict(k=0), dict(k=20, itopk=10), dict(itopk=1024), dict(width=0), dict(width=64),
+               dict(ctas_per_query=100), dict(threads_per_cta=48), dict(n_seeds=1000)):
+        with pytest.raises(algas.AlgasError):
+            idx.search(Q, params=algas.default_params(**kw))
+
+
+# ------------------------------------------------------------------ search: float recall parity
+@pytest.mark.parametrize("kw", [dict(itopk=32, width=1), dict(itopk=64, width=4, offset_beam=16),
+                                dict(itopk=128, width=4, offset_beam=32, ctas_per_query=4)])
+def test_search_float_recall_parity_C1(kw):
+    X, Q, G, ti, td = float_case()
+    p = algas.default_params(k=10, n_seeds=32, seed=3, **({"ctas_per_query": 1} | kw))
+    r = algas.Index(X, G).search(Q, params=p)
+    oi, od, ost = oracle.search(X, G, Q, _oracle_params(p))
+    rg, ro = oracle.recall(r["ids"], ti, 10), oracle.recall(oi, ti, 10)
+    assert rg >= ro - 0.005, (rg, ro)
+    _check_invariants(X, Q, r["ids"], r["dists"], algas.L2, 10)
+
+
+# ------------------------------------------------------------------ batch invariance
+@pytest.mark.parametrize("slots,T", [(1, 1), (4, 2), (32, 1), (7, 3)])
+def test_dynamic_queue_equals_batch(slots, T):
+    X, Q, G = lattice_case(2000, 128, algas.L2, 32, seed=300)
+    p = algas.default_params(k=10, itopk=48, width=2, offset_beam=8, n_seeds=16, ctas_per_query=T,
+                             threads_per_cta=64, slots=slots, seed=5)
+    idx = algas.Index(X, G)
+    b = idx.search(Q, params=p, tag0=1000)
+    dq = _torch_cuda(Q)
+    d = idx.search_dynamic(dq, p, tag0=1000)
+    np.testing.assert_array_equal(d["ids"], b["ids"])
+    np.testing.assert_array_equal(_bits(d["dists"]), _bits(b["dists"]))
+    np.testing.assert_array_equal(d["stats"]["iters"], b["stats"]["iters"])
+    assert (d["stats"]["t_end_ns"] >= d["stats"]["t_start_ns"]).all()
+
+
+@pytest.mark.parametrize("slots,T", [(1, 1), (8, 2), (32, 1)])
+def test_server_equals_batch(slots, T):
+    X, Q, G = lattice_case(2000, 128, algas.L2, 32, seed=301)
+    p = algas.default_params(k=10, itopk=48, width=2, offset_beam=8, n_seeds=16, ctas_per_query=T,
+                             threads_per_cta=64, slots=slots, seed=5)
+    idx = algas.Index(X, G)
+    b = idx.search(Q, params=p, tag0=0)
+    rng = np.random.default_rng(slots)
+    order = rng.permutation(Q.shape[0])
+    got = {}
+    with algas.Server(idx, p) as srv:
+        pending = list(order)
+        t0 = time.time()
+        while (pending or srv.inflight() > 0) and time.time() - t0 < 60:
+            while pending and srv.submit(Q[pending[0]], tag=int(pending[0])):
+                pending.pop(0)
+            tags, ids, ds, st = srv.poll(64)
+            for t, i, dd in zip(tags, ids, ds):
+                assert int(t) not in got, "a tag completed twice"
+                got[int(t)] = (i.copy(), dd.copy())
+    assert len(got) == Q.shape[0]
+    for t in range(Q.shape[0]):
+        np.testing.assert_array_equal(got[t][0], b["ids"][t])
+        np.testing.assert_array_equal(_bits(got[t][1]), _bits(b["dists"][t]))
+
+
+def test_server_smaller_per_query_params_and_rejects():
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=302)
+    p = algas.default_params(k=10, itopk=64, width=4, n_seeds=8, ctas_per_query=1, threads_per_cta=64, slots=4)
+    idx = algas.Index(X, G)
+    with algas.Server(idx, p) as srv:
+        assert srv.submit(Q[0], tag=1, k=5, itopk=16, width=1)
+        with pytest.raises(algas.AlgasError):
+            srv.submit(Q[1], tag=2, k=20)
+        t0 = time.time()
+        out = []
+        while not out and time.time() - t0 < 30:
+            out = list(zip(*srv.poll(4)))
+    assert len(out) == 1
+    tag, ids, ds, st = out[0]
+    p5 = algas.default_params(k=5, itopk=16, width=1, n_seeds=8, ctas_per_query=1, threads_per_cta=64)
+    b = idx.search(Q[:1], params=p5, tag0=1)
+    np.testing.assert_array_equal(ids[:5], b["ids"][0])
+    assert np.all(ids[5:] == SENT)
