@@ -1,0 +1,430 @@
+"""bench.py -- ALGAS hot path on B200: QPS and p50/p99 latency at recall@10 >= 0.95.
+
+Workload (BASELINE.json configs[1]): SIFT1M-shaped 1M x 128 fp32 L2, degree-64
+CAGRA-style graph (exact 128-NN + prune), k=10, B=32 query slots in flight
+(dynamic batching).  Inputs are seeded synthetic data (synth/).
+
+One step = one pass of the whole hot path over one batch of NQ_STEP queries:
+the persistent search kernel keeps B slots busy from an HBM-resident query
+queue (a1-a8), every slot's CTAs publish per-CTA top-k, the host merges
+(a9).  `value` = queries/s of the device-resident path (CUDA events on the
+launch stream, inputs already in HBM).  `e2e` = the same metric through the
+public persistent-server API (algas_submit / algas_poll): queries copied
+from host memory into the host-mapped slot ring, read by the GPU over PCIe,
+results written back to host memory, merged on the host.
+
+Multi-GPU (torchrun, one process per GPU): replicas only -- every rank holds
+the full index and serves its own query stream; no data-path collective
+(DESIGN.md §7).  value = all ranks' queries / max-over-ranks time.
+
+--impl reference: the CPU oracle (oracle/, O2 reference search, T=1, same
+graph and parameters) timed on the host cores, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC_NAME = "p50/p99 query latency and QPS at recall@10=0.95, batch 1-32, 1/2/4/8 B200"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            mp = json.load(f)
+        return float(mp["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.samples.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for s in self.samples:
+            for nm, v in zip(names, s[3:7]):
+                if v.strip().lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
+
+
+def recall_at(found, truth, k):
+    hits = 0
+    for f, t in zip(found[:, :k], truth[:, :k]):
+        hits += len(set(f.tolist()) & set(t.tolist()))
+    return hits / float(truth.shape[0] * k)
+
+
+def dist_init():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def build_workload(w, nq, dev):
+    """Synthetic data + graph + ground truth on this rank's GPU (setup, untimed)."""
+    import torch
+
+    import paper_conf_ipps_chencyzw025_b200 as algas
+    import synth
+    t0 = time.time()
+    X = synth.base_vectors(w)
+    Q = synth.query_vectors(w, nq)
+    Xd = torch.from_numpy(X).to(dev)
+    Qd = torch.from_numpy(Q).to(dev)
+    knn, _ = algas.knn(Xd, Xd, w.knn_degree, w.metric, self_base=0)
+    G = algas.prune(knn, w.degree) if w.prune else knn[:, :w.degree].contiguous()
+    G = G.cpu().numpy().view(np.uint32)
+    del knn
+    ti, _ = algas.knn(Xd, Qd, w.k, w.metric)
+    ti = ti.cpu().numpy().view(np.uint32)
+    torch.cuda.synchronize()
+    return X, Q, Xd, Qd, G, ti, time.time() - t0
+
+
+def choose_operating_point(idx, Qd, truth, w, slots, target=0.95, T=1, threads=64, width=4):
+    """Smallest L in the sweep whose recall@k >= target (BASELINE metric)."""
+    import paper_conf_ipps_chencyzw025_b200 as algas
+    sweep = []
+    chosen = None
+    for L in [16, 24, 32, 48, 64, 96, 128, 192, 256, 384, 512]:
+        if L < w.k:
+            continue
+        p = algas.default_params(k=w.k, itopk=L, width=width if L > 32 else min(width, 2),
+                                 offset_beam=max(1, L // 4), ctas_per_query=T, threads_per_cta=threads,
+                                 slots=slots, n_seeds=32, seed=1)
+        r = idx.search_dynamic(Qd, p)
+        rec = recall_at(r["ids"], truth, w.k)
+        sweep.append({"itopk": L, "width": p.width, "recall": round(rec, 5)})
+        if rec >= target and chosen is None:
+            chosen = p
+            break
+    return chosen, sweep
+
+
+def run_algas(a, rank, world, local):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_chencyzw025_b200 as algas
+    import synth
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    w = synth.WORKLOADS[a.config]
+    X, Q, Xd, Qd, G, truth, t_setup = build_workload(w, a.nq, dev)
+    idx = algas.Index(Xd, G, w.metric)
+    p, sweep = choose_operating_point(idx, Qd, truth, w, a.batch, T=a.ctas, threads=a.threads, width=a.width)
+    if p is None:
+        raise SystemExit("no swept itopk reaches recall 0.95")
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # 256 MB > 126 MB L2
+
+    def step():
+        return idx.search_dynamic(Qd, p, stream=stream)
+
+    for _ in range(a.warmup):
+        r = step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    kern_ms, lat, evals, parents, recs = [], [], [], [], []
+    with ClockSampler(local) as clk:
+        for i in range(a.steps):
+            flush.zero_()                       # L2 flush between timed steps (untimed)
+            torch.cuda.synchronize()
+            ev[i][0].record(stream)
+            r = step()
+            ev[i][1].record(stream)
+            torch.cuda.synchronize()
+            kern_ms.append(r["info"].kernel_ms)
+            st = r["stats"]
+            lat.append((st["t_end_ns"] - st["t_start_ns"]) / 1e3)
+            evals.append(st["dist_evals"].astype(np.float64))
+            parents.append(st["parents"].astype(np.float64))
+            recs.append(recall_at(r["ids"], truth, w.k))
+    step_ms = np.array([e0.elapsed_time(e1) for e0, e1 in ev])
+    t_local = float(step_ms.sum())
+    if world > 1:
+        t = torch.tensor([t_local], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_max = float(t.item())
+    else:
+        t_max = t_local
+    total_q = a.nq * a.steps * world
+    value = total_q / (t_max / 1e3)
+    lat = np.concatenate(lat)
+    evals = np.concatenate(evals)
+    parents = np.concatenate(parents)
+
+    # ---- roofline of the dominant kernel (the persistent search kernel)
+    # algorithmic bytes per query: neighbour rows + gathered
+    # vectors + the query + per-CTA results
+    Rp = (w.degree + 3) // 4 * 4
+    bytes_q = parents * Rp * 4 + evals * w.dim * 4 + w.dim * 4 + p.ctas_per_query * w.k * 8
+    algo_bytes_per_launch = float(bytes_q.mean()) * a.nq
+    kernel_s = float(np.mean(kern_ms)) / 1e3
+    achieved = algo_bytes_per_launch / kernel_s / 1e9
+    peak, peak_src = _peaks()
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"traffic_{a.config}.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("dram_bytes_per_launch_per_query")
+            if traffic is not None:
+                traffic = float(traffic) * a.nq
+        except Exception:
+            traffic = None
+
+    # ---- e2e through the persistent server (host queries, host results)
+    e2e = None
+    lat_e2e = None
+    if not a.no_e2e:
+        srv = algas.Server(idx, p)
+        try:
+            def serve(nq):
+                done = 0
+                lats = []
+                pending = 0
+                t0 = time.perf_counter()
+                while done < nq:
+                    while pending < nq and srv.submit(Q[pending % Q.shape[0]], tag=pending):
+                        pending += 1
+                    tags, ids, ds, st = srv.poll(256)
+                    done += len(tags)
+                    lats.append(st["latency_ns"])
+                return time.perf_counter() - t0, np.concatenate(lats) if lats else np.zeros(0)
+            serve(min(2000, a.nq))  # warm-up
+            if world > 1:
+                dist.barrier()
+            el, le = serve(a.nq * a.e2e_steps)
+            if world > 1:
+                t = torch.tensor([el], device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                el = float(t.item())
+            q_e2e = a.nq * a.e2e_steps * world
+            e2e = {"value": q_e2e / el, "unit": "queries/s",
+                   "h2d_bytes_per_step": int(a.nq * (w.dim * 4 + 32)),
+                   "d2h_bytes_per_step": int(a.nq * (p.ctas_per_query * (w.k * 8 + 32) + 4)),
+                   "p50_us": float(np.percentile(le / 1e3, 50)), "p99_us": float(np.percentile(le / 1e3, 99)),
+                   "path": "algas_submit/algas_poll (host-mapped slot ring, persistent kernel, host merge)"}
+        finally:
+            srv.close()
+
+    # ---- batch-size sweep (dynamic batching, device-resident), informational
+    batch_sweep = []
+    if not a.no_sweep:
+        for B in (1, 8, 16, 32):
+            pb = algas.default_params(k=p.k, itopk=p.itopk, width=p.width, offset_beam=p.offset_beam,
+                                      ctas_per_query=p.ctas_per_query, threads_per_cta=p.threads_per_cta,
+                                      slots=B, n_seeds=p.n_seeds, seed=p.seed)
+            nqb = min(a.nq, 400 * B)
+            rb = idx.search_dynamic(Qd[:nqb], pb, stream=stream)
+            lb = (rb["stats"]["t_end_ns"] - rb["stats"]["t_start_ns"]) / 1e3
+            batch_sweep.append({"batch": B, "qps": nqb / (rb["info"].kernel_ms / 1e3),
+                                "p50_us": float(np.percentile(lb, 50)), "p99_us": float(np.percentile(lb, 99)),
+                                "recall": round(recall_at(rb["ids"], truth[:nqb], w.k), 5)})
+
+    # ---- CPU baseline: the oracle as it stands, bounded sample, rank 0 only
+    cpu = None
+    if rank == 0 and not a.no_cpu:
+        cpu = cpu_baseline(X, G, Q, truth, w, p, budget_s=a.cpu_budget)
+
+    if world > 1:
+        dist.barrier()
+    if rank != 0:
+        return
+    line = {
+        "metric": METRIC_NAME,
+        "value": value,
+        "unit": "queries/s",
+        "n_gpus": world,
+        "steps": a.steps,
+        "warmup": a.warmup,
+        "ms_per_step": t_max / a.steps,
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f32",
+        "data": "synthetic (seeded clustered Gaussian mixture, SIFT1M-shaped; synth/)",
+        "config": {"workload": w.name, "n": w.n, "dim": w.dim, "metric": "L2" if w.metric == 0 else "IP",
+                   "degree": w.degree, "k": w.k, "batch_slots": a.batch, "queries_per_step": a.nq,
+                   "itopk": p.itopk, "width": p.width, "offset_beam": p.offset_beam,
+                   "ctas_per_query": p.ctas_per_query, "threads_per_cta": p.threads_per_cta,
+                   "n_seeds": p.n_seeds, "recall_at_k": float(np.mean(recs)), "recall_target": 0.95,
+                   "parallelism": f"replicas x{world}",
+                   "l2": "flushed (256 MB write) between timed steps; index working set 768 MB > L2"},
+        "latency_us": {"p50": float(np.percentile(lat, 50)), "p99": float(np.percentile(lat, 99)),
+                       "definition": "device globaltimer, slot pickup -> last CTA published"},
+        "clocks": clk.summary(),
+        "e2e": e2e,
+        "gpu_launches": a.steps,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                     "kernel": "persistent_kernel (dynamic batching, HBM queue)",
+                     "algorithmic_bytes_per_query": float(bytes_q.mean()),
+                     "kernel_ms": float(np.mean(kern_ms))},
+        "cpu_baseline": cpu,
+        "work": {"dist_evals_per_query": float(evals.mean()), "parents_per_query": float(parents.mean()),
+                 "setup_s": t_setup},
+        "recall_sweep": sweep,
+        "batch_sweep": batch_sweep,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(X, G, Q, truth, w, p, budget_s=15.0):
+    """O2 (oracle/) single-threaded on the host, same graph and parameters
+    with T=1, on a bounded sample of the query stream."""
+    import oracle
+    op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=1, S=p.n_seeds,
+                            max_iter=4 * p.itopk + 256, seed=p.seed)
+    done = 0
+    lats = []
+    ids_all = []
+    t0 = time.perf_counter()
+    while time.perf_counter() - t0 < budget_s and done < Q.shape[0]:
+        q0 = time.perf_counter()
+        ids, ds, st = oracle.search(X, G, Q[done:done + 1], op, metric=w.metric, tag0=done)
+        lats.append(time.perf_counter() - q0)
+        ids_all.append(ids)
+        done += 1
+    el = time.perf_counter() - t0
+    ids_all = np.concatenate(ids_all)
+    return {"value": done / el, "unit": "queries/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {done} queries of the step's query set, one query at a time, "
+                      f"O2 with T=1 (itopk={p.itopk}, width={p.width}), {el:.1f} s",
+            "p50_us": float(np.percentile(np.array(lats) * 1e6, 50)),
+            "p99_us": float(np.percentile(np.array(lats) * 1e6, 99)),
+            "recall_at_k": recall_at(ids_all, truth[:done], w.k)}
+
+
+def run_reference(a, rank, world, local):
+    """--impl reference: the oracle on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    import torch
+
+    import paper_conf_ipps_chencyzw025_b200 as algas
+    import synth
+    w = synth.WORKLOADS[a.config]
+    dev = torch.device("cuda", local) if torch.cuda.is_available() else None
+    if dev is None:
+        print(json.dumps({"impl": "reference", "unavailable": "needs the GPU-built graph of the workload"}))
+        return
+    torch.cuda.set_device(dev)
+    X, Q, Xd, Qd, G, truth, _ = build_workload(w, a.nq, dev)
+    idx = algas.Index(Xd, G, w.metric)
+    p, sweep = choose_operating_point(idx, Qd, truth, w, a.batch, T=a.ctas, threads=a.threads, width=a.width)
+    del idx
+    import oracle
+    op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=1, S=p.n_seeds,
+                            max_iter=4 * p.itopk + 256, seed=p.seed)
+    per_step = max(1, a.ref_queries_per_step)
+    for i in range(a.warmup):
+        oracle.search(X, G, Q[:per_step], op, metric=w.metric)
+    times = []
+    ids_all = []
+    for i in range(a.steps):
+        qs = Q[(i * per_step) % Q.shape[0]:(i * per_step) % Q.shape[0] + per_step]
+        t0 = time.perf_counter()
+        ids, ds, st = oracle.search(X, G, qs, op, metric=w.metric, tag0=i * per_step)
+        times.append(time.perf_counter() - t0)
+        ids_all.append(ids)
+    tot = float(np.sum(times))
+    value = per_step * a.steps / tot
+    line = {"impl": "reference", "metric": METRIC_NAME, "value": value, "unit": "queries/s", "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": tot * 1e3 / a.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": w.name, "n": w.n, "dim": w.dim, "degree": w.degree, "k": w.k,
+                       "itopk": p.itopk, "width": p.width, "ctas_per_query": 1, "queries_per_step": per_step},
+            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{per_step} queries per step, single-threaded O2"},
+            "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "recall_at_k": recall_at(np.concatenate(ids_all), truth[:per_step * a.steps], w.k)
+            if per_step * a.steps <= truth.shape[0] else None}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="algas", choices=["algas", "reference"])
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--nq", type=int, default=10000, help="queries per step")
+    ap.add_argument("--batch", type=int, default=32, help="query slots in flight (B)")
+    ap.add_argument("--ctas", type=int, default=1, help="CTAs per query (T)")
+    ap.add_argument("--threads", type=int, default=256)
+    ap.add_argument("--width", type=int, default=4)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--ref-queries-per-step", type=int, default=100)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true")
+    a = ap.parse_args()
+    if a.warmup < 3:
+        a.warmup = 3
+    rank, world, local = dist_init()
+    if a.impl == "reference":
+        run_reference(a, rank, world, local)
+    else:
+        run_algas(a, rank, world, local)
+
+
+if __name__ == "__main__":
+    main()

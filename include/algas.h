@@ -86,7 +86,7 @@ typedef struct algas_params {
     int32_t visited_mode;    /* enum algas_visited                                  */
     int32_t slots;           /* persistent path: B query slots; 0 -> 32     */
     int32_t hash_bits;       /* log2 of the per-CTA shared-memory visited hash; 0 -> tuner */
-    int32_t reserved0;
+    int32_t stage_rows;      /* vectors per shared-memory staging buffer (2 buffers); 0 -> tuner */
     uint64_t seed;           /* entry-point generator seed (R5)                      */
 } algas_params;
 
@@ -103,6 +103,12 @@ typedef struct algas_query_stats {
     uint64_t t_start_ns;  /* device globaltimer at pickup (persistent/dynamic path) */
     uint64_t t_end_ns;    /* device globaltimer when the last CTA published         */
     uint64_t latency_ns;  /* host: submit -> merged result ready (server path)      */
+    /* SM cycles spent per search phase (summed over CTAs; the paper's
+     * calculation-vs-sorting breakdown, Fig. 3 / Fig. 17) */
+    uint64_t cyc_select;  /* parent selection (P:L217 step 1)                    */
+    uint64_t cyc_gather;  /* neighbour-id gather + visited filter (steps 1-2)    */
+    uint64_t cyc_dist;    /* vector gathers + distances (step 3)                 */
+    uint64_t cyc_sort;    /* sort + merge into the candidate list (step 4)       */
 } algas_query_stats;
 
 /* Optional per-call timing filled by the search entry points. */
@@ -236,6 +242,8 @@ typedef struct algas_tuning {
     int32_t width;
     int32_t offset_beam;
     int32_t hash_bits;
+    int32_t stage_rows;
+    int32_t reserved;
 } algas_tuning;
 
 /* Properties of the current device (props of P:L280-291 Table II). */

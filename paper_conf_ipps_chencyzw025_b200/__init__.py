@@ -41,20 +41,22 @@ class Params(ctypes.Structure):
                 ("offset_beam", ctypes.c_int32), ("ctas_per_query", ctypes.c_int32),
                 ("threads_per_cta", ctypes.c_int32), ("n_seeds", ctypes.c_int32),
                 ("max_iter", ctypes.c_int32), ("visited_mode", ctypes.c_int32), ("slots", ctypes.c_int32),
-                ("hash_bits", ctypes.c_int32), ("reserved0", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class QueryStats(ctypes.Structure):
     _fields_ = [("iters", ctypes.c_uint32), ("max_iters", ctypes.c_uint32), ("parents", ctypes.c_uint32),
                 ("dist_evals", ctypes.c_uint32), ("cap_hits", ctypes.c_uint32), ("spills", ctypes.c_uint32),
                 ("overflows", ctypes.c_uint32), ("ctas", ctypes.c_uint32), ("t_start_ns", ctypes.c_uint64),
-                ("t_end_ns", ctypes.c_uint64), ("latency_ns", ctypes.c_uint64)]
+                ("t_end_ns", ctypes.c_uint64), ("latency_ns", ctypes.c_uint64), ("cyc_select", ctypes.c_uint64),
+                ("cyc_gather", ctypes.c_uint64), ("cyc_dist", ctypes.c_uint64), ("cyc_sort", ctypes.c_uint64)]
 
 
 STATS_DTYPE = np.dtype([("iters", np.uint32), ("max_iters", np.uint32), ("parents", np.uint32),
                         ("dist_evals", np.uint32), ("cap_hits", np.uint32), ("spills", np.uint32),
                         ("overflows", np.uint32), ("ctas", np.uint32), ("t_start_ns", np.uint64),
-                        ("t_end_ns", np.uint64), ("latency_ns", np.uint64)])
+                        ("t_end_ns", np.uint64), ("latency_ns", np.uint64), ("cyc_select", np.uint64),
+                        ("cyc_gather", np.uint64), ("cyc_dist", np.uint64), ("cyc_sort", np.uint64)])
 assert STATS_DTYPE.itemsize == ctypes.sizeof(QueryStats)
 
 
@@ -74,7 +76,7 @@ class Tuning(ctypes.Structure):
     _fields_ = [("ctas_per_query", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
                 ("smem_avail_per_block", ctypes.c_int64), ("smem_per_block", ctypes.c_int64),
                 ("threads_per_cta", ctypes.c_int32), ("width", ctypes.c_int32), ("offset_beam", ctypes.c_int32),
-                ("hash_bits", ctypes.c_int32)]
+                ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 # every symbol include/algas.h declares (checked by tests/test_abi.py)

@@ -40,9 +40,9 @@ struct Workspace {
 struct algas_index {
   int device = 0;
   int64_t n = 0;
-  int32_t dim = 0, d4 = 0, metric = 0, degree = 0, rp4 = 0;
+  int32_t dim = 0, d4 = 0, metric = 0, degree = 0, rp_shift = 0;
   float* d_data = nullptr;      // n x dim
-  uint32_t* d_graph = nullptr;  // n x (4*rp4), sentinel padded
+  uint32_t* d_graph = nullptr;  // n x (1 << rp_shift), sentinel padded
   algas::Workspace* ws = nullptr;
 };
 
@@ -63,6 +63,32 @@ struct Plan {
 };
 
 int chunk_config_for(int d4);          // -1 if unsupported
+
+// Shared-memory sizing inside a per-CTA budget: staging rows =
+// one step's new vectors (w x Rp, <= 128, two buffers within a quarter of the
+// budget), then the largest visited hash (<= 2^15) that still fits.  Values
+// already > 0 in *hash_bits / *stage_rows are kept (explicit overrides).
+inline void choose_smem(int dp4, int L, int ncap, int S, int w, int Rp, int64_t budget, int* hash_bits,
+                        int* stage_rows) {
+  const int row_bytes = dp4 * 16;
+  int sr = *stage_rows;
+  if (sr < 0) {
+    sr = 0;  // register gather path: no staging buffers
+  } else if (sr == 0) {
+    sr = 1;
+    while (sr < (w * Rp < 128 ? w * Rp : 128)) sr <<= 1;
+    while (sr > 4 && (int64_t)2 * sr * row_bytes > budget / 4) sr >>= 1;
+  }
+  int hb = *hash_bits;
+  if (hb <= 0) {
+    int hb_min = 6;
+    while ((1LL << hb_min) < 2LL * (S + w * Rp)) ++hb_min;
+    hb = 15;
+    while (hb > hb_min && smem_layout(dp4, L, ncap, hb, sr).total > budget) --hb;
+  }
+  *hash_bits = hb;
+  *stage_rows = sr;
+}
 int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent);
 
 // spill tables: ensure >= entries, returns base pointer (workspace locked by caller)
@@ -129,6 +155,30 @@ inline void carve_control(uint8_t* cb, int slots, PersistArgs* pa) {
   pa->slot_fin = reinterpret_cast<unsigned int*>(cb + 256 + (size_t)slots * 32);
 }
 int max_blocks_per_sm(const Plan& pl, bool persistent, int* out);
+
+// per-query counters from the T per-CTA records
+inline void aggregate_cta_stats(const CtaStats* cs, int T, algas_query_stats* q) {
+  *q = algas_query_stats{};
+  q->ctas = (uint32_t)T;
+  unsigned long long t0 = ~0ull, t1 = 0;
+  for (int c = 0; c < T; ++c) {
+    q->iters += cs[c].iters;
+    if (cs[c].iters > q->max_iters) q->max_iters = cs[c].iters;
+    q->parents += cs[c].parents;
+    q->dist_evals += cs[c].dist_evals;
+    q->cap_hits += cs[c].cap_hit;
+    q->spills += cs[c].spilled;
+    q->overflows += cs[c].overflow;
+    q->cyc_select += cs[c].cyc_select;
+    q->cyc_gather += cs[c].cyc_gather;
+    q->cyc_dist += cs[c].cyc_dist;
+    q->cyc_sort += cs[c].cyc_sort;
+    if (cs[c].t_start < t0) t0 = cs[c].t_start;
+    if (cs[c].t_end > t1) t1 = cs[c].t_end;
+  }
+  q->t_start_ns = t0 == ~0ull ? 0 : t0;
+  q->t_end_ns = t1;
+}
 
 // host TopK merge (runtime.cpp)
 int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t* out_ids, float* out_d);

@@ -136,23 +136,7 @@ static void poller_main(algas_server* s) {
       } else {
         merge_cta_lists(r, T, s->kmax, k, d.ids.data(), d.d.data());
       }
-      memset(&d.st, 0, sizeof(d.st));
-      d.st.ctas = (uint32_t)T;
-      uint64_t t0 = ~0ull, t1 = 0;
-      for (int c = 0; c < T; ++c) {
-        const CtaStats& cs = s->st_h[(size_t)q * T + c];
-        d.st.iters += cs.iters;
-        d.st.max_iters = std::max(d.st.max_iters, cs.iters);
-        d.st.parents += cs.parents;
-        d.st.dist_evals += cs.dist_evals;
-        d.st.cap_hits += cs.cap_hit;
-        d.st.spills += cs.spilled;
-        d.st.overflows += cs.overflow;
-        t0 = std::min<uint64_t>(t0, cs.t_start);
-        t1 = std::max<uint64_t>(t1, cs.t_end);
-      }
-      d.st.t_start_ns = t0;
-      d.st.t_end_ns = t1;
+      aggregate_cta_stats(s->st_h + (size_t)q * T, T, &d.st);
       d.st.latency_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
                             std::chrono::steady_clock::now() - s->t_submit[q])
                             .count();
@@ -424,9 +408,10 @@ int algas_device_query(algas_device_props* out) {
 }
 
 // Full tuner.  Policy ("tuner"):
-//  * threads/CTA: the paper fixes one warp; on B200 the distance
-//    gathers need more loads in flight per query, so 64 threads for d <= 128,
-//    128 above (one 16-B chunk per lane per vector row at 512 B rows).
+//  * threads/CTA: the paper fixes one warp; on B200 a search step is
+//    latency-bound (dependent select -> gather -> distance -> merge) and the
+//    per-SM random-gather rate grows with loads in flight, so 8 warps
+//    (measured: 64 -> 256 threads = 2x QPS at C2, profiles/round1_c2.md).
 //  * N_parallel: the largest T allowed by P:L231 whose per-block shared memory
 //    fits P:L245 (with M_reserved grown for wide vectors), capped at
 //    T_cap = 8 beyond which extra CTAs mostly repeat work (measured in
@@ -443,45 +428,51 @@ int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int3
     if (rc) return rc;
     props = &dp;
   }
-  const int nt = dim <= 128 ? 64 : 128;
+  const int nt = 256;
   const int w = itopk <= 32 ? 1 : (itopk <= 64 ? 2 : 4);
-  const int Rp = (degree + 3) / 4 * 4;
+  int Rp = 4;
+  while (Rp < degree) Rp <<= 1;
   const int S = 32;
   int ncap = 1;
   while (ncap < std::max(S, w * Rp)) ncap <<= 1;
-  long long need = 8LL * itopk + 2LL * (S + w * Rp);
-  int hb = 10;
-  while ((1LL << hb) < need && hb < 15) ++hb;
-  const int d4 = dim / 4;
-  const int64_t smem = smem_layout(d4, itopk, ncap, hb).total;
+  const int cc = chunk_config_for(dim / 4);
+  if (cc < 0) return set_error(ALGAS_EINVAL, "algas_tune: dim %d unsupported", dim);
+  const int dp4 = chunk_tl(cc) * chunk_cpl(cc);
   // M_reserved_per_block: driver reservation + extra L1 for wide rows
   const int64_t reserved = props->smem_reserved_per_block + (dim > 256 ? 8 * 1024 : 0);
   const int tmax_eq = algas_tuner_max_parallel(slots, props->n_sm, props->max_blocks_per_sm);
   const int tcap = std::min(8, ALGAS_MAX_CTAS);
-  int best = 0, best_bps = 0;
-  int64_t best_avail = 0;
+  int best = 0, best_bps = 0, best_hb = 0, best_sr = 0;
+  int64_t best_avail = 0, best_smem = 0;
   for (int T = std::min(tmax_eq, tcap); T >= 1; --T) {
-    const int bps = algas_tuner_blocks_per_sm(T, slots, props->n_sm);
+    const int bps = algas_tuner_blocks_per_sm(T, slots, props->n_sm);        // P:L235
     if (bps > props->max_blocks_per_sm) continue;
     if ((int64_t)bps * nt > props->max_threads_per_sm) continue;
-    const int64_t avail = algas_tuner_smem_per_block(props->smem_per_sm, bps, reserved);
-    if (smem <= avail) {
+    const int64_t avail = algas_tuner_smem_per_block(props->smem_per_sm, bps, reserved);  // P:L245
+    int hb = 0, sr = 0;
+    choose_smem(dp4, itopk, ncap, S, w, Rp, avail, &hb, &sr);
+    const int64_t smem = smem_layout(dp4, itopk, ncap, hb, sr).total;
+    if (smem <= avail && smem <= props->smem_per_block_optin - props->smem_reserved_per_block) {
       best = T;
       best_bps = bps;
       best_avail = avail;
+      best_hb = hb;
+      best_sr = sr;
+      best_smem = smem;
       break;
     }
   }
-  if (best == 0) return set_error(ALGAS_EINVAL, "algas_tune: no N_parallel fits %d slots (smem %lld B)", slots, (long long)smem);
+  if (best == 0) return set_error(ALGAS_EINVAL, "algas_tune: no N_parallel fits %d slots", slots);
   memset(out, 0, sizeof(*out));
   out->ctas_per_query = best;
   out->blocks_per_sm = best_bps;
   out->smem_avail_per_block = best_avail;
-  out->smem_per_block = smem;
+  out->smem_per_block = best_smem;
   out->threads_per_cta = nt;
   out->width = w;
   out->offset_beam = std::max(1, itopk / 4);
-  out->hash_bits = hb;
+  out->hash_bits = best_hb;
+  out->stage_rows = best_sr;
   (void)k;
   return ALGAS_OK;
 }

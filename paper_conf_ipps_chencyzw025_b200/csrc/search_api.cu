@@ -33,12 +33,6 @@ bool is_device_ptr(const void* p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-static int ilog2_ceil(long long x) {
-  int b = 0;
-  while ((1LL << b) < x) ++b;
-  return b;
-}
-
 int ensure_gtab(algas_index* idx, size_t entries) {
   Workspace* ws = idx->ws;
   if (ws->gtab_entries >= entries) return ALGAS_OK;
@@ -89,22 +83,34 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
     return set_error(ALGAS_EINVAL, "threads_per_cta %d not in {32,64,128,256}", nt);
   const int cc = chunk_config_for(idx->d4);
   if (cc < 0) return set_error(ALGAS_EINVAL, "dim %d unsupported", idx->dim);
-  const int Rp = idx->rp4 * 4;
+  const int Rp = 1 << idx->rp_shift;
+  const int dp4 = chunk_tl(cc) * chunk_cpl(cc);
   int ncap = 1;
   while (ncap < std::max(S, w * Rp)) ncap <<= 1;
-  int hb = p->hash_bits;
-  if (hb <= 0) {
-    long long need = 8LL * L + 2LL * (S + w * Rp);
-    hb = std::min(15, std::max(10, ilog2_ceil(need)));
-  }
+  int optin = 0, dev = 0, smem_sm = 0, reserved = 0, nsm = 0;
+  ALGAS_CUDA_TRY(cudaGetDevice(&dev));
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev));
+  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  // Shared-memory budget per CTA: M_avail = M_per_SM / N_block_per_SM
+  // - M_reserved, with N_block_per_SM from P:L235 for a persistent grid of
+  // slots x T CTAs, or a target occupancy of 8 CTAs/SM for a static batch.
+  const int bps = persistent ? std::max(1, (int)(((int64_t)slots * T + nsm - 1) / nsm)) : 8;
+  const int64_t budget = std::min<int64_t>((int64_t)smem_sm / bps - reserved, (int64_t)optin - reserved);
+  // vector-gather path: 0 = LDG.128 into registers (default),
+  // 1 = cp.async (LDGSTS) staging, 2 = cp.async.bulk staging; the staged
+  // paths are kept as measured alternatives (ALGAS_GATHER_MODE)
+  const char* gm_env = getenv("ALGAS_GATHER_MODE");
+  const int gather_mode = gm_env ? atoi(gm_env) : 0;
+  if (gather_mode < 0 || gather_mode > 2) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0, 1 or 2");
+  int hb = p->hash_bits, sr = gather_mode == 0 ? -1 : p->stage_rows;
+  choose_smem(dp4, L, ncap, S, w, Rp, budget, &hb, &sr);
   if (hb < 6 || hb > 16) return set_error(ALGAS_EINVAL, "hash_bits %d not in [6,16]", hb);
   if ((1 << hb) < 2 * (S + w * Rp))
     return set_error(ALGAS_EINVAL, "visited hash 2^%d too small for seeds + one step (%d)", hb, S + w * Rp);
-  SmemLayout lay = smem_layout(idx->d4, L, ncap, hb);
-  int optin = 0, dev = 0;
-  ALGAS_CUDA_TRY(cudaGetDevice(&dev));
-  ALGAS_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
-  if (lay.total + 1024 > optin)
+  SmemLayout lay = smem_layout(dp4, L, ncap, hb, sr);
+  if (lay.total + reserved > optin)
     return set_error(ALGAS_EINVAL, "search needs %d B shared memory per CTA, device allows %d", lay.total, optin);
 
   pl.nt = nt;
@@ -116,19 +122,26 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   pl.metric = idx->metric;
   SearchCfg& c = pl.cfg;
   c.data = reinterpret_cast<const float4*>(idx->d_data);
-  c.graph = reinterpret_cast<const uint4*>(idx->d_graph);
+  c.graph = idx->d_graph;
   c.n = (uint64_t)idx->n;
   c.d4 = idx->d4;
+  c.dp4 = dp4;
   c.R = idx->degree;
-  c.rp4 = idx->rp4;
+  c.rp_shift = idx->rp_shift;
   c.L = L;
   c.w = w;
   c.off = p->offset_beam < 0 ? std::max(1, L / 4) : std::min(p->offset_beam, L);
   c.S = S;
   c.max_iter = p->max_iter > 0 ? p->max_iter : 4 * L + 256;
   c.hash_bits = hb;
-  c.gtab_bits = std::min(20, hb + 2);
+  c.gtab_bits = std::min(20, std::max(16, hb + 2));
   c.ncap = ncap;
+  c.stage_rows = sr;
+  c.gather_mode = gather_mode;
+  {
+    const char* pf = getenv("ALGAS_PREFETCH");  // experiment switch
+    c.prefetch = pf ? atoi(pf) : 0;
+  }
   c.seed = p->seed;
   int nb = 0;
   int rc = max_blocks_per_sm(pl, persistent, &nb);
@@ -161,25 +174,6 @@ struct DevBuf {
   }
 };
 
-static void aggregate_stats(const CtaStats* cs, int T, algas_query_stats* q) {
-  memset(q, 0, sizeof(*q));
-  q->ctas = (uint32_t)T;
-  uint64_t t0 = ~0ull, t1 = 0;
-  for (int c = 0; c < T; ++c) {
-    q->iters += cs[c].iters;
-    q->max_iters = std::max(q->max_iters, cs[c].iters);
-    q->parents += cs[c].parents;
-    q->dist_evals += cs[c].dist_evals;
-    q->cap_hits += cs[c].cap_hit;
-    q->spills += cs[c].spilled;
-    q->overflows += cs[c].overflow;
-    t0 = std::min<uint64_t>(t0, cs[c].t_start);
-    t1 = std::max<uint64_t>(t1, cs[c].t_end);
-  }
-  q->t_start_ns = t0 == ~0ull ? 0 : t0;
-  q->t_end_ns = t1;
-}
-
 // Host merge of nq x T x k per-CTA lists into the caller's outputs.
 static int finish_outputs(const std::vector<ResultEntry>& res, const std::vector<CtaStats>& cst, int64_t nq,
                           int T, int kin, int k, uint32_t* out_ids, float* out_dists, uint32_t* out_cta_ids,
@@ -211,7 +205,7 @@ static int finish_outputs(const std::vector<ResultEntry>& res, const std::vector
   *overflow = false;
   for (int64_t q = 0; q < nq; ++q) {
     algas_query_stats qs;
-    aggregate_stats(cst.data() + q * T, T, &qs);
+    aggregate_cta_stats(cst.data() + q * T, T, &qs);
     if (qs.overflows) *overflow = true;
     if (out_stats) out_stats[q] = qs;
   }
@@ -309,10 +303,11 @@ algas_index* algas_index_create(const float* data, int64_t n, int32_t dim, int32
   idx->d4 = dim / 4;
   idx->metric = metric;
   idx->degree = degree;
-  idx->rp4 = (degree + 3) / 4;
+  idx->rp_shift = 2;  // graph rows padded to a power-of-two stride (>= 4 ids)
+  while ((1 << idx->rp_shift) < degree) ++idx->rp_shift;
   idx->ws = new Workspace();
   cudaGetDevice(&idx->device);
-  const size_t dbytes = (size_t)n * dim * 4, gpitch = (size_t)idx->rp4 * 16;
+  const size_t dbytes = (size_t)n * dim * 4, gpitch = (size_t)4 << idx->rp_shift;
   auto fail = [&](const char* what, cudaError_t e) -> algas_index* {
     set_error(e == cudaErrorMemoryAllocation ? ALGAS_ENOMEM : ALGAS_ECUDA, "algas_index_create: %s: %s", what,
               cudaGetErrorString(e));
@@ -362,7 +357,7 @@ int algas_index_info(const algas_index* idx, int64_t* n, int32_t* dim, int32_t* 
   if (dim) *dim = idx->dim;
   if (metric) *metric = idx->metric;
   if (degree) *degree = idx->degree;
-  if (graph_stride) *graph_stride = idx->rp4 * 4;
+  if (graph_stride) *graph_stride = 1 << idx->rp_shift;
   if (dev_data) *dev_data = idx->d_data;
   if (dev_graph) *dev_graph = idx->d_graph;
   return ALGAS_OK;

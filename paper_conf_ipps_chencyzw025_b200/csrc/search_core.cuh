@@ -3,13 +3,17 @@
 // One CTA runs one (query, cta_rank) search:
 //   select  : first unchecked candidate(s) of the sorted list            (P:L217 step 1, Alg.1 l.6)
 //             -- w parents at once after the list offset reaches off   (beam extend)
-//   gather  : the parents' neighbour ids, 16-B vector loads of graph rows (P:L217 step 1)
+//   gather  : the parents' neighbour ids (one id per thread)             (P:L217 step 1)
 //   filter  : test-and-set in a shared-memory visited hash               (P:L217 step 2)
-//   distance: coalesced 16-B gathers of the neighbour vectors, a team of
-//             TL lanes per vector, shuffle-tree reduction                (P:L217 step 3, Alg.1 l.9-12)
-//   update  : keys that cannot enter the list are dropped, survivors are
-//             bitonic-sorted and MERGED (rank merge, no re-sort) into the
-//             sorted list, keeping the first L                           (P:L219 step 4, Alg.1 l.15-18)
+//   distance: the surviving neighbours' vectors are copied into shared
+//             memory asynchronously (16-B cp.async per lane, or one
+//             cp.async.bulk per row on an mbarrier) so every row of a step
+//             is in flight at once without holding registers; a team of TL
+//             lanes per row reduces (q-x)^2 / q.x with a shuffle tree    (P:L217 step 3, Alg.1 l.9-12)
+//   update  : keys that cannot enter the list are dropped; survivors are
+//             MERGED into the sorted list by rank (position = rank among
+//             the new keys + lower bound in the list), keeping the first L,
+//             with no re-sort of the list                                (P:L219 step 4, Alg.1 l.15-18)
 //   finish  : all L entries checked (or the max_iter cap)                ("Finish")
 // The CTA then writes its first k (id, dist).
 //
@@ -63,13 +67,6 @@ __device__ __forceinline__ uint32_t entry_point(uint64_t seed, uint64_t tag, uin
 }
 
 // ------------------------------------------------------------------ memory helpers
-__device__ __forceinline__ float4 ldg_stream(const float4* p) {
-  float4 r;
-  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
-               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
-               : "l"(p));
-  return r;
-}
 __device__ __forceinline__ uint4 ldg_u4(const uint4* p) {
   uint4 r;
   asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -82,25 +79,87 @@ __device__ __forceinline__ uint64_t globaltimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+// mbarrier + bulk async copy (TMA engine, non-tensor), CTA scope
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(phase)
+        : "memory");
+  }
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
 
 // ------------------------------------------------------------------ configuration
+// Distance "chunk configs": TL lanes per vector, CPL 16-B chunks per lane.
+// A vector of d4 = dim/4 chunks is stored in shared memory padded to
+// dp4 = TL*CPL chunks (zero tail) so the distance loop needs no masks.
+//   cc: 0      1      2      3      4       5       6
+//   d4: <=8   <=16   <=32   <=64   <=128   <=256   <=512
+__host__ __device__ inline int chunk_tl(int cc) { const int t[7] = {8, 16, 32, 32, 32, 32, 32}; return t[cc]; }
+__host__ __device__ inline int chunk_cpl(int cc) { const int t[7] = {1, 1, 1, 2, 4, 8, 16}; return t[cc]; }
+__device__ __forceinline__ float4 ldg_f4_stream(const float4* p) {
+  float4 r;
+  // volatile: keeps every gather load of a pass ahead of the first use (the
+  // scheduler otherwise interleaves loads with the FMAs of earlier rows and
+  // serialises the DRAM round trips)
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+  return r;
+}
+
 struct SearchCfg {
   const float4* data;    // n x d4 float4 (row-major, 16-B aligned rows)
-  const uint4* graph;    // n x rp4 uint4 (row stride Rp = 4*rp4, padded with sentinels)
+  const uint32_t* graph; // n x Rp u32 (Rp = 1 << rp_shift, padded with sentinels)
   uint64_t n;
   int32_t d4;            // dim / 4
+  int32_t dp4;           // padded row length in shared memory (TL*CPL)
   int32_t R;             // out-degree
-  int32_t rp4;           // padded row length / 4
+  int32_t rp_shift;      // log2 of the graph row stride
   int32_t L, w, off, S, max_iter;
   int32_t hash_bits;     // shared-memory visited hash: 2^hash_bits u32
   int32_t gtab_bits;     // HBM spill table per CTA: 2^gtab_bits u64
-  int32_t ncap;          // capacity of the new-key buffer (power of two)
+  int32_t ncap;          // capacity of the new-key buffer
+  int32_t stage_rows;    // vectors per shared-memory staging buffer (2 buffers)
+  int32_t gather_mode;   // 0: LDG.128 into registers, many rows in flight per warp (default)
+                         // 1: 16-B cp.async (LDGSTS) staging, 2: cp.async.bulk staging (mbarrier)
+  int32_t prefetch;      // 1: L2 bulk prefetch of each surviving row at filter time
   uint64_t seed;
 };
 
 struct CtaStats {
   uint32_t iters, parents, dist_evals, cap_hit, spilled, overflow;
   unsigned long long t_start, t_end;  // globaltimer (persistent paths)
+  unsigned long long cyc_select, cyc_gather, cyc_dist, cyc_sort;  // SM cycles per phase
 };
 
 struct ResultEntry {
@@ -111,23 +170,26 @@ struct ResultEntry {
 struct Ctrl {
   int cnt, nnew, nkeys, np, done, diffusing, vis_count, spilled, overflow, cur;
   uint32_t iters, parents, dist_evals, cap_hit;
+  uint32_t phase;  // bit b: parity of staging barrier b
 };
 
 // Shared-memory carve-up (bytes, all 16-B aligned).
 struct SmemLayout {
-  int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_hash, off_ctrl, total;
+  int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_hash, off_stage, off_bar, off_ctrl, total;
 };
 __host__ __device__ inline int align16(int x) { return (x + 15) & ~15; }
-__host__ __device__ inline SmemLayout smem_layout(int d4, int L, int ncap, int hash_bits) {
+__host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int hash_bits, int stage_rows) {
   SmemLayout s;
   int o = 0;
-  s.off_q = o;     o += align16(d4 * 16);
+  s.off_stage = o; o += 2 * stage_rows * dp4 * 16;  // 128-B aligned at offset 0
+  s.off_q = o;     o += align16(dp4 * 16);
   s.off_listA = o; o += align16(L * 8);
   s.off_listB = o; o += align16(L * 8);
   s.off_newk = o;  o += align16(ncap * 8);
   s.off_newid = o; o += align16(ncap * 4);
   s.off_sel = o;   o += align16(64 * 4);
   s.off_hash = o;  o += align16((1 << hash_bits) * 4);
+  s.off_bar = o;   o += 16;
   s.off_ctrl = o;  o += align16((int)sizeof(Ctrl));
   s.total = o;
   return s;
@@ -140,6 +202,8 @@ struct Smem {
   uint32_t* newid;
   int* sel;         // [0,32): selected positions, [32,64): parent ids
   uint32_t* hash;
+  float4* stage;    // 2 x stage_rows x dp4
+  uint64_t* bar;    // 2 mbarriers
   Ctrl* ctrl;
 };
 __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
@@ -151,8 +215,25 @@ __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
   s.newid = reinterpret_cast<uint32_t*>(base + l.off_newid);
   s.sel = reinterpret_cast<int*>(base + l.off_sel);
   s.hash = reinterpret_cast<uint32_t*>(base + l.off_hash);
+  s.stage = reinterpret_cast<float4*>(base + l.off_stage);
+  s.bar = reinterpret_cast<uint64_t*>(base + l.off_bar);
   s.ctrl = reinterpret_cast<Ctrl*>(base + l.off_ctrl);
   return s;
+}
+// once per CTA lifetime (kernel start): staging barriers; zero staging and
+// query buffers so the padded tail chunks of every row read as 0
+template <int NT>
+__device__ __forceinline__ void init_cta(const Smem& s, const SearchCfg& cfg) {
+  const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int i = threadIdx.x; i < 2 * cfg.stage_rows * cfg.dp4; i += NT) s.stage[i] = z;
+  for (int i = threadIdx.x; i < cfg.dp4; i += NT) s.q[i] = z;
+  if (threadIdx.x == 0) {
+    mbar_init(s.bar + 0, 1);
+    mbar_init(s.bar + 1, 1);
+    mbar_fence_init();
+    s.ctrl->phase = 0;
+  }
+  __syncthreads();
 }
 
 // ------------------------------------------------------------------ visited set
@@ -203,38 +284,6 @@ __device__ __forceinline__ int gmem_visit(unsigned long long* tab, int bits, uin
   return kVisFull;
 }
 
-// ------------------------------------------------------------------ sorting
-// ascending bitonic sort of one u64 per lane
-__device__ __forceinline__ uint64_t warp_bitonic32(uint64_t v, int lane) {
-#pragma unroll
-  for (int k = 2; k <= 32; k <<= 1) {
-#pragma unroll
-    for (int j = k >> 1; j > 0; j >>= 1) {
-      uint64_t o = __shfl_xor_sync(0xffffffffu, v, j);
-      bool up = (lane & k) == 0;
-      bool lower = (lane & j) == 0;
-      bool keep_min = (lower == up);
-      v = keep_min ? (o < v ? o : v) : (o > v ? o : v);
-    }
-  }
-  return v;
-}
-// ascending bitonic sort of s[0..P), P power of two; all NT threads call
-template <int NT>
-__device__ __forceinline__ void cta_bitonic(uint64_t* s, int P, int tid) {
-  for (int k = 2; k <= P; k <<= 1) {
-    for (int j = k >> 1; j > 0; j >>= 1) {
-      for (int i = tid; i < (P >> 1); i += NT) {
-        int lo = 2 * j * (i / j) + (i % j);
-        int hi = lo + j;
-        bool up = (lo & k) == 0;
-        uint64_t a = s[lo], b = s[hi];
-        if ((a > b) == up) { s[lo] = b; s[hi] = a; }
-      }
-      __syncthreads();
-    }
-  }
-}
 template <typename K>
 __device__ __forceinline__ int lower_bound_u64(const K* a, int n, K x) {
   int lo = 0, hi = n;
@@ -246,50 +295,66 @@ __device__ __forceinline__ int lower_bound_u64(const K* a, int n, K x) {
 }
 
 // ------------------------------------------------------------------ distance (P:L217 step 3)
-template <int TL, int CPL, int METRIC>
+template <int TL, int CPL>
 struct QueryRegs {
   float4 q[CPL];
-  __device__ __forceinline__ void load(const float4* qs, int d4, int tl) {
+  __device__ __forceinline__ void load(const float4* qs, int tl) {
 #pragma unroll
-    for (int c = 0; c < CPL; ++c) {
-      int ch = tl + c * TL;
-      q[c] = (ch < d4) ? qs[ch] : make_float4(0.f, 0.f, 0.f, 0.f);
-    }
+    for (int c = 0; c < CPL; ++c) q[c] = qs[tl + c * TL];  // padded with zeros
   }
 };
 
+// partial sum of one team lane over a (zero-padded) row in shared memory
 template <int TL, int CPL, int METRIC>
-__device__ __forceinline__ float team_partial(const QueryRegs<TL, CPL, METRIC>& Q, const float4* x, int d4,
-                                              int tl) {
-  float4 v[CPL];
-#pragma unroll
-  for (int c = 0; c < CPL; ++c) {
-    int ch = tl + c * TL;
-    v[c] = (ch < d4) ? ldg_stream(x + ch) : make_float4(0.f, 0.f, 0.f, 0.f);
-  }
+__device__ __forceinline__ float team_partial_smem(const QueryRegs<TL, CPL>& Q, const float4* x, int tl) {
   float acc = 0.f;
 #pragma unroll
   for (int c = 0; c < CPL; ++c) {
+    const float4 v = x[tl + c * TL];
     if (METRIC == kL2) {
-      float a = Q.q[c].x - v[c].x, b = Q.q[c].y - v[c].y, e = Q.q[c].z - v[c].z, f = Q.q[c].w - v[c].w;
+      float a = Q.q[c].x - v.x, b = Q.q[c].y - v.y, e = Q.q[c].z - v.z, f = Q.q[c].w - v.w;
       acc = fmaf(a, a, acc); acc = fmaf(b, b, acc); acc = fmaf(e, e, acc); acc = fmaf(f, f, acc);
     } else {
-      acc = fmaf(Q.q[c].x, v[c].x, acc); acc = fmaf(Q.q[c].y, v[c].y, acc);
-      acc = fmaf(Q.q[c].z, v[c].z, acc); acc = fmaf(Q.q[c].w, v[c].w, acc);
+      acc = fmaf(Q.q[c].x, v.x, acc); acc = fmaf(Q.q[c].y, v.y, acc);
+      acc = fmaf(Q.q[c].z, v.z, acc); acc = fmaf(Q.q[c].w, v.w, acc);
     }
   }
   return acc;
 }
-template <int TL>
-__device__ __forceinline__ float team_reduce(float acc) {
-#pragma unroll
-  for (int o = TL >> 1; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-  return acc;
+
+// copies of rows [r0, r0+cnt) of newid into staging buffer b.
+// gather_mode 0: each warp takes rows, its lanes issue 16-B cp.async
+// (LDGSTS) chunks, one commit group for the CTA.  gather_mode 1: warp 0's
+// lanes issue one cp.async.bulk per row, all completing on mbarrier b.
+template <int NT>
+__device__ __forceinline__ void stage_issue(const SearchCfg& cfg, const Smem& s, int b, int r0, int cnt, int warp,
+                                            int lane) {
+  float4* dst = s.stage + (size_t)b * cfg.stage_rows * cfg.dp4;
+  if (cfg.gather_mode == 1) {
+    constexpr int NW = NT / 32;
+    for (int r = warp; r < cnt; r += NW) {
+      const uint32_t id = s.newid[r0 + r];
+      const float4* src = cfg.data + (uint64_t)id * cfg.d4;
+      float4* d = dst + (size_t)r * cfg.dp4;
+      for (int c = lane; c < cfg.d4; c += 32) cp_async16(d + c, src + c);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  } else if (warp == 0) {
+    const uint32_t row_bytes = (uint32_t)cfg.d4 * 16u;
+    fence_proxy_async_smem();
+    if (lane == 0) mbar_arrive_expect_tx(s.bar + b, row_bytes * (uint32_t)cnt);
+    __syncwarp();
+    for (int r = lane; r < cnt; r += 32) {
+      const uint32_t id = s.newid[r0 + r];
+      bulk_g2s(dst + (size_t)r * cfg.dp4, cfg.data + (uint64_t)id * cfg.d4, row_bytes, s.bar + b);
+    }
+  }
 }
 
 // ------------------------------------------------------------------ the search
-// Preconditions: s.q holds the query (d4 float4).  Writes min(k, |list|)
-// results to out[0..k) (rest padded) and the CTA's counters to *st.
+// Preconditions: s.q holds the query (d4 float4, zero tail); init_cta() ran.
+// Writes min(k, |list|) results to out[0..k) (rest padded) and the CTA's
+// counters to *st.
 template <int NT, int TL, int CPL, int METRIC>
 __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, uint32_t cta_rank, int k,
                            unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st) {
@@ -303,22 +368,28 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   const int L = cfg.L;
   const int hbits = cfg.hash_bits;
   const int hcap = 1 << hbits;
-  const int step_max_new = cfg.w * cfg.rp4 * 4;
+  const int Rp = 1 << cfg.rp_shift;
+  const int step_max_new = cfg.w * Rp;
 
-  // ---- reset per-query state
-  for (int i = tid; i < hcap; i += NT) s.hash[i] = kHashEmpty;
+  // ---- reset per-query state (16-B stores)
+  {
+    uint4* h4 = reinterpret_cast<uint4*>(s.hash);
+    const uint4 e = make_uint4(kHashEmpty, kHashEmpty, kHashEmpty, kHashEmpty);
+    for (int i = tid; i < (hcap >> 2); i += NT) h4[i] = e;
+  }
   if (tid == 0) {
     C->cnt = 0; C->nnew = 0; C->nkeys = 0; C->np = 0; C->done = 0; C->diffusing = 0;
     C->vis_count = 0; C->spilled = 0; C->overflow = 0; C->cur = 0;
     C->iters = 0; C->parents = 0; C->dist_evals = 0; C->cap_hit = 0;
   }
-  QueryRegs<TL, CPL, METRIC> Q;
-  Q.load(s.q, cfg.d4, tl);
+  QueryRegs<TL, CPL> Q;
+  Q.load(s.q, tl);
+  uint32_t phase = C->phase;  // staging-barrier parities carried across queries
   __syncthreads();
 
-  // ---- entry points (Alg.1 l.5): S seeds, duplicates dropped
-  // Seeds are inserted sequentially by warp 0 in j order so the visited set
-  // sees exactly the deduplicated seed set.
+  // ---- entry points (Alg.1 l.5): S seeds, duplicates dropped.
+  // Lane 0 of warp 0 inserts them in j order so the visited set holds
+  // exactly the deduplicated seed set.
   if (warp == 0) {
     for (int j0 = 0; j0 < cfg.S; j0 += 32) {
       int j = j0 + lane;
@@ -336,6 +407,17 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   }
   __syncthreads();
 
+  // per-phase SM cycles (thread 0; the paper's calc/sort split, Fig. 3/17)
+  long long tp = clock64();
+  unsigned long long cyc[4] = {0, 0, 0, 0};  // select, gather+filter, distance, merge
+  auto lap = [&](int ph) {
+    if (tid == 0) {
+      long long t = clock64();
+      cyc[ph] += (unsigned long long)(t - tp);
+      tp = t;
+    }
+  };
+
   int cur = 0;
   bool first = true;
   for (;;) {
@@ -343,7 +425,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     if (!first) {
       if (warp == 0) {
         const int cnt = C->cnt;
-        const uint64_t* list = (cur ? s.list[1] : s.list[0]);
+        uint64_t* list = cur ? s.list[1] : s.list[0];
         int found = 0;
         for (int base = 0; base < cnt && found < cfg.w; base += 32) {
           int i = base + lane;
@@ -367,8 +449,8 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           np = diff ? found : 1;
           if (lane < np) {
             int pos = s.sel[lane];
-            uint64_t kk = (cur ? s.list[1] : s.list[0])[pos];
-            (cur ? s.list[1] : s.list[0])[pos] = kk | 1ull;              // mark checked (Alg.1 l.7)
+            uint64_t kk = list[pos];
+            list[pos] = kk | 1ull;                    // mark checked (Alg.1 l.7)
             s.sel[32 + lane] = (int)key_id(kk);
           }
           if (lane == 0) C->diffusing = diff;
@@ -384,48 +466,49 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
         }
       }
       __syncthreads();
+      lap(0);
       if (C->done) break;
 
       // ================= gather + visited filter (P:L217 steps 1-2) =================
       {
         const int np = C->np;
         const int spilled = C->spilled;
-        const int per_row = cfg.rp4;
-        const int total = np * per_row;
+        const int total = np << cfg.rp_shift;  // one neighbour id per thread and pass
         for (int base = 0; base < total; base += NT) {
-          int idx = base + tid;
-          uint32_t ids[4] = {kSentinel, kSentinel, kSentinel, kSentinel};
+          const int idx = base + tid;
+          uint32_t id = kSentinel;
           if (idx < total) {
-            int p = idx / per_row;
-            int c = idx - p * per_row;
-            uint32_t parent = (uint32_t)s.sel[32 + p];
-            uint4 v = ldg_u4(cfg.graph + (uint64_t)parent * per_row + c);
-            ids[0] = v.x; ids[1] = v.y; ids[2] = v.z; ids[3] = v.w;
+            const uint32_t parent = (uint32_t)s.sel[32 + (idx >> cfg.rp_shift)];
+            id = __ldg(cfg.graph + ((uint64_t)parent << cfg.rp_shift) + (idx & (Rp - 1)));
           }
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            bool keep = false;
-            uint32_t id = ids[e];
-            if (id != kSentinel) {
-              if (!spilled) {
-                int r = smem_visit(s.hash, hbits, id);
-                keep = (r == kVisNew);
-                if (r == kVisFull) atomicOr(&C->overflow, 1);
-              } else if (!smem_contains(s.hash, hbits, id)) {
-                int r = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
-                keep = (r == kVisNew);
-                if (r == kVisFull) atomicOr(&C->overflow, 1);
-              }
+          bool keep = false;
+          if (id != kSentinel) {
+            if (!spilled) {
+              const int r = smem_visit(s.hash, hbits, id);
+              keep = (r == kVisNew);
+              if (r == kVisFull) atomicOr(&C->overflow, 1);
+            } else if (!smem_contains(s.hash, hbits, id)) {
+              const int r = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
+              keep = (r == kVisNew);
+              if (r == kVisFull) atomicOr(&C->overflow, 1);
             }
-            unsigned m = __ballot_sync(0xffffffffu, keep);
+          }
+          if (keep && cfg.prefetch == 1) {
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.data + (uint64_t)id * cfg.d4),
+                         "r"((uint32_t)cfg.d4 * 16u)
+                         : "memory");
+          }
+          const unsigned m = __ballot_sync(0xffffffffu, keep);
+          if (m) {
             int wbase = 0;
-            if (lane == 0 && m) wbase = atomicAdd(&C->nnew, __popc(m));
+            if (lane == 0) wbase = atomicAdd(&C->nnew, __popc(m));
             wbase = __shfl_sync(0xffffffffu, wbase, 0);
             if (keep) s.newid[wbase + __popc(m & ((1u << lane) - 1u))] = id;
           }
         }
         __syncthreads();
         if (tid == 0 && !spilled) C->vis_count += C->nnew;
+        lap(1);
       }
     }
     first = false;
@@ -435,76 +518,181 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       const int M = C->nnew;
       const int cnt = C->cnt;
       const uint64_t worst = (cnt >= L) ? (cur ? s.list[1] : s.list[0])[L - 1] : kKeyMax;
-      // warp-uniform trip count: every lane joins the team shuffles
-      for (int base = 0; base < M; base += NTEAMS) {
-        const int i = base + team;
-        const bool valid = i < M;
-        const uint32_t id = valid ? s.newid[i] : 0u;
-        float acc = 0.f;
-        if (valid) acc = team_partial<TL, CPL, METRIC>(Q, cfg.data + (uint64_t)id * cfg.d4, cfg.d4, tl);
-        acc = team_reduce<TL>(acc);
-        if (valid && tl == 0) {
-          float d = (METRIC == kL2) ? acc : -acc;
-          uint64_t key = make_key(d, id);
-          if (key < worst) {
-            int pos = atomicAdd(&C->nkeys, 1);
-            s.newk[pos] = key;
+      if (cfg.gather_mode == 0) {
+        // LDG.128 straight into registers: each team keeps B rows in flight
+        // (NT/TL*B rows per CTA), then reduces them with interleaved shuffle
+        // trees.  The measured single-SM random-gather rate of this path is
+        // 2-3x that of the async-copy paths (profiles/gather_microbench.txt).
+        constexpr int B = CPL >= 16 ? 1 : 16 / CPL;
+        constexpr int PASS = NTEAMS * B;
+        for (int base = 0; base < M; base += PASS) {
+          float4 v[B][CPL];
+#pragma unroll
+          for (int b = 0; b < B; ++b) {
+            const int r = base + b * NTEAMS + team;
+            const float4* row = cfg.data + (uint64_t)(r < M ? s.newid[r] : 0u) * cfg.d4;
+#pragma unroll
+            for (int c = 0; c < CPL; ++c) {
+              const int chn = tl + c * TL;
+              v[b][c] = (r < M && chn < cfg.d4) ? ldg_f4_stream(row + chn) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+          }
+          // all loads of the pass are issued before any use: the warp barrier
+          // keeps ptxas from hoisting FMAs of early rows between the loads
+          // (which would serialise the DRAM round trips)
+          __syncwarp();
+          float acc[B];
+#pragma unroll
+          for (int b = 0; b < B; ++b) {
+            float a = 0.f;
+#pragma unroll
+            for (int c = 0; c < CPL; ++c) {
+              const float4 x = v[b][c];
+              if (METRIC == kL2) {
+                float d0 = Q.q[c].x - x.x, d1 = Q.q[c].y - x.y, d2 = Q.q[c].z - x.z, d3 = Q.q[c].w - x.w;
+                a = fmaf(d0, d0, a); a = fmaf(d1, d1, a); a = fmaf(d2, d2, a); a = fmaf(d3, d3, a);
+              } else {
+                a = fmaf(Q.q[c].x, x.x, a); a = fmaf(Q.q[c].y, x.y, a);
+                a = fmaf(Q.q[c].z, x.z, a); a = fmaf(Q.q[c].w, x.w, a);
+              }
+            }
+            acc[b] = a;
+          }
+#pragma unroll
+          for (int o = TL >> 1; o > 0; o >>= 1)
+#pragma unroll
+            for (int b = 0; b < B; ++b) acc[b] += __shfl_xor_sync(0xffffffffu, acc[b], o);
+          // keys of this pass; one warp-wide scan + one atomic per warp
+          uint64_t key[B];
+          int nkeep = 0;
+#pragma unroll
+          for (int b = 0; b < B; ++b) {
+            const int r = base + b * NTEAMS + team;
+            key[b] = kKeyMax;
+            if (tl == 0 && r < M) key[b] = make_key((METRIC == kL2) ? acc[b] : -acc[b], s.newid[r]);
+            nkeep += (key[b] < worst) ? 1 : 0;
+          }
+          int incl = nkeep;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += t;
+          }
+          const int wtotal = __shfl_sync(0xffffffffu, incl, 31);
+          if (wtotal > 0) {
+            int wbase = 0;
+            if (lane == 0) wbase = atomicAdd(&C->nkeys, wtotal);
+            wbase = __shfl_sync(0xffffffffu, wbase, 0);
+            int pos = wbase + incl - nkeep;
+#pragma unroll
+            for (int b = 0; b < B; ++b)
+              if (key[b] < worst) s.newk[pos++] = key[b];
           }
         }
+        __syncthreads();
       }
-      __syncthreads();
+      const int SR = cfg.stage_rows;
+      const int nchunks = cfg.gather_mode == 0 ? 0 : (M + SR - 1) / SR;
+      if (nchunks > 0) stage_issue<NT>(cfg, s, 0, 0, M < SR ? M : SR, warp, lane);
+      for (int ch = 0; ch < nchunks; ++ch) {
+        const int b = ch & 1;
+        if (ch + 1 < nchunks) {
+          const int r1 = (ch + 1) * SR;
+          stage_issue<NT>(cfg, s, b ^ 1, r1, (M - r1) < SR ? (M - r1) : SR, warp, lane);
+        }
+        if (cfg.gather_mode == 2) {
+          mbar_wait(s.bar + b, (phase >> b) & 1u);
+          phase ^= (1u << b);
+        } else {
+          if (ch + 1 < nchunks) asm volatile("cp.async.wait_group 1;" ::: "memory");
+          else asm volatile("cp.async.wait_group 0;" ::: "memory");
+          __syncthreads();
+        }
+        const int r0 = ch * SR;
+        const int rows = (M - r0) < SR ? (M - r0) : SR;
+        const float4* buf = s.stage + (size_t)b * SR * cfg.dp4;
+        // each team reduces RB rows at once (independent shuffle trees
+        // interleave); rows past `rows` compute garbage that is masked
+        constexpr int RB = (CPL <= 4) ? 4 : (CPL <= 8 ? 2 : 1);
+        for (int base = 0; base < rows; base += NTEAMS * RB) {
+          float acc[RB];
+#pragma unroll
+          for (int j = 0; j < RB; ++j) {
+            const int r = base + team + j * NTEAMS;
+            const int rr = r < SR ? r : SR - 1;
+            acc[j] = team_partial_smem<TL, CPL, METRIC>(Q, buf + (size_t)rr * cfg.dp4, tl);
+          }
+#pragma unroll
+          for (int o = TL >> 1; o > 0; o >>= 1)
+#pragma unroll
+            for (int j = 0; j < RB; ++j) acc[j] += __shfl_xor_sync(0xffffffffu, acc[j], o);
+#pragma unroll
+          for (int j = 0; j < RB; ++j) {
+            const int r = base + team + j * NTEAMS;
+            const bool valid = (tl == 0) && (r < rows);
+            uint64_t key = kKeyMax;
+            if (valid) key = make_key((METRIC == kL2) ? acc[j] : -acc[j], s.newid[r0 + r]);
+            const bool keep = valid && (key < worst);
+            const unsigned m = __ballot_sync(0xffffffffu, keep);
+            if (m) {
+              int wbase = 0;
+              if (lane == 0) wbase = atomicAdd(&C->nkeys, __popc(m));
+              wbase = __shfl_sync(0xffffffffu, wbase, 0);
+              if (keep) s.newk[wbase + __popc(m & ((1u << lane) - 1u))] = key;
+            }
+          }
+        }
+        __syncthreads();  // buffer b fully read before it is re-issued (chunk ch+2)
+      }
       if (tid == 0) C->dist_evals += M;
+      lap(2);
     }
 
-    // ================= sort new keys + merge into the list (P:L219 step 4) =================
+    // ================= merge the new keys into the list (P:L219 step 4) =================
+    // position of a new key = its rank among the new keys + the number of
+    // list keys below it; position of a list key = its index + the number
+    // of new keys below it.  Keys are unique, so positions are unique; the
+    // first L positions form the new list (a merge, not a re-sort).
     {
       const int nk = C->nkeys;
       const int cnt = C->cnt;
       if (nk > 0) {
-        int P = 1;
-        while (P < nk) P <<= 1;
-        if (P <= 32) {
-          if (warp == 0) {
-            uint64_t v = (lane < nk) ? s.newk[lane] : kKeyMax;
-            v = warp_bitonic32(v, lane);
-            if (lane < nk) s.newk[lane] = v;
-          }
-          __syncthreads();
-        } else {
-          for (int i = nk + tid; i < P; i += NT) s.newk[i] = kKeyMax;
-          __syncthreads();
-          cta_bitonic<NT>(s.newk, P, tid);
-        }
-        const uint64_t* src = (cur ? s.list[1] : s.list[0]);
-        uint64_t* dst = (cur ? s.list[0] : s.list[1]);
+        const uint64_t* src = cur ? s.list[1] : s.list[0];
+        uint64_t* dst = cur ? s.list[0] : s.list[1];
         for (int i = tid; i < nk; i += NT) {
-          uint64_t key = s.newk[i];
-          int pos = i + lower_bound_u64(src, cnt, key);
+          const uint64_t key = s.newk[i];
+          int rn = 0;
+          for (int j = 0; j < nk; ++j) rn += (s.newk[j] < key) ? 1 : 0;
+          const int pos = rn + lower_bound_u64(src, cnt, key);
           if (pos < L) dst[pos] = key;
         }
         for (int j = tid; j < cnt; j += NT) {
-          uint64_t key = src[j];
-          int pos = j + lower_bound_u64(s.newk, nk, key);
+          const uint64_t key = src[j];
+          int rn = 0;
+          for (int i = 0; i < nk; ++i) rn += (s.newk[i] < key) ? 1 : 0;
+          const int pos = j + rn;
           if (pos < L) dst[pos] = key;
         }
         cur ^= 1;
         __syncthreads();
         if (tid == 0) {
-          int nc = cnt + nk;
+          const int nc = cnt + nk;
           C->cnt = nc < L ? nc : L;
         }
       }
       if (tid == 0) C->iters += (C->np > 0) ? 1 : 0;
       __syncthreads();
+      lap(3);
     }
   }
 
   // ================= publish the first k =================
   const int cnt = C->cnt;
+  const uint64_t* fin = cur ? s.list[1] : s.list[0];
   for (int i = tid; i < k; i += NT) {
     ResultEntry r;
     if (i < cnt) {
-      uint64_t key = (cur ? s.list[1] : s.list[0])[i];
+      uint64_t key = fin[i];
       r.id = key_id(key);
       r.dist = key_dist(key);
     } else {
@@ -513,13 +701,20 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     }
     out[i] = r;
   }
-  if (tid == 0 && st) {
-    st->iters = C->iters;
-    st->parents = C->parents;
-    st->dist_evals = C->dist_evals;
-    st->cap_hit = C->cap_hit;
-    st->spilled = C->spilled;
-    st->overflow = C->overflow;
+  if (tid == 0) {
+    C->phase = phase;
+    if (st) {
+      st->iters = C->iters;
+      st->parents = C->parents;
+      st->dist_evals = C->dist_evals;
+      st->cap_hit = C->cap_hit;
+      st->spilled = C->spilled;
+      st->overflow = C->overflow;
+      st->cyc_select = cyc[0];
+      st->cyc_gather = cyc[1];
+      st->cyc_dist = cyc[2];
+      st->cyc_sort = cyc[3];
+    }
   }
 }
 

@@ -64,9 +64,10 @@ struct BatchArgs {
 
 template <int NT, int TL, int CPL, int METRIC>
 __global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
-  extern __shared__ __align__(16) uint8_t smem_raw[];
-  const SmemLayout lay = smem_layout(a.cfg.d4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits);
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const SmemLayout lay = smem_layout(a.cfg.dp4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits, a.cfg.stage_rows);
   const Smem s = carve(smem_raw, lay);
+  init_cta<NT>(s, a.cfg);
   __shared__ int s_item;
   const int64_t total = a.nq * a.T;
   unsigned long long* gt = a.gtab ? a.gtab + ((uint64_t)blockIdx.x << a.cfg.gtab_bits) : nullptr;
@@ -97,9 +98,10 @@ constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
 
 template <int NT, int TL, int CPL, int METRIC>
 __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
-  extern __shared__ __align__(16) uint8_t smem_raw[];
-  const SmemLayout lay = smem_layout(A.cfg.d4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits);
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows);
   const Smem s = carve(smem_raw, lay);
+  init_cta<NT>(s, A.cfg);
   const PersistArgs& P = A.p;
   const int slot = blockIdx.x / P.T;
   const int rank = blockIdx.x % P.T;
@@ -247,28 +249,29 @@ struct KSel {
   static void* persist() { return (void*)persistent_kernel<NT, TL, CPL, M>; }
 };
 
-// chunk configs: (TL lanes per vector, CPL float4 chunks per lane)
-//   0:(8,3) d4<=24   1:(8,4) d4<=32   2:(16,4) d4<=64
-//   3:(32,4) d4<=128 4:(32,8) d4<=256 5:(32,16) d4<=512
+// chunk configs (TL lanes per vector, CPL float4 chunks per lane), see
+// chunk_tl()/chunk_cpl() in search_core.cuh
 int chunk_config_for(int d4) {
-  if (d4 <= 24) return 0;
-  if (d4 <= 32) return 1;
-  if (d4 <= 64) return 2;
-  if (d4 <= 128) return 3;
-  if (d4 <= 256) return 4;
-  if (d4 <= 512) return 5;
+  if (d4 <= 8) return 0;
+  if (d4 <= 16) return 1;
+  if (d4 <= 32) return 2;
+  if (d4 <= 64) return 3;
+  if (d4 <= 128) return 4;
+  if (d4 <= 256) return 5;
+  if (d4 <= 512) return 6;
   return -1;
 }
 
 template <int NT, int M>
 static void* pick_cc(int cc, bool persist) {
   switch (cc) {
-    case 0: return persist ? KSel<NT, 8, 3, M>::persist() : KSel<NT, 8, 3, M>::batch();
-    case 1: return persist ? KSel<NT, 8, 4, M>::persist() : KSel<NT, 8, 4, M>::batch();
-    case 2: return persist ? KSel<NT, 16, 4, M>::persist() : KSel<NT, 16, 4, M>::batch();
-    case 3: return persist ? KSel<NT, 32, 4, M>::persist() : KSel<NT, 32, 4, M>::batch();
-    case 4: return persist ? KSel<NT, 32, 8, M>::persist() : KSel<NT, 32, 8, M>::batch();
-    case 5: return persist ? KSel<NT, 32, 16, M>::persist() : KSel<NT, 32, 16, M>::batch();
+    case 0: return persist ? KSel<NT, 8, 1, M>::persist() : KSel<NT, 8, 1, M>::batch();
+    case 1: return persist ? KSel<NT, 16, 1, M>::persist() : KSel<NT, 16, 1, M>::batch();
+    case 2: return persist ? KSel<NT, 32, 1, M>::persist() : KSel<NT, 32, 1, M>::batch();
+    case 3: return persist ? KSel<NT, 32, 2, M>::persist() : KSel<NT, 32, 2, M>::batch();
+    case 4: return persist ? KSel<NT, 32, 4, M>::persist() : KSel<NT, 32, 4, M>::batch();
+    case 5: return persist ? KSel<NT, 32, 8, M>::persist() : KSel<NT, 32, 8, M>::batch();
+    case 6: return persist ? KSel<NT, 32, 16, M>::persist() : KSel<NT, 32, 16, M>::batch();
   }
   return nullptr;
 }
