@@ -87,6 +87,10 @@ typedef struct algas_params {
     int32_t slots;           /* persistent path: B query slots; 0 -> 32     */
     int32_t hash_bits;       /* log2 of the per-CTA shared-memory visited hash; 0 -> tuner */
     int32_t stage_rows;      /* vectors per shared-memory staging buffer (2 buffers); 0 -> tuner */
+    int32_t cluster_size;    /* persistent paths: CTAs (SMs) per search as a thread-block
+                                cluster sharing the distance gathers through DSMEM;
+                                1 = off, 2/4/8 (needs threads_per_cta = 256); 0 -> 1 */
+    int32_t reserved1;
     uint64_t seed;           /* entry-point generator seed (R5)                      */
 } algas_params;
 

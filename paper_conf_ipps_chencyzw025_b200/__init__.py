@@ -41,7 +41,8 @@ class Params(ctypes.Structure):
                 ("offset_beam", ctypes.c_int32), ("ctas_per_query", ctypes.c_int32),
                 ("threads_per_cta", ctypes.c_int32), ("n_seeds", ctypes.c_int32),
                 ("max_iter", ctypes.c_int32), ("visited_mode", ctypes.c_int32), ("slots", ctypes.c_int32),
-                ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32),
+                ("cluster_size", ctypes.c_int32), ("reserved1", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class QueryStats(ctypes.Structure):

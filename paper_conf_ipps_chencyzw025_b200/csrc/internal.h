@@ -60,7 +60,10 @@ struct Plan {
   int k;
   int visited_mode;
   int metric;
+  int cluster;     // CTAs per search (thread-block cluster), persistent paths
 };
+int max_active_clusters(const Plan& pl, int* out);
+int check_coresident(const Plan& pl, int slots);
 
 int chunk_config_for(int d4);          // -1 if unsupported
 

@@ -178,13 +178,9 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   s->kmax = s->plan.k;
   s->dim = idx->dim;
   s->d4 = idx->d4;
-  int nsm = 0, dev = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  if ((int64_t)slots * s->T > (int64_t)s->plan.blocks_per_sm * nsm) {
+  if ((rc = check_coresident(s->plan, slots))) {
     delete s;
-    return set_error(ALGAS_EINVAL, "%d slots x %d CTAs exceed co-resident capacity %d x %d SMs (P:L231)", slots,
-                     s->plan.T, s->plan.blocks_per_sm, nsm);
+    return rc;
   }
   auto cleanup = [&](int code) {
     algas_server_destroy(s);

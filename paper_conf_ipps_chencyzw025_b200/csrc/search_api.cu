@@ -96,7 +96,9 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   // Shared-memory budget per CTA: M_avail = M_per_SM / N_block_per_SM
   // - M_reserved, with N_block_per_SM from P:L235 for a persistent grid of
   // slots x T CTAs, or a target occupancy of 8 CTAs/SM for a static batch.
-  const int bps = persistent ? std::max(1, (int)(((int64_t)slots * T + nsm - 1) / nsm)) : 8;
+  const int cs = persistent ? (p->cluster_size > 0 ? p->cluster_size : 1) : 1;
+  if (cs != 1 && cs != 2 && cs != 4 && cs != 8) return set_error(ALGAS_EINVAL, "cluster_size %d not in {1,2,4,8}", cs);
+  const int bps = persistent ? std::max(1, (int)(((int64_t)slots * T * cs + nsm - 1) / nsm)) : 8;
   const int64_t budget = std::min<int64_t>((int64_t)smem_sm / bps - reserved, (int64_t)optin - reserved);
   // vector-gather path: 0 = LDG.128 into registers (default),
   // 1 = cp.async (LDGSTS) staging, 2 = cp.async.bulk staging; the staged
@@ -104,6 +106,7 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   const char* gm_env = getenv("ALGAS_GATHER_MODE");
   const int gather_mode = gm_env ? atoi(gm_env) : 0;
   if (gather_mode < 0 || gather_mode > 2) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0, 1 or 2");
+  if (cs > 1 && gather_mode != 0) return set_error(ALGAS_EINVAL, "cluster_size > 1 needs the register gather path");
   int hb = p->hash_bits, sr = gather_mode == 0 ? -1 : p->stage_rows;
   choose_smem(dp4, L, ncap, S, w, Rp, budget, &hb, &sr);
   if (hb < 6 || hb > 16) return set_error(ALGAS_EINVAL, "hash_bits %d not in [6,16]", hb);
@@ -120,6 +123,7 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   pl.smem = lay.total;
   pl.visited_mode = p->visited_mode;
   pl.metric = idx->metric;
+  pl.cluster = cs;
   SearchCfg& c = pl.cfg;
   c.data = reinterpret_cast<const float4*>(idx->d_data);
   c.graph = idx->d_graph;
@@ -158,6 +162,24 @@ static int num_sms() {
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
   return n;
+}
+
+// Every slot's searches must be co-resident for the persistent kernel to
+// make progress (Eq. P:L231 with the measured occupancy).
+int check_coresident(const Plan& pl, int slots) {
+  if (pl.cluster <= 1) {
+    if ((int64_t)slots * pl.T > (int64_t)pl.blocks_per_sm * num_sms())
+      return set_error(ALGAS_EINVAL, "%d slots x %d CTAs exceed co-resident capacity %d x %d SMs (P:L231)", slots,
+                       pl.T, pl.blocks_per_sm, num_sms());
+    return ALGAS_OK;
+  }
+  int nc = 0;
+  int rc = max_active_clusters(pl, &nc);
+  if (rc) return rc;
+  if ((int64_t)slots * pl.T > nc)
+    return set_error(ALGAS_EINVAL, "%d slots x %d searches exceed the %d co-resident %d-CTA clusters (P:L231)", slots,
+                     pl.T, nc, pl.cluster);
+  return ALGAS_OK;
 }
 
 // RAII device buffer on a stream
@@ -445,11 +467,9 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   Plan pl;
   int rc = make_plan(idx, params, slots, &pl, true);
   if (rc) return rc;
-  if ((int64_t)slots * pl.T > (int64_t)pl.blocks_per_sm * num_sms())
-    return set_error(ALGAS_EINVAL, "%d slots x %d CTAs exceed co-resident capacity %d x %d SMs (P:L231)", slots, pl.T,
-                     pl.blocks_per_sm, num_sms());
+  if ((rc = check_coresident(pl, slots))) return rc;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  const int ctas = slots * pl.T;
+  const int ctas = slots * pl.T * pl.cluster;
   const int64_t items = nq * pl.T;
 
   std::lock_guard<std::mutex> lk(idx->ws->mu);

@@ -24,6 +24,7 @@
 // implementation of the same paper passages.
 #pragma once
 
+#include <cooperative_groups.h>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -122,10 +123,12 @@ __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
 // Distance "chunk configs": TL lanes per vector, CPL 16-B chunks per lane.
 // A vector of d4 = dim/4 chunks is stored in shared memory padded to
 // dp4 = TL*CPL chunks (zero tail) so the distance loop needs no masks.
+// Four 16-B chunks per lane (64 B of a row) keep the shuffle tree short
+// (log2 TL levels) while a warp-wide load still covers whole 128-B lines.
 //   cc: 0      1      2      3      4       5       6
 //   d4: <=8   <=16   <=32   <=64   <=128   <=256   <=512
-__host__ __device__ inline int chunk_tl(int cc) { const int t[7] = {8, 16, 32, 32, 32, 32, 32}; return t[cc]; }
-__host__ __device__ inline int chunk_cpl(int cc) { const int t[7] = {1, 1, 1, 2, 4, 8, 16}; return t[cc]; }
+__host__ __device__ inline int chunk_tl(int cc) { const int t[7] = {2, 4, 8, 16, 32, 32, 32}; return t[cc]; }
+__host__ __device__ inline int chunk_cpl(int cc) { const int t[7] = {4, 4, 4, 4, 4, 8, 16}; return t[cc]; }
 __device__ __forceinline__ float4 ldg_f4_stream(const float4* p) {
   float4 r;
   // volatile: keeps every gather load of a pass ahead of the first use (the
@@ -171,6 +174,7 @@ struct Ctrl {
   int cnt, nnew, nkeys, np, done, diffusing, vis_count, spilled, overflow, cur;
   uint32_t iters, parents, dist_evals, cap_hit;
   uint32_t phase;  // bit b: parity of staging barrier b
+  uint64_t worst;  // prefilter key of the current step (read by cluster workers)
 };
 
 // Shared-memory carve-up (bytes, all 16-B aligned).
@@ -352,10 +356,123 @@ __device__ __forceinline__ void stage_issue(const SearchCfg& cfg, const Smem& s,
 }
 
 // ------------------------------------------------------------------ the search
+// ------------------------------------------------------------------ cluster helpers (CS > 1)
+// One search may be spread over a thread-block cluster of CS CTAs (one per
+// SM): CTA rank 0 (the leader) owns the candidate list and visited set and
+// runs select / gather / filter / merge; the distance step's vector gathers
+// are split over all CS CTAs, which read the step's ids from the leader's
+// shared memory and deliver keys into it through distributed shared memory.
+// A single SM sustains only ~10 GB/s of random 512-B row gathers
+// (profiles/gather_microbench.txt); CS SMs multiply the gather rate of one
+// query.
+__device__ __forceinline__ void cluster_barrier() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+template <typename T>
+__device__ __forceinline__ T* leader_ptr(T* local) {
+  // generic address of the same shared-memory object in cluster CTA 0
+  return cooperative_groups::this_cluster().map_shared_rank(local, 0);
+}
+
+// Distance step for rows r = r0, r0+rstep, ... < M of newid (P:L217 step 3):
+// LDG.128 straight into registers, each team keeping B rows in flight
+// (NT/TL*B rows per CTA), interleaved shuffle-tree reductions, prefilter
+// against `worst`, one warp-wide scan + one atomic per warp to append the
+// surviving keys to newk.  newid/newk/nkeys may live in another CTA's
+// shared memory (cluster leader).
+template <int NT, int TL, int CPL, int METRIC>
+__device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const QueryRegs<TL, CPL>& Q, int M, int r0, int rstep,
+                                         uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  constexpr int NTEAMS = NT / TL;
+  const int team = tid / TL, tl = tid % TL;
+  constexpr int B = CPL >= 16 ? 1 : 16 / CPL;
+  constexpr int PASS = NTEAMS * B;
+  const int Mc = M > r0 ? (M - r0 + rstep - 1) / rstep : 0;  // rows of this CTA
+  for (int base = 0; base < Mc; base += PASS) {
+    float4 v[B][CPL];
+    uint32_t ids[B];
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const int j = base + b * NTEAMS + team;
+      ids[b] = j < Mc ? newid[r0 + j * rstep] : 0u;
+    }
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const int j = base + b * NTEAMS + team;
+      const float4* row = cfg.data + (uint64_t)ids[b] * cfg.d4;
+#pragma unroll
+      for (int c = 0; c < CPL; ++c) {
+        const int chn = tl + c * TL;
+        v[b][c] = (j < Mc && chn < cfg.d4) ? ldg_f4_stream(row + chn) : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+    // all loads of the pass are issued before any use: the warp barrier
+    // keeps ptxas from hoisting FMAs of early rows between the loads
+    // (which would serialise the DRAM round trips)
+    __syncwarp();
+    // row groups of this pass that hold any row (uniform across the CTA):
+    // the FMA and shuffle work of empty groups is skipped
+    const int nb = (Mc - base + NTEAMS - 1) / NTEAMS;
+    float acc[B];
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      float a = 0.f;
+      if (b >= nb) {
+        acc[b] = 0.f;
+        continue;
+      }
+#pragma unroll
+      for (int c = 0; c < CPL; ++c) {
+        const float4 x = v[b][c];
+        if (METRIC == kL2) {
+          float d0 = Q.q[c].x - x.x, d1 = Q.q[c].y - x.y, d2 = Q.q[c].z - x.z, d3 = Q.q[c].w - x.w;
+          a = fmaf(d0, d0, a); a = fmaf(d1, d1, a); a = fmaf(d2, d2, a); a = fmaf(d3, d3, a);
+        } else {
+          a = fmaf(Q.q[c].x, x.x, a); a = fmaf(Q.q[c].y, x.y, a);
+          a = fmaf(Q.q[c].z, x.z, a); a = fmaf(Q.q[c].w, x.w, a);
+        }
+      }
+      acc[b] = a;
+    }
+#pragma unroll
+    for (int o = TL >> 1; o > 0; o >>= 1)
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+        if (b < nb) acc[b] += __shfl_xor_sync(0xffffffffu, acc[b], o);
+    uint64_t key[B];
+    int nkeep = 0;
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const int j = base + b * NTEAMS + team;
+      key[b] = kKeyMax;
+      if (tl == 0 && j < Mc) key[b] = make_key((METRIC == kL2) ? acc[b] : -acc[b], ids[b]);
+      nkeep += (key[b] < worst) ? 1 : 0;
+    }
+    int incl = nkeep;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
+    }
+    const int wtotal = __shfl_sync(0xffffffffu, incl, 31);
+    if (wtotal > 0) {
+      int wbase = 0;
+      if (lane == 0) wbase = atomicAdd(nkeys, wtotal);
+      wbase = __shfl_sync(0xffffffffu, wbase, 0);
+      int pos = wbase + incl - nkeep;
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+        if (key[b] < worst) newk[pos++] = key[b];
+    }
+  }
+}
+
 // Preconditions: s.q holds the query (d4 float4, zero tail); init_cta() ran.
 // Writes min(k, |list|) results to out[0..k) (rest padded) and the CTA's
-// counters to *st.
-template <int NT, int TL, int CPL, int METRIC>
+// counters to *st.  CS > 1: this CTA is the leader of a cluster whose
+// other CTAs run search_worker() in lock step (two cluster barriers per step).
+template <int NT, int TL, int CPL, int METRIC, int CS = 1>
 __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, uint32_t cta_rank, int k,
                            unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st) {
   const int tid = threadIdx.x;
@@ -426,15 +543,21 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       if (warp == 0) {
         const int cnt = C->cnt;
         uint64_t* list = cur ? s.list[1] : s.list[0];
+        // also look past the parents: the next few unchecked candidates are
+        // the likely parents of the next step, whose graph rows are
+        // prefetched into L2 now (prefetch bit 1; results are unaffected)
+        const int pf = (cfg.prefetch & 2) ? (cfg.w < 16 ? cfg.w : 32 - cfg.w) : 0;
+        const int want = cfg.w + pf;
         int found = 0;
-        for (int base = 0; base < cnt && found < cfg.w; base += 32) {
+        for (int base = 0; base < cnt && found < want; base += 32) {
           int i = base + lane;
           bool un = (i < cnt) && !(list[i] & 1ull);
           unsigned m = __ballot_sync(0xffffffffu, un);
           int rank = found + __popc(m & ((1u << lane) - 1u));
-          if (un && rank < cfg.w) s.sel[rank] = i;
+          if (un && rank < want) s.sel[rank] = i;
           found += __popc(m);
         }
+        const int found_all = found < want ? found : want;
         if (found > cfg.w) found = cfg.w;
         __syncwarp();
         int done = 0, np = 0;
@@ -452,6 +575,11 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
             uint64_t kk = list[pos];
             list[pos] = kk | 1ull;                    // mark checked (Alg.1 l.7)
             s.sel[32 + lane] = (int)key_id(kk);
+          } else if (lane < found_all) {
+            const uint32_t nid = key_id(list[s.sel[lane]]);
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)nid << cfg.rp_shift)),
+                         "r"(4u << cfg.rp_shift)
+                         : "memory");
           }
           if (lane == 0) C->diffusing = diff;
         }
@@ -467,7 +595,10 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       }
       __syncthreads();
       lap(0);
-      if (C->done) break;
+      if (C->done) {
+        if constexpr (CS > 1) cluster_barrier();  // B: workers see done and leave
+        break;
+      }
 
       // ================= gather + visited filter (P:L217 steps 1-2) =================
       {
@@ -493,7 +624,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
               if (r == kVisFull) atomicOr(&C->overflow, 1);
             }
           }
-          if (keep && cfg.prefetch == 1) {
+          if (keep && (cfg.prefetch & 1)) {
             asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.data + (uint64_t)id * cfg.d4),
                          "r"((uint32_t)cfg.d4 * 16u)
                          : "memory");
@@ -519,77 +650,16 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       const int cnt = C->cnt;
       const uint64_t worst = (cnt >= L) ? (cur ? s.list[1] : s.list[0])[L - 1] : kKeyMax;
       if (cfg.gather_mode == 0) {
-        // LDG.128 straight into registers: each team keeps B rows in flight
-        // (NT/TL*B rows per CTA), then reduces them with interleaved shuffle
-        // trees.  The measured single-SM random-gather rate of this path is
-        // 2-3x that of the async-copy paths (profiles/gather_microbench.txt).
-        constexpr int B = CPL >= 16 ? 1 : 16 / CPL;
-        constexpr int PASS = NTEAMS * B;
-        for (int base = 0; base < M; base += PASS) {
-          float4 v[B][CPL];
-#pragma unroll
-          for (int b = 0; b < B; ++b) {
-            const int r = base + b * NTEAMS + team;
-            const float4* row = cfg.data + (uint64_t)(r < M ? s.newid[r] : 0u) * cfg.d4;
-#pragma unroll
-            for (int c = 0; c < CPL; ++c) {
-              const int chn = tl + c * TL;
-              v[b][c] = (r < M && chn < cfg.d4) ? ldg_f4_stream(row + chn) : make_float4(0.f, 0.f, 0.f, 0.f);
-            }
-          }
-          // all loads of the pass are issued before any use: the warp barrier
-          // keeps ptxas from hoisting FMAs of early rows between the loads
-          // (which would serialise the DRAM round trips)
-          __syncwarp();
-          float acc[B];
-#pragma unroll
-          for (int b = 0; b < B; ++b) {
-            float a = 0.f;
-#pragma unroll
-            for (int c = 0; c < CPL; ++c) {
-              const float4 x = v[b][c];
-              if (METRIC == kL2) {
-                float d0 = Q.q[c].x - x.x, d1 = Q.q[c].y - x.y, d2 = Q.q[c].z - x.z, d3 = Q.q[c].w - x.w;
-                a = fmaf(d0, d0, a); a = fmaf(d1, d1, a); a = fmaf(d2, d2, a); a = fmaf(d3, d3, a);
-              } else {
-                a = fmaf(Q.q[c].x, x.x, a); a = fmaf(Q.q[c].y, x.y, a);
-                a = fmaf(Q.q[c].z, x.z, a); a = fmaf(Q.q[c].w, x.w, a);
-              }
-            }
-            acc[b] = a;
-          }
-#pragma unroll
-          for (int o = TL >> 1; o > 0; o >>= 1)
-#pragma unroll
-            for (int b = 0; b < B; ++b) acc[b] += __shfl_xor_sync(0xffffffffu, acc[b], o);
-          // keys of this pass; one warp-wide scan + one atomic per warp
-          uint64_t key[B];
-          int nkeep = 0;
-#pragma unroll
-          for (int b = 0; b < B; ++b) {
-            const int r = base + b * NTEAMS + team;
-            key[b] = kKeyMax;
-            if (tl == 0 && r < M) key[b] = make_key((METRIC == kL2) ? acc[b] : -acc[b], s.newid[r]);
-            nkeep += (key[b] < worst) ? 1 : 0;
-          }
-          int incl = nkeep;
-#pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {
-            const int t = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += t;
-          }
-          const int wtotal = __shfl_sync(0xffffffffu, incl, 31);
-          if (wtotal > 0) {
-            int wbase = 0;
-            if (lane == 0) wbase = atomicAdd(&C->nkeys, wtotal);
-            wbase = __shfl_sync(0xffffffffu, wbase, 0);
-            int pos = wbase + incl - nkeep;
-#pragma unroll
-            for (int b = 0; b < B; ++b)
-              if (key[b] < worst) s.newk[pos++] = key[b];
-          }
+        if constexpr (CS > 1) {
+          // B: publish the step (newid[0..M), worst) to the cluster workers
+          if (tid == 0) C->worst = worst;
+          cluster_barrier();
+          dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
+          cluster_barrier();  // C: every CTA's keys delivered into newk
+        } else {
+          dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, 1, worst, s.newid, s.newk, &C->nkeys);
+          __syncthreads();
         }
-        __syncthreads();
       }
       const int SR = cfg.stage_rows;
       const int nchunks = cfg.gather_mode == 0 ? 0 : (M + SR - 1) / SR;
@@ -715,6 +785,27 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       st->cyc_dist = cyc[2];
       st->cyc_sort = cyc[3];
     }
+  }
+}
+
+// Cluster worker (CTA rank crank > 0): mirrors the leader's two cluster
+// barriers per step and evaluates its share (rows crank, crank+CS, ...) of
+// every distance step, reading ids from and delivering keys into the
+// leader's shared memory.  Preconditions: s.q holds the query.
+template <int NT, int TL, int CPL, int METRIC, int CS>
+__device__ void search_worker(const SearchCfg& cfg, const Smem& s, int crank) {
+  QueryRegs<TL, CPL> Q;
+  Q.load(s.q, threadIdx.x % TL);
+  Ctrl* LC = leader_ptr(s.ctrl);
+  const uint32_t* lnewid = leader_ptr(s.newid);
+  uint64_t* lnewk = leader_ptr(s.newk);
+  for (;;) {
+    cluster_barrier();  // B
+    if (*((volatile int*)&LC->done)) break;
+    const int M = *((volatile int*)&LC->nnew);
+    const uint64_t worst = *((volatile uint64_t*)&LC->worst);
+    dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, crank, CS, worst, lnewid, lnewk, &LC->nkeys);
+    cluster_barrier();  // C
   }
 }
 

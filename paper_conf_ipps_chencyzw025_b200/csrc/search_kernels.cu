@@ -96,20 +96,43 @@ struct PKArgs {
 
 constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
 
-template <int NT, int TL, int CPL, int METRIC>
+template <int NT, int TL, int CPL, int METRIC, int CS>
 __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows);
   const Smem s = carve(smem_raw, lay);
   init_cta<NT>(s, A.cfg);
   const PersistArgs& P = A.p;
-  const int slot = blockIdx.x / P.T;
-  const int rank = blockIdx.x % P.T;
+  // a search unit = one (slot, cta_rank) search = one cluster of CS CTAs
+  const int unit = blockIdx.x / CS;
+  const int crank = blockIdx.x % CS;  // rank inside the cluster (1-D clusters)
+  const int slot = unit / P.T;
+  const int rank = unit % P.T;
   const int tid = threadIdx.x;
-  unsigned long long* gt = P.gtab ? P.gtab + ((uint64_t)blockIdx.x << A.cfg.gtab_bits) : nullptr;
   __shared__ unsigned long long s_mbox;
   __shared__ int4 s_par;
   __shared__ unsigned long long s_tag, s_t0;
+
+  if constexpr (CS > 1) {
+    if (crank != 0) {
+      // cluster worker: follow the leader query by query (barrier A)
+      const unsigned long long* lmb = leader_ptr(&s_mbox);
+      const float4* lq = leader_ptr(s.q);
+      for (;;) {
+        cluster_barrier();  // A: leader staged the next query (or quit)
+        if (*((volatile unsigned long long*)lmb) == kMboxQuit) {
+          cluster_barrier();  // Z: the leader's shared memory outlives our last read
+          return;
+        }
+        for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = lq[i];
+        __syncthreads();
+        search_worker<NT, TL, CPL, METRIC, CS>(A.cfg, s, crank);
+        __syncthreads();
+      }
+    }
+  }
+
+  unsigned long long* gt = P.gtab ? P.gtab + ((uint64_t)unit << A.cfg.gtab_bits) : nullptr;
   uint32_t served = 0;  // queries this CTA has finished (= last epoch in devq mode)
   uint32_t last_epoch = 0;
 
@@ -185,7 +208,13 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
       __syncthreads();
     }
     const unsigned long long mb = s_mbox;
-    if (mb == kMboxQuit) break;
+    if (mb == kMboxQuit) {
+      if constexpr (CS > 1) {
+        cluster_barrier();  // A: release the workers
+        cluster_barrier();  // Z: they have read the quit word
+      }
+      break;
+    }
     const uint32_t epoch = (uint32_t)(mb >> 32);
     const uint32_t item = (uint32_t)mb;
     if (tid == 0) {
@@ -202,6 +231,7 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
                                        : P.queries + (uint64_t)item * A.cfg.d4;
     for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = (P.mode == 0) ? ld_volatile_f4(qsrc + i) : qsrc[i];
     __syncthreads();
+    if constexpr (CS > 1) cluster_barrier();  // A: workers copy the query
 
     SearchCfg cfg = A.cfg;
     cfg.L = par.y;
@@ -218,8 +248,8 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
       stp = P.dq_stats + (uint64_t)item * P.T + rank;
     }
     CtaStats local;
-    search_cta<NT, TL, CPL, METRIC>(cfg, s, tag, (uint32_t)rank, k, gt,
-                                    P.epoch_base + served, out, &local);
+    search_cta<NT, TL, CPL, METRIC, CS>(cfg, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
+                                        &local);
     __syncthreads();
     if (tid == 0) {
       local.t_start = s_t0;
@@ -243,12 +273,6 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
 }
 
 // ------------------------------------------------------------------ dispatch
-template <int NT, int TL, int CPL, int M>
-struct KSel {
-  static void* batch() { return (void*)batch_kernel<NT, TL, CPL, M>; }
-  static void* persist() { return (void*)persistent_kernel<NT, TL, CPL, M>; }
-};
-
 // chunk configs (TL lanes per vector, CPL float4 chunks per lane), see
 // chunk_tl()/chunk_cpl() in search_core.cuh
 int chunk_config_for(int d4) {
@@ -262,40 +286,76 @@ int chunk_config_for(int d4) {
   return -1;
 }
 
+template <int NT, int TL, int CPL, int M>
+static void* sel_kernel(bool persist, int cs) {
+  if (!persist) return (void*)batch_kernel<NT, TL, CPL, M>;
+  switch (cs) {
+    case 1: return (void*)persistent_kernel<NT, TL, CPL, M, 1>;
+    // cluster-split searches: instantiated for the 256-thread configuration only
+    case 2: return NT == 256 ? (void*)persistent_kernel<NT, TL, CPL, M, (NT == 256 ? 2 : 1)> : nullptr;
+    case 4: return NT == 256 ? (void*)persistent_kernel<NT, TL, CPL, M, (NT == 256 ? 4 : 1)> : nullptr;
+    case 8: return NT == 256 ? (void*)persistent_kernel<NT, TL, CPL, M, (NT == 256 ? 8 : 1)> : nullptr;
+  }
+  return nullptr;
+}
 template <int NT, int M>
-static void* pick_cc(int cc, bool persist) {
+static void* pick_cc(int cc, bool persist, int cs) {
   switch (cc) {
-    case 0: return persist ? KSel<NT, 8, 1, M>::persist() : KSel<NT, 8, 1, M>::batch();
-    case 1: return persist ? KSel<NT, 16, 1, M>::persist() : KSel<NT, 16, 1, M>::batch();
-    case 2: return persist ? KSel<NT, 32, 1, M>::persist() : KSel<NT, 32, 1, M>::batch();
-    case 3: return persist ? KSel<NT, 32, 2, M>::persist() : KSel<NT, 32, 2, M>::batch();
-    case 4: return persist ? KSel<NT, 32, 4, M>::persist() : KSel<NT, 32, 4, M>::batch();
-    case 5: return persist ? KSel<NT, 32, 8, M>::persist() : KSel<NT, 32, 8, M>::batch();
-    case 6: return persist ? KSel<NT, 32, 16, M>::persist() : KSel<NT, 32, 16, M>::batch();
+    case 0: return sel_kernel<NT, 2, 4, M>(persist, cs);
+    case 1: return sel_kernel<NT, 4, 4, M>(persist, cs);
+    case 2: return sel_kernel<NT, 8, 4, M>(persist, cs);
+    case 3: return sel_kernel<NT, 16, 4, M>(persist, cs);
+    case 4: return sel_kernel<NT, 32, 4, M>(persist, cs);
+    case 5: return sel_kernel<NT, 32, 8, M>(persist, cs);
+    case 6: return sel_kernel<NT, 32, 16, M>(persist, cs);
   }
   return nullptr;
 }
 template <int NT>
-static void* pick_metric(int metric, int cc, bool persist) {
-  return metric == kL2 ? pick_cc<NT, kL2>(cc, persist) : pick_cc<NT, kIP>(cc, persist);
+static void* pick_metric(int metric, int cc, bool persist, int cs) {
+  return metric == kL2 ? pick_cc<NT, kL2>(cc, persist, cs) : pick_cc<NT, kIP>(cc, persist, cs);
 }
 static void* kernel_for(const Plan& pl, int metric, bool persist) {
+  const int cs = persist ? pl.cluster : 1;
   switch (pl.nt) {
-    case 32: return pick_metric<32>(metric, pl.ccfg, persist);
-    case 64: return pick_metric<64>(metric, pl.ccfg, persist);
-    case 128: return pick_metric<128>(metric, pl.ccfg, persist);
-    case 256: return pick_metric<256>(metric, pl.ccfg, persist);
+    case 32: return pick_metric<32>(metric, pl.ccfg, persist, cs);
+    case 64: return pick_metric<64>(metric, pl.ccfg, persist, cs);
+    case 128: return pick_metric<128>(metric, pl.ccfg, persist, cs);
+    case 256: return pick_metric<256>(metric, pl.ccfg, persist, cs);
   }
   return nullptr;
 }
 
 int max_blocks_per_sm(const Plan& pl, bool persistent, int* out) {
   void* fn = kernel_for(pl, pl.metric, persistent);
-  if (!fn) return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d", pl.nt, pl.ccfg);
+  if (!fn)
+    return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d cluster=%d (cluster > 1 needs 256 threads)",
+                     pl.nt, pl.ccfg, pl.cluster);
   ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
   int nb = 0;
   ALGAS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, pl.nt, pl.smem));
   *out = nb;
+  return ALGAS_OK;
+}
+
+int max_active_clusters(const Plan& pl, int* out) {
+  void* fn = kernel_for(pl, pl.metric, true);
+  if (!fn) return set_error(ALGAS_EINVAL, "no persistent kernel for cluster=%d", pl.cluster);
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(pl.cluster);
+  cfg.blockDim = dim3(pl.nt);
+  cfg.dynamicSmemBytes = pl.smem;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = pl.cluster;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  int n = 0;
+  ALGAS_CUDA_TRY(cudaOccupancyMaxActiveClusters(&n, fn, &cfg));
+  *out = n;
   return ALGAS_OK;
 }
 
@@ -323,20 +383,40 @@ int launch_batch(const Plan& pl, const BatchLaunch& bl, cudaStream_t st) {
 
 int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st) {
   void* fn = kernel_for(pl, pl.metric, true);
-  if (!fn) return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d", pl.nt, pl.ccfg);
+  if (!fn) return set_error(ALGAS_EINVAL, "no kernel for threads=%d chunk=%d cluster=%d", pl.nt, pl.ccfg, pl.cluster);
   ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
   PKArgs A;
   A.cfg = pl.cfg;
   A.p = pa;
   void* args[] = {&A};
   // cooperative launch: the runtime refuses a grid that cannot be fully
-  // co-resident, which a persistent kernel needs for forward progress
-  cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(pa.slots * pa.T), dim3(pl.nt), args, pl.smem, st);
+  // co-resident, which a persistent kernel needs for forward progress;
+  // cluster dimension = the CTAs of one cluster-split search
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(pa.slots * pa.T * pl.cluster);
+  cfg.blockDim = dim3(pl.nt);
+  cfg.dynamicSmemBytes = pl.smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  int na = 0;
+  at[na].id = cudaLaunchAttributeCooperative;
+  at[na].val.cooperative = 1;
+  ++na;
+  if (pl.cluster > 1) {
+    at[na].id = cudaLaunchAttributeClusterDimension;
+    at[na].val.clusterDim.x = pl.cluster;
+    at[na].val.clusterDim.y = 1;
+    at[na].val.clusterDim.z = 1;
+    ++na;
+  }
+  cfg.attrs = at;
+  cfg.numAttrs = na;
+  cudaError_t e = cudaLaunchKernelExC(&cfg, fn, args);
   if (e != cudaSuccess) {
     (void)cudaGetLastError();
     return set_error(e == cudaErrorCooperativeLaunchTooLarge ? ALGAS_EINVAL : ALGAS_ECUDA,
-                     "persistent launch (%d slots x %d CTAs x %d threads, %d B smem) failed: %s", pa.slots,
-                     pa.T, pl.nt, pl.smem, cudaGetErrorString(e));
+                     "persistent launch (%d slots x %d searches x %d-CTA clusters x %d threads, %d B smem) failed: %s",
+                     pa.slots, pa.T, pl.cluster, pl.nt, pl.smem, cudaGetErrorString(e));
   }
   return ALGAS_OK;
 }

@@ -69,13 +69,20 @@ def main():
     for L in Ls:
         for (wd, T, nt) in [(1, 1, 64), (4, 1, 64), (4, 1, 128), (4, 4, 64), (2, 8, 64), (4, 8, 64)]:
             grid.append((L, wd, T, nt))
-    if a.quick:
-        grid = [(64, 4, 1, 64), (64, 4, 1, 128), (64, 4, 1, 256), (64, 1, 1, 256), (64, 8, 1, 256),
-                (64, 4, 4, 256), (64, 4, 4, 128), (128, 4, 1, 256)]
-    for (L, wd, T, nt) in grid:
+    if os.environ.get("GRID") == "pf":
+        grid = [(64, 4, 1, 256, 1), (64, 8, 1, 256, 1), (64, 4, 2, 256, 1), (56, 4, 2, 256, 1), (48, 4, 4, 256, 1),
+                (56, 4, 4, 256, 1), (64, 4, 1, 128, 1)]
+    elif os.environ.get("GRID") == "cs":
+        grid = [(64, 4, 1, 256, 1), (64, 4, 1, 256, 4), (64, 8, 1, 256, 4), (64, 8, 1, 256, 8)]
+    elif a.quick:
+        grid = [(64, 4, 1, 256, 1), (64, 4, 1, 256, 2), (64, 4, 1, 256, 4), (64, 8, 1, 256, 4),
+                (64, 4, 2, 256, 2), (48, 4, 2, 256, 2), (48, 4, 4, 256, 1), (64, 8, 1, 256, 2),
+                (128, 8, 1, 256, 4), (64, 2, 1, 256, 4)]
+    grid = [g if len(g) == 5 else g + (1,) for g in grid]
+    for (L, wd, T, nt, cs) in grid:
         for slots in ([32] if not a.quick else [32]):
             p = algas.default_params(k=w.k, itopk=L, width=wd, offset_beam=max(1, L // 4), ctas_per_query=T,
-                                     threads_per_cta=nt, slots=slots, n_seeds=32, seed=1)
+                                     threads_per_cta=nt, slots=slots, n_seeds=32, seed=1, cluster_size=cs)
             try:
                 r = idx.search_dynamic(Qd, p)
             except algas.AlgasError as e:
@@ -85,7 +92,7 @@ def main():
             st = r["stats"]
             lat = (st["t_end_ns"] - st["t_start_ns"]) / 1e3
             rec = recall(r["ids"], ti, w.k)
-            row = dict(L=L, w=wd, T=T, threads=nt, slots=slots, recall=rec, qps=a.nq / (ms / 1e3),
+            row = dict(L=L, w=wd, T=T, threads=nt, cs=cs, slots=slots, recall=rec, qps=a.nq / (ms / 1e3),
                        kernel_ms=ms, lat_p50_us=float(np.percentile(lat, 50)),
                        lat_p99_us=float(np.percentile(lat, 99)), iters=float(st["iters"].mean() / T),
                        dist_evals=float(st["dist_evals"].mean()), spills=int((st["spills"] > 0).sum()),

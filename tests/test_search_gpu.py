@@ -256,6 +256,48 @@ def test_dynamic_queue_equals_batch(slots, T):
     assert (d["stats"]["t_end_ns"] >= d["stats"]["t_start_ns"]).all()
 
 
+@pytest.mark.parametrize("cs", [2, 4, 8])
+@pytest.mark.parametrize("metric,d", [(algas.L2, 128), (algas.IP, 100), (algas.L2, 960)])
+def test_cluster_split_equals_batch(cs, metric, d):
+    """One search spread over a cluster of cs CTAs (DSMEM) computes the same
+    distances and the same set of keys per step: bitwise equal to the
+    single-CTA batch path (and hence to the oracle on lattice data)."""
+    X, Q, G = lattice_case(2000, d, metric, 32, seed=310 + d)
+    p = algas.default_params(k=10, itopk=48, width=4, offset_beam=8, n_seeds=16, ctas_per_query=2,
+                             threads_per_cta=256, slots=5, seed=3)
+    idx = algas.Index(X, G, metric)
+    b = idx.search(Q, params=p, tag0=7)
+    pc = algas.default_params(k=10, itopk=48, width=4, offset_beam=8, n_seeds=16, ctas_per_query=2,
+                              threads_per_cta=256, slots=5, seed=3, cluster_size=cs)
+    d_ = idx.search_dynamic(_torch_cuda(Q), pc, tag0=7)
+    np.testing.assert_array_equal(d_["ids"], b["ids"])
+    np.testing.assert_array_equal(_bits(d_["dists"]), _bits(b["dists"]))
+    np.testing.assert_array_equal(d_["stats"]["dist_evals"], b["stats"]["dist_evals"])
+    oi, od, ost = oracle.search(X, G, Q, _oracle_params(p), metric=metric, tag0=7)
+    np.testing.assert_array_equal(d_["ids"], oi)
+
+
+def test_cluster_server_equals_batch():
+    X, Q, G = lattice_case(2000, 128, algas.L2, 32, seed=320)
+    p = algas.default_params(k=10, itopk=48, width=4, offset_beam=8, n_seeds=16, ctas_per_query=1,
+                             threads_per_cta=256, slots=6, seed=5, cluster_size=4)
+    idx = algas.Index(X, G)
+    b = idx.search(Q, params=algas.default_params(k=10, itopk=48, width=4, offset_beam=8, n_seeds=16,
+                                                  ctas_per_query=1, threads_per_cta=256, seed=5))
+    got = {}
+    with algas.Server(idx, p) as srv:
+        pending = list(range(Q.shape[0]))
+        t0 = time.time()
+        while (pending or srv.inflight() > 0) and time.time() - t0 < 60:
+            while pending and srv.submit(Q[pending[0]], tag=pending[0]):
+                pending.pop(0)
+            for t, i, dd, st in zip(*srv.poll(64)):
+                got[int(t)] = i.copy()
+    assert len(got) == Q.shape[0]
+    for t in range(Q.shape[0]):
+        np.testing.assert_array_equal(got[t], b["ids"][t])
+
+
 @pytest.mark.parametrize("slots,T", [(1, 1), (8, 2), (32, 1)])
 def test_server_equals_batch(slots, T):
     X, Q, G = lattice_case(2000, 128, algas.L2, 32, seed=301)
