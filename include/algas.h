@@ -223,6 +223,12 @@ int algas_server_destroy(algas_server *s);
  * the number of real entries written. */
 int32_t algas_merge_topk(const uint32_t *ids, const float *dists, int32_t m, int32_t k,
                          uint32_t *out_ids, float *out_dists);
+/* Row-wise batch form for the sharded layout: nq independent merges of the
+ * entries ids[p*stride_part + q*m_per + j] (parts p < nparts, j < m_per):
+ * the per-shard [nparts][nq][m_per] results of an all-gather.  HOST arrays;
+ * out_ids / out_dists: nq x k.  Returns ALGAS_OK or ALGAS_EINVAL. */
+int algas_merge_topk_parts(const uint32_t *ids, const float *dists, int32_t nparts, int64_t nq,
+                           int32_t m_per, int32_t k, uint32_t *out_ids, float *out_dists);
 
 /* ------------------------------------------------------------------ */
 /* Adaptive tuning.                                        */

@@ -27,7 +27,7 @@ VISITED_SHARED = 1
 OK, EINVAL, ENOMEM, ECUDA, EAGAIN, ESTATE, ENCCL, EOVERFLOW = 0, -1, -2, -3, -4, -5, -6, -7
 
 __all__ = ["Index", "Server", "Params", "QueryStats", "RunInfo", "lib", "knn", "prune", "build_graph",
-           "merge_topk", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP"]
+           "merge_topk", "merge_topk_parts", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP"]
 
 
 class AlgasError(RuntimeError):
@@ -84,7 +84,7 @@ class Tuning(ctypes.Structure):
 EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_index_create",
            "algas_index_destroy", "algas_index_info", "algas_search", "algas_search_ex", "algas_search_dynamic",
            "algas_server_create", "algas_submit", "algas_poll", "algas_server_inflight", "algas_server_destroy",
-           "algas_merge_topk", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
+           "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_prune", "algas_build_graph"]
 
 _lock = threading.Lock()
@@ -123,6 +123,7 @@ def lib(build_if_missing: bool = True):
         L.algas_server_destroy.argtypes = [P]
         L.algas_merge_topk.argtypes = [P, P, i32, i32, P, P]
         L.algas_merge_topk.restype = i32
+        L.algas_merge_topk_parts.argtypes = [P, P, i32, i64, i32, i32, P, P]
         L.algas_device_query.argtypes = [ctypes.POINTER(DeviceProps)]
         L.algas_tuner_max_parallel.argtypes = [i32, i32, i32]
         L.algas_tuner_max_parallel.restype = i32
@@ -367,6 +368,17 @@ def merge_topk(ids, dists, k: int):
     if n < 0:
         _check(n)
     return oi, od, n
+
+
+def merge_topk_parts(ids, dists, k: int):
+    """Host merge of per-part sorted rows: ids/dists [nparts, nq, m] -> [nq, k]."""
+    ids = np.ascontiguousarray(ids, np.uint32)
+    dists = np.ascontiguousarray(dists, np.float32)
+    P_, nq, m = ids.shape
+    oi = np.empty((nq, k), np.uint32)
+    od = np.empty((nq, k), np.float32)
+    _check(lib().algas_merge_topk_parts(_ptr(ids)[0], _ptr(dists)[0], P_, nq, m, k, _ptr(oi)[0], _ptr(od)[0]))
+    return oi, od
 
 
 def device_props() -> DeviceProps:

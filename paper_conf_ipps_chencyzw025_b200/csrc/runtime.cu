@@ -365,6 +365,23 @@ int32_t algas_merge_topk(const uint32_t* ids, const float* dists, int32_t m, int
   return merge_cta_lists(one.data(), 1, (int)all.size() + 1, k, out_ids, out_dists);
 }
 
+int algas_merge_topk_parts(const uint32_t* ids, const float* dists, int32_t nparts, int64_t nq, int32_t m_per,
+                           int32_t k, uint32_t* out_ids, float* out_dists) {
+  if (!ids || !dists || !out_ids || !out_dists || nparts < 1 || nq < 0 || m_per < 1 || k < 1)
+    return set_error(ALGAS_EINVAL, "algas_merge_topk_parts: bad arguments");
+  // each part's row is sorted (a shard's TopK): the T-way heap merge applies
+  std::vector<ResultEntry> rows((size_t)nparts * m_per);
+  for (int64_t q = 0; q < nq; ++q) {
+    for (int p = 0; p < nparts; ++p)
+      for (int j = 0; j < m_per; ++j) {
+        const size_t src = ((size_t)p * nq + q) * m_per + j;
+        rows[(size_t)p * m_per + j] = ResultEntry{ids[src], dists[src]};
+      }
+    merge_cta_lists(rows.data(), nparts, m_per, k, out_ids + q * k, out_dists + q * k);
+  }
+  return ALGAS_OK;
+}
+
 // ------------------------------------------------------------------ tuner
 int32_t algas_tuner_max_parallel(int32_t slots, int32_t n_sm, int32_t max_blocks_per_sm) {
   if (slots < 1) return 0;

@@ -342,3 +342,33 @@ def test_server_smaller_per_query_params_and_rejects():
     b = idx.search(Q[:1], params=p5, tag0=1)
     np.testing.assert_array_equal(ids[:5], b["ids"][0])
     assert np.all(ids[5:] == SENT)
+
+
+def test_sharded_index_nccl_world1_equals_index():
+    """Shard layout over NCCL with world_size 1 (the degenerate single-GPU
+    case): exchange + merge must leave the local answer unchanged."""
+    import os
+    import socket
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_chencyzw025_b200 import shard
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=330)
+    p = algas.default_params(k=10, itopk=32, width=2, offset_beam=8, n_seeds=8, ctas_per_query=2,
+                             threads_per_cta=128, seed=2)
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        si = shard.ShardedIndex(X, 0, G)
+        r = si.search(Q, p, device=torch.device("cuda", 0))
+    finally:
+        dist.destroy_process_group()
+    b = algas.Index(X, G).search(Q, params=p)
+    np.testing.assert_array_equal(r["ids"], b["ids"])
+    np.testing.assert_array_equal(r["dists"], b["dists"])
