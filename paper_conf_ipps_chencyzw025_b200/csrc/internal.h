@@ -33,6 +33,10 @@ struct Workspace {
   size_t gtab_entries = 0;
   int* counters = nullptr;             // small device scratch (work counters ...)
   uint32_t epoch = 1;                  // next epoch for the spill tables
+  void* h_res = nullptr;               // pinned staging of per-CTA results
+  size_t h_res_bytes = 0;
+  void* h_st = nullptr;                // pinned staging of per-CTA counters
+  size_t h_st_bytes = 0;
 };
 
 }  // namespace algas

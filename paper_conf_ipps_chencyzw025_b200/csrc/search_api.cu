@@ -5,6 +5,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
+#include <thread>
 #include <vector>
 
 #include "internal.h"
@@ -197,9 +198,29 @@ struct DevBuf {
 };
 
 // Host merge of nq x T x k per-CTA lists into the caller's outputs.
-static int finish_outputs(const std::vector<ResultEntry>& res, const std::vector<CtaStats>& cst, int64_t nq,
-                          int T, int kin, int k, uint32_t* out_ids, float* out_dists, uint32_t* out_cta_ids,
-                          float* out_cta_dists, algas_query_stats* out_stats, bool* overflow) {
+// run f(lo, hi) over [0, n) on up to 16 host threads (serial for small n)
+template <typename F>
+static void parallel_for(int64_t n, int64_t grain, F f) {
+  const int hw = (int)std::max(1u, std::thread::hardware_concurrency());
+  const int nt = (int)std::min<int64_t>(std::min(16, hw), (n + grain - 1) / grain);
+  if (nt <= 1) {
+    f((int64_t)0, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  const int64_t chunk = (n + nt - 1) / nt;
+  for (int t = 0; t < nt; ++t) {
+    const int64_t lo = t * chunk, hi = std::min(n, lo + chunk);
+    if (lo < hi) th.emplace_back([=] { f(lo, hi); });
+  }
+  for (auto& x : th) x.join();
+}
+
+// Host TopK merge of nq x T x kin per-CTA lists into the caller's
+// outputs, plus per-query counters; parallel over queries.
+static int finish_outputs(const ResultEntry* res, const CtaStats* cst, int64_t nq, int T, int kin, int k,
+                          uint32_t* out_ids, float* out_dists, uint32_t* out_cta_ids, float* out_cta_dists,
+                          algas_query_stats* out_stats, bool* overflow) {
   const bool dev_ids = is_device_ptr(out_ids), dev_d = is_device_ptr(out_dists);
   std::vector<uint32_t> hid;
   std::vector<float> hd;
@@ -207,29 +228,52 @@ static int finish_outputs(const std::vector<ResultEntry>& res, const std::vector
   float* ds = out_dists;
   if (dev_ids) { hid.resize((size_t)nq * k); ids = hid.data(); }
   if (dev_d) { hd.resize((size_t)nq * k); ds = hd.data(); }
-  for (int64_t q = 0; q < nq; ++q) {
-    const ResultEntry* r = res.data() + (size_t)q * T * kin;
-    if (T == 1) {
-      for (int i = 0; i < k; ++i) { ids[q * k + i] = r[i].id; ds[q * k + i] = r[i].dist; }
-    } else {
-      merge_cta_lists(r, T, kin, k, ids + q * k, ds + q * k);
+  std::atomic<bool> ovf{false};
+  parallel_for(nq, 1024, [&](int64_t lo, int64_t hi) {
+    bool o = false;
+    for (int64_t q = lo; q < hi; ++q) {
+      const ResultEntry* r = res + (size_t)q * T * kin;
+      if (T == 1) {
+        for (int i = 0; i < k; ++i) { ids[q * k + i] = r[i].id; ds[q * k + i] = r[i].dist; }
+      } else {
+        merge_cta_lists(r, T, kin, k, ids + q * k, ds + q * k);
+      }
+      algas_query_stats qs;
+      aggregate_cta_stats(cst + q * T, T, &qs);
+      if (qs.overflows) o = true;
+      if (out_stats) out_stats[q] = qs;
     }
-  }
+    if (o) ovf = true;
+  });
   if (dev_ids) ALGAS_CUDA_TRY(cudaMemcpy(out_ids, hid.data(), hid.size() * 4, cudaMemcpyHostToDevice));
   if (dev_d) ALGAS_CUDA_TRY(cudaMemcpy(out_dists, hd.data(), hd.size() * 4, cudaMemcpyHostToDevice));
   if (out_cta_ids || out_cta_dists) {
-    std::vector<uint32_t> ci((size_t)nq * T * kin);
-    std::vector<float> cd((size_t)nq * T * kin);
-    for (size_t i = 0; i < ci.size(); ++i) { ci[i] = res[i].id; cd[i] = res[i].dist; }
-    if (out_cta_ids) ALGAS_CUDA_TRY(cudaMemcpy(out_cta_ids, ci.data(), ci.size() * 4, cudaMemcpyDefault));
-    if (out_cta_dists) ALGAS_CUDA_TRY(cudaMemcpy(out_cta_dists, cd.data(), cd.size() * 4, cudaMemcpyDefault));
+    const size_t m = (size_t)nq * T * kin;
+    std::vector<uint32_t> ci(m);
+    std::vector<float> cd(m);
+    for (size_t i = 0; i < m; ++i) { ci[i] = res[i].id; cd[i] = res[i].dist; }
+    if (out_cta_ids) ALGAS_CUDA_TRY(cudaMemcpy(out_cta_ids, ci.data(), m * 4, cudaMemcpyDefault));
+    if (out_cta_dists) ALGAS_CUDA_TRY(cudaMemcpy(out_cta_dists, cd.data(), m * 4, cudaMemcpyDefault));
   }
-  *overflow = false;
-  for (int64_t q = 0; q < nq; ++q) {
-    algas_query_stats qs;
-    aggregate_cta_stats(cst.data() + q * T, T, &qs);
-    if (qs.overflows) *overflow = true;
-    if (out_stats) out_stats[q] = qs;
+  *overflow = ovf.load();
+  return ALGAS_OK;
+}
+
+// pinned host staging for per-CTA results / counters (workspace-cached)
+static int ensure_pinned(Workspace* ws, size_t res_bytes, size_t st_bytes) {
+  if (ws->h_res_bytes < res_bytes) {
+    if (ws->h_res) cudaFreeHost(ws->h_res);
+    ws->h_res = nullptr;
+    ws->h_res_bytes = 0;
+    ALGAS_CUDA_TRY(cudaMallocHost(&ws->h_res, res_bytes));
+    ws->h_res_bytes = res_bytes;
+  }
+  if (ws->h_st_bytes < st_bytes) {
+    if (ws->h_st) cudaFreeHost(ws->h_st);
+    ws->h_st = nullptr;
+    ws->h_st_bytes = 0;
+    ALGAS_CUDA_TRY(cudaMallocHost(&ws->h_st, st_bytes));
+    ws->h_st_bytes = st_bytes;
   }
   return ALGAS_OK;
 }
@@ -366,6 +410,8 @@ int algas_index_destroy(algas_index* idx) {
   if (idx->ws) {
     if (idx->ws->gtab) cudaFree(idx->ws->gtab);
     if (idx->ws->counters) cudaFree(idx->ws->counters);
+    if (idx->ws->h_res) cudaFreeHost(idx->ws->h_res);
+    if (idx->ws->h_st) cudaFreeHost(idx->ws->h_st);
     delete idx->ws;
   }
   delete idx;
@@ -438,10 +484,12 @@ int algas_search_ex(const algas_index* cidx, const float* queries, int64_t nq, c
   if ((rc = tm.start())) return rc;
   if ((rc = launch_batch(pl, bl, st))) return rc;
   if ((rc = tm.stop())) return rc;
-  std::vector<ResultEntry> res((size_t)items * pl.k);
-  std::vector<CtaStats> cst((size_t)items);
-  ALGAS_CUDA_TRY(cudaMemcpyAsync(res.data(), rb.p, res.size() * sizeof(ResultEntry), cudaMemcpyDeviceToHost, st));
-  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst.data(), sb.p, cst.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost, st));
+  const size_t res_bytes = (size_t)items * pl.k * sizeof(ResultEntry), st_bytes = (size_t)items * sizeof(CtaStats);
+  if ((rc = ensure_pinned(idx->ws, res_bytes, st_bytes))) return rc;
+  ResultEntry* res = (ResultEntry*)idx->ws->h_res;
+  CtaStats* cst = (CtaStats*)idx->ws->h_st;
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(res, rb.p, res_bytes, cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst, sb.p, st_bytes, cudaMemcpyDeviceToHost, st));
   ALGAS_CUDA_TRY(cudaStreamSynchronize(st));
   ALGAS_CUDA_TRY(cudaGetLastError());
   if (info) fill_info(info, pl, grid, tm.ms());
@@ -504,10 +552,12 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   if ((rc = tm.start())) return rc;
   if ((rc = launch_persistent(pl, pa, st))) return rc;
   if ((rc = tm.stop())) return rc;
-  std::vector<ResultEntry> res((size_t)items * pl.k);
-  std::vector<CtaStats> cst((size_t)items);
-  ALGAS_CUDA_TRY(cudaMemcpyAsync(res.data(), rb.p, res.size() * sizeof(ResultEntry), cudaMemcpyDeviceToHost, st));
-  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst.data(), sb.p, cst.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost, st));
+  const size_t res_bytes = (size_t)items * pl.k * sizeof(ResultEntry), st_bytes = (size_t)items * sizeof(CtaStats);
+  if ((rc = ensure_pinned(idx->ws, res_bytes, st_bytes))) return rc;
+  ResultEntry* res = (ResultEntry*)idx->ws->h_res;
+  CtaStats* cst = (CtaStats*)idx->ws->h_st;
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(res, rb.p, res_bytes, cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst, sb.p, st_bytes, cudaMemcpyDeviceToHost, st));
   ALGAS_CUDA_TRY(cudaStreamSynchronize(st));
   ALGAS_CUDA_TRY(cudaGetLastError());
   if (info) fill_info(info, pl, ctas, tm.ms());

@@ -75,6 +75,18 @@ __device__ __forceinline__ uint4 ldg_u4(const uint4* p) {
                : "l"(p));
   return r;
 }
+// graph rows are re-read by every query (hub neighbourhoods): keep them in L2
+// with an evict_last policy while the vector gathers stream past
+__device__ __forceinline__ uint64_t l2_evict_last_policy() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ uint32_t ldg_u32_hint(const uint32_t* p, uint64_t pol) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -173,9 +185,15 @@ struct ResultEntry {
 struct Ctrl {
   int cnt, nnew, nkeys, np, done, diffusing, vis_count, spilled, overflow, cur;
   uint32_t iters, parents, dist_evals, cap_hit;
-  uint32_t phase;  // bit b: parity of staging barrier b
-  uint64_t worst;  // prefilter key of the current step (read by cluster workers)
+  uint32_t phase;  // bit b: parity of staging barrier b (b=2: step-ready, b=3: keys)
+  uint64_t worst;  // prefilter key of the current step
+  // cluster worker mailbox (written remotely by the leader before it arrives
+  // on the worker's step-ready barrier)
+  int w_cmd;       // kCmdStep / kCmdQuit
+  int w_m;         // rows of this worker in the step
+  uint64_t w_worst;
 };
+enum { kCmdStep = 1, kCmdQuit = 2 };
 
 // Shared-memory carve-up (bytes, all 16-B aligned).
 struct SmemLayout {
@@ -193,7 +211,7 @@ __host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int 
   s.off_newid = o; o += align16(ncap * 4);
   s.off_sel = o;   o += align16(64 * 4);
   s.off_hash = o;  o += align16((1 << hash_bits) * 4);
-  s.off_bar = o;   o += 16;
+  s.off_bar = o;   o += 32;
   s.off_ctrl = o;  o += align16((int)sizeof(Ctrl));
   s.total = o;
   return s;
@@ -226,14 +244,19 @@ __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
 }
 // once per CTA lifetime (kernel start): staging barriers; zero staging and
 // query buffers so the padded tail chunks of every row read as 0
+// bar[0..1]: staging buffers; bar[2]: "step ready" (cluster worker, 1
+// arrival from the leader); bar[3]: "keys delivered" (cluster leader, CS-1
+// arrivals).
 template <int NT>
-__device__ __forceinline__ void init_cta(const Smem& s, const SearchCfg& cfg) {
+__device__ __forceinline__ void init_cta(const Smem& s, const SearchCfg& cfg, int cs = 1) {
   const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
   for (int i = threadIdx.x; i < 2 * cfg.stage_rows * cfg.dp4; i += NT) s.stage[i] = z;
   for (int i = threadIdx.x; i < cfg.dp4; i += NT) s.q[i] = z;
   if (threadIdx.x == 0) {
     mbar_init(s.bar + 0, 1);
     mbar_init(s.bar + 1, 1);
+    mbar_init(s.bar + 2, 1);
+    mbar_init(s.bar + 3, cs > 1 ? cs - 1 : 1);
     mbar_fence_init();
     s.ctrl->phase = 0;
   }
@@ -369,9 +392,35 @@ __device__ __forceinline__ void cluster_barrier() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 template <typename T>
+__device__ __forceinline__ T* rank_ptr(T* local, int rank) {
+  // generic address of the same shared-memory object in cluster CTA `rank`
+  return cooperative_groups::this_cluster().map_shared_rank(local, (unsigned)rank);
+}
+template <typename T>
 __device__ __forceinline__ T* leader_ptr(T* local) {
-  // generic address of the same shared-memory object in cluster CTA 0
-  return cooperative_groups::this_cluster().map_shared_rank(local, 0);
+  return rank_ptr(local, 0);
+}
+// Point-to-point cluster signalling on mbarriers (cheaper than a full
+// barrier.cluster: only the signalling thread and the waiters take part).
+// The sender's prior writes (by any thread of its CTA, ordered before it by
+// __syncthreads) are released at cluster scope by fence + arrive.release.
+__device__ __forceinline__ void fence_cluster() { asm volatile("fence.acq_rel.cluster;" ::: "memory"); }
+__device__ __forceinline__ void mbar_remote_arrive(uint64_t* bar, int rank) {
+  uint32_t ra;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(bar)), "r"(rank));
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
 }
 
 // Distance step for rows r = r0, r0+rstep, ... < M of newid (P:L217 step 3):
@@ -536,12 +585,14 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   };
 
   int cur = 0;
+  int lcnt = 0;            // list length (uniform register copy in every thread)
+  uint32_t liters = 0;     // steps taken
   bool first = true;
   for (;;) {
     // ================= select (warp 0) =================
     if (!first) {
       if (warp == 0) {
-        const int cnt = C->cnt;
+        const int cnt = lcnt;
         uint64_t* list = cur ? s.list[1] : s.list[0];
         // also look past the parents: the next few unchecked candidates are
         // the likely parents of the next step, whose graph rows are
@@ -563,7 +614,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
         int done = 0, np = 0;
         if (found == 0) {
           done = 1;
-        } else if ((int)C->iters >= cfg.max_iter) {
+        } else if ((int)liters >= cfg.max_iter) {
           done = 1;
           if (lane == 0) C->cap_hit = 1;
         } else {
@@ -595,10 +646,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       }
       __syncthreads();
       lap(0);
-      if (C->done) {
-        if constexpr (CS > 1) cluster_barrier();  // B: workers see done and leave
-        break;
-      }
+      if (C->done) break;
 
       // ================= gather + visited filter (P:L217 steps 1-2) =================
       {
@@ -610,7 +658,8 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           uint32_t id = kSentinel;
           if (idx < total) {
             const uint32_t parent = (uint32_t)s.sel[32 + (idx >> cfg.rp_shift)];
-            id = __ldg(cfg.graph + ((uint64_t)parent << cfg.rp_shift) + (idx & (Rp - 1)));
+            const uint32_t* gp = cfg.graph + ((uint64_t)parent << cfg.rp_shift) + (idx & (Rp - 1));
+            id = (cfg.prefetch & 4) ? ldg_u32_hint(gp, l2_evict_last_policy()) : __ldg(gp);
           }
           bool keep = false;
           if (id != kSentinel) {
@@ -647,15 +696,30 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     // ================= distances (P:L217 step 3) + prefilter =================
     {
       const int M = C->nnew;
-      const int cnt = C->cnt;
+      const int cnt = lcnt;
       const uint64_t worst = (cnt >= L) ? (cur ? s.list[1] : s.list[0])[L - 1] : kKeyMax;
       if (cfg.gather_mode == 0) {
         if constexpr (CS > 1) {
-          // B: publish the step (newid[0..M), worst) to the cluster workers
-          if (tid == 0) C->worst = worst;
-          cluster_barrier();
+          // hand worker c the rows r = c, c+CS, ... (ids pushed into its shared
+          // memory), its row count and the prefilter key, then signal it
+          for (int r = tid; r < M; r += NT) {
+            const int c = r % CS;
+            if (c) rank_ptr(s.newid, c)[r / CS] = s.newid[r];
+          }
+          __syncthreads();
+          if (tid < CS - 1) {  // one thread per worker
+            const int c = tid + 1;
+            Ctrl* wc = rank_ptr(C, c);
+            wc->w_cmd = kCmdStep;
+            wc->w_m = M > c ? (M - c + CS - 1) / CS : 0;
+            wc->w_worst = worst;
+            fence_cluster();
+            mbar_remote_arrive(s.bar + 2, c);
+          }
           dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
-          cluster_barrier();  // C: every CTA's keys delivered into newk
+          mbar_wait_cluster(s.bar + 3, (phase >> 3) & 1u);  // all workers' keys delivered
+          phase ^= 8u;
+          __syncthreads();
         } else {
           dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, 1, worst, s.newid, s.newk, &C->nkeys);
           __syncthreads();
@@ -725,7 +789,8 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     // first L positions form the new list (a merge, not a re-sort).
     {
       const int nk = C->nkeys;
-      const int cnt = C->cnt;
+      const int npv = C->np;  // read before warp 0 may start the next select
+      const int cnt = lcnt;
       if (nk > 0) {
         const uint64_t* src = cur ? s.list[1] : s.list[0];
         uint64_t* dst = cur ? s.list[0] : s.list[1];
@@ -744,20 +809,20 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           if (pos < L) dst[pos] = key;
         }
         cur ^= 1;
-        __syncthreads();
-        if (tid == 0) {
-          const int nc = cnt + nk;
-          C->cnt = nc < L ? nc : L;
-        }
+        lcnt = (cnt + nk) < L ? cnt + nk : L;
       }
-      if (tid == 0) C->iters += (C->np > 0) ? 1 : 0;
+      liters += npv > 0 ? 1 : 0;
       __syncthreads();
       lap(3);
     }
   }
 
   // ================= publish the first k =================
-  const int cnt = C->cnt;
+  if (tid == 0) {
+    C->cnt = lcnt;
+    C->iters = liters;
+  }
+  const int cnt = lcnt;
   const uint64_t* fin = cur ? s.list[1] : s.list[0];
   for (int i = tid; i < k; i += NT) {
     ResultEntry r;
@@ -792,20 +857,46 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
 // barriers per step and evaluates its share (rows crank, crank+CS, ...) of
 // every distance step, reading ids from and delivering keys into the
 // leader's shared memory.  Preconditions: s.q holds the query.
-template <int NT, int TL, int CPL, int METRIC, int CS>
-__device__ void search_worker(const SearchCfg& cfg, const Smem& s, int crank) {
+// One command from the leader: wait on the step-ready barrier, evaluate this
+// CTA's rows (ids in its own shared memory, the query in s.q as pushed by the
+// leader at query start), deliver the keys into the leader's newk, signal.
+// Returns the command (kCmdStep or kCmdQuit).
+template <int NT, int TL, int CPL, int METRIC>
+__device__ int worker_step(const SearchCfg& cfg, const Smem& s, uint32_t& phase) {
+  mbar_wait_cluster(s.bar + 2, (phase >> 2) & 1u);
+  phase ^= 4u;
+  const int cmd = *((volatile int*)&s.ctrl->w_cmd);
+  if (cmd != kCmdStep) return cmd;
+  const int M = *((volatile int*)&s.ctrl->w_m);
+  const uint64_t worst = *((volatile uint64_t*)&s.ctrl->w_worst);
   QueryRegs<TL, CPL> Q;
   Q.load(s.q, threadIdx.x % TL);
   Ctrl* LC = leader_ptr(s.ctrl);
-  const uint32_t* lnewid = leader_ptr(s.newid);
-  uint64_t* lnewk = leader_ptr(s.newk);
-  for (;;) {
-    cluster_barrier();  // B
-    if (*((volatile int*)&LC->done)) break;
-    const int M = *((volatile int*)&LC->nnew);
-    const uint64_t worst = *((volatile uint64_t*)&LC->worst);
-    dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, crank, CS, worst, lnewid, lnewk, &LC->nkeys);
-    cluster_barrier();  // C
+  dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, 1, worst, s.newid, leader_ptr(s.newk), &LC->nkeys);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    fence_cluster();
+    mbar_remote_arrive(s.bar + 3, 0);
+  }
+  return cmd;
+}
+// leader: push the query into every worker's shared memory (released by the
+// next step signal)
+template <int NT, int CS>
+__device__ __forceinline__ void push_query(const Smem& s, int d4) {
+  for (int c = 1; c < CS; ++c) {
+    float4* wq = rank_ptr(s.q, c);
+    for (int i = threadIdx.x; i < d4; i += NT) wq[i] = s.q[i];
+  }
+}
+// leader: tell every worker to leave
+template <int CS>
+__device__ __forceinline__ void post_quit(const Smem& s) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int c = 1; c < CS; ++c) rank_ptr(s.ctrl, c)->w_cmd = kCmdQuit;
+    fence_cluster();
+    for (int c = 1; c < CS; ++c) mbar_remote_arrive(s.bar + 2, c);
   }
 }
 

@@ -101,7 +101,8 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows);
   const Smem s = carve(smem_raw, lay);
-  init_cta<NT>(s, A.cfg);
+  init_cta<NT>(s, A.cfg, CS);
+  if constexpr (CS > 1) cluster_barrier();  // every CTA's mbarriers exist before any remote arrive
   const PersistArgs& P = A.p;
   // a search unit = one (slot, cta_rank) search = one cluster of CS CTAs
   const int unit = blockIdx.x / CS;
@@ -115,20 +116,11 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
 
   if constexpr (CS > 1) {
     if (crank != 0) {
-      // cluster worker: follow the leader query by query (barrier A)
-      const unsigned long long* lmb = leader_ptr(&s_mbox);
-      const float4* lq = leader_ptr(s.q);
-      for (;;) {
-        cluster_barrier();  // A: leader staged the next query (or quit)
-        if (*((volatile unsigned long long*)lmb) == kMboxQuit) {
-          cluster_barrier();  // Z: the leader's shared memory outlives our last read
-          return;
-        }
-        for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = lq[i];
-        __syncthreads();
-        search_worker<NT, TL, CPL, METRIC, CS>(A.cfg, s, crank);
-        __syncthreads();
+      // cluster worker: serve the leader's distance steps until it quits
+      uint32_t ph = 0;
+      while (worker_step<NT, TL, CPL, METRIC>(A.cfg, s, ph) == kCmdStep) {
       }
+      return;
     }
   }
 
@@ -209,10 +201,7 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
     }
     const unsigned long long mb = s_mbox;
     if (mb == kMboxQuit) {
-      if constexpr (CS > 1) {
-        cluster_barrier();  // A: release the workers
-        cluster_barrier();  // Z: they have read the quit word
-      }
+      if constexpr (CS > 1) post_quit<CS>(s);
       break;
     }
     const uint32_t epoch = (uint32_t)(mb >> 32);
@@ -230,8 +219,8 @@ __global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
     const float4* qsrc = (P.mode == 0) ? P.qbuf + (uint64_t)slot * A.cfg.d4
                                        : P.queries + (uint64_t)item * A.cfg.d4;
     for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = (P.mode == 0) ? ld_volatile_f4(qsrc + i) : qsrc[i];
+    if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
     __syncthreads();
-    if constexpr (CS > 1) cluster_barrier();  // A: workers copy the query
 
     SearchCfg cfg = A.cfg;
     cfg.L = par.y;

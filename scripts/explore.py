@@ -69,7 +69,10 @@ def main():
     for L in Ls:
         for (wd, T, nt) in [(1, 1, 64), (4, 1, 64), (4, 1, 128), (4, 4, 64), (2, 8, 64), (4, 8, 64)]:
             grid.append((L, wd, T, nt))
-    if os.environ.get("GRID") == "pf":
+    if os.environ.get("GRID") == "tune":
+        grid = [(64, 4, 1, 256, 1), (64, 8, 1, 256, 1), (64, 16, 1, 256, 1), (56, 8, 2, 256, 1),
+                (48, 8, 4, 256, 1), (56, 8, 4, 256, 1), (96, 16, 1, 256, 1), (64, 8, 2, 256, 1)]
+    elif os.environ.get("GRID") == "pf":
         grid = [(64, 4, 1, 256, 1), (64, 8, 1, 256, 1), (64, 4, 2, 256, 1), (56, 4, 2, 256, 1), (48, 4, 4, 256, 1),
                 (56, 4, 4, 256, 1), (64, 4, 1, 128, 1)]
     elif os.environ.get("GRID") == "cs":

@@ -106,10 +106,12 @@ def base_vectors(w: Workload, n: int | None = None) -> np.ndarray:
     return _finish(w, _mixture(rng, n, w.dim, centers, bases, w.spread, w.noise))
 
 
-def query_vectors(w: Workload, nq: int | None = None) -> np.ndarray:
+def query_vectors(w: Workload, nq: int | None = None, stream: int = 0) -> np.ndarray:
+    """Queries from the base distribution; `stream` selects an independent
+    query set (stream 1 = the calibration set used to pick operating points)."""
     nq = w.n_queries if nq is None else nq
     centers, bases = _model(w, w.dim)
-    rng = np.random.default_rng(w.seed_query)
+    rng = np.random.default_rng(w.seed_query + 1000003 * stream)
     return _finish(w, _mixture(rng, nq, w.dim, centers, bases, w.spread, w.noise))
 
 
