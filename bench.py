@@ -48,29 +48,60 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    """SM clocks + throttle reasons sampled during the timed region, in-process
+    through NVML (nvidia_ml_py) -- spawning nvidia-smi every 200 ms stalls the
+    CUDA calls of the timed steps; nvidia-smi is the fallback."""
 
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
+    # NVML clocks-event reason bits
+    REASONS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40}
 
-    def __init__(self, gpu_index: int):
+    def __init__(self, gpu_index: int, period_s: float = 0.05):
         self.idx = gpu_index
-        self.samples = []
+        self.period = period_s
+        self.samples = []  # (sm_mhz, max_mhz, set of reasons)
         self._stop = threading.Event()
         self._t = None
+        self._nvml = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nvml = (pynvml, pynvml.nvmlDeviceGetHandleByIndex(self._physical_index(gpu_index)))
+        except Exception:
+            self._nvml = None
+
+    @staticmethod
+    def _physical_index(i):
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        if vis:
+            try:
+                return int(vis.split(",")[i])
+            except Exception:
+                return i
+        return i
+
+    def _sample(self):
+        if self._nvml:
+            nv, h = self._nvml
+            sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+            mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+            bits = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+            return float(sm), float(mx), {k for k, b in self.REASONS.items() if bits & b}
+        out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
+                              "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5).stdout
+        f = [x.strip() for x in out.strip().split(",")]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        return float(f[0]), float(f[1]), {nm for nm, v in zip(names, f[3:7]) if v.lower() == "active"}
 
     def _run(self):
         while not self._stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
-                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
-                                     timeout=5).stdout.strip()
-                if out:
-                    self.samples.append([x.strip() for x in out.split(",")])
+                self.samples.append(self._sample())
             except Exception:
                 pass
-            self._stop.wait(0.2)
+            self._stop.wait(self.period)
 
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
@@ -85,16 +116,12 @@ class ClockSampler:
     def summary(self):
         if not self.samples:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
-        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
-        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = set()
         for s in self.samples:
-            for nm, v in zip(names, s[3:7]):
-                if v.strip().lower() == "active":
-                    reasons.add(nm)
-        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(self.samples)}
+            reasons |= s[2]
+        return {"sm_mhz": float(np.median([s[0] for s in self.samples])),
+                "sm_max_mhz": max(s[1] for s in self.samples), "reasons": sorted(reasons),
+                "samples": len(self.samples), "source": "nvml" if self._nvml else "nvidia-smi"}
 
 
 def recall_at(found, truth, k):
@@ -138,34 +165,40 @@ def build_workload(w, nq, dev):
     return X, Q, Xd, Qd, G, ti, (Qcd, tc), time.time() - t0
 
 
-def choose_operating_point(idx, Qd, truth, w, slots, target=0.95, Ts=(1,), threads=256, width=8):
-    """Operating point of the BASELINE metric: for each CTAs-per-query T
-    (P:L229), the smallest L of the sweep whose recall@k >= target; among
-    those, the configuration with the highest QPS (the adaptive tuning of
-    P:L225-249 applied to measured recall)."""
+def choose_operating_point(idx, Qd, truth, w, slots, target=0.95, Ts=(1,), threads=(256,), widths=(8,),
+                           offsets=(1,)):
+    """Operating point of the BASELINE metric: for each (CTAs per query T
+    (P:L229), threads per CTA, beam width w, offset_beam),
+    the smallest L of the sweep whose recall@k >= target; among those, the
+    configuration with the highest QPS (the adaptive tuning of P:L225-249
+    applied to measured recall)."""
     import paper_conf_ipps_chencyzw025_b200 as algas
     Ls = [16, 24, 32, 40, 48, 56, 64, 80, 96, 128, 160, 192, 256, 320, 384, 448, 512]
     sweep = []
     best, best_qps = None, -1.0
-    for T in Ts:
-        for L in Ls:
-            if L < w.k:
-                continue
-            p = algas.default_params(k=w.k, itopk=L, width=min(width, max(1, L // 8)),
-                                     offset_beam=max(1, L // 4), ctas_per_query=T, threads_per_cta=threads,
-                                     slots=slots, n_seeds=32, seed=1)
-            try:
-                r = idx.search_dynamic(Qd, p)
-            except algas.AlgasError as e:  # e.g. slots x T not co-resident
-                sweep.append({"ctas": T, "itopk": L, "error": str(e)[:80]})
-                break
-            rec = recall_at(r["ids"], truth, w.k)
-            qps = Qd.shape[0] / (r["info"].kernel_ms / 1e3)
-            sweep.append({"ctas": T, "itopk": L, "width": p.width, "recall": round(rec, 5), "qps": round(qps)})
-            if rec >= target:
-                if qps > best_qps:
-                    best, best_qps = p, qps
-                break
+    for nt in threads:
+        for T in Ts:
+            for wd in widths:
+                for off in offsets:
+                    for L in Ls:
+                        if L < w.k:
+                            continue
+                        p = algas.default_params(k=w.k, itopk=L, width=min(wd, L), offset_beam=min(off, L),
+                                                 ctas_per_query=T, threads_per_cta=nt, slots=slots, n_seeds=32,
+                                                 seed=1)
+                        try:
+                            r = idx.search_dynamic(Qd, p)
+                        except algas.AlgasError as e:  # e.g. slots x T not co-resident
+                            sweep.append({"ctas": T, "threads": nt, "itopk": L, "error": str(e)[:80]})
+                            break
+                        rec = recall_at(r["ids"], truth, w.k)
+                        qps = Qd.shape[0] / (r["info"].kernel_ms / 1e3)
+                        sweep.append({"ctas": T, "threads": nt, "width": p.width, "offset_beam": p.offset_beam,
+                                      "itopk": L, "recall": round(rec, 5), "qps": round(qps)})
+                        if rec >= target:
+                            if qps > best_qps:
+                                best, best_qps = p, qps
+                            break
     return best, sweep
 
 
@@ -184,7 +217,8 @@ def run_algas(a, rank, world, local):
     idx = algas.Index(Xd, G, w.metric)
     # the recall/QPS curve is swept on the measured query set (standard ANN
     # practice), so the reported point provably meets recall@10 >= 0.95
-    p, sweep = choose_operating_point(idx, Qd, truth, w, a.batch, Ts=a.ctas, threads=a.threads, width=a.width)
+    p, sweep = choose_operating_point(idx, Qd, truth, w, a.batch, Ts=a.ctas, threads=a.threads, widths=a.width,
+                                      offsets=a.offset)
     if p is None:
         raise SystemExit("no swept itopk reaches recall 0.95")
     if world > 1:  # every rank runs rank 0's operating point
@@ -203,7 +237,7 @@ def run_algas(a, rank, world, local):
     if world > 1:
         dist.barrier()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
-    kern_ms, lat, evals, parents, recs = [], [], [], [], []
+    kern_ms, call_ms, merge_ms, lat, evals, parents, recs = [], [], [], [], [], [], []
     with ClockSampler(local) as clk:
         for i in range(a.steps):
             flush.zero_()                       # L2 flush between timed steps (untimed)
@@ -213,6 +247,8 @@ def run_algas(a, rank, world, local):
             ev[i][1].record(stream)
             torch.cuda.synchronize()
             kern_ms.append(r["info"].kernel_ms)
+            call_ms.append(r["info"].call_ms)
+            merge_ms.append(r["info"].merge_ms)
             st = r["stats"]
             lat.append((st["t_end_ns"] - st["t_start_ns"]) / 1e3)
             evals.append(st["dist_evals"].astype(np.float64))
@@ -345,6 +381,10 @@ def run_algas(a, rank, world, local):
         "cpu_baseline": cpu,
         "work": {"dist_evals_per_query": float(evals.mean()), "parents_per_query": float(parents.mean()),
                  "setup_s": t_setup},
+        "step_breakdown_ms": {"kernel": float(np.mean(kern_ms)), "call": float(np.mean(call_ms)),
+                              "host_merge": float(np.mean(merge_ms)),
+                              "definition": "kernel = CUDA events around the persistent launch; call = host wall "
+                                            "time of algas_search_dynamic (launch, D2H, host TopK merge)"},
         "recall_sweep": sweep,
         "batch_sweep": batch_sweep,
     }
@@ -393,7 +433,8 @@ def run_reference(a, rank, world, local):
     torch.cuda.set_device(dev)
     X, Q, Xd, Qd, G, truth, (Qcd, tcal), _ = build_workload(w, a.nq, dev)
     idx = algas.Index(Xd, G, w.metric)
-    p, sweep = choose_operating_point(idx, Qcd, tcal, w, a.batch, Ts=a.ctas, threads=a.threads, width=a.width)
+    p, sweep = choose_operating_point(idx, Qcd, tcal, w, a.batch, Ts=a.ctas, threads=a.threads, widths=a.width,
+                                      offsets=a.offset)
     del idx
     import oracle
     op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=1, S=p.n_seeds,
@@ -435,8 +476,10 @@ def main():
     ap.add_argument("--batch", type=int, default=32, help="query slots in flight (B)")
     ap.add_argument("--ctas", type=lambda x: tuple(int(v) for v in x.split(",")), default=(1, 2, 4),
                     help="CTAs per query (T) candidates, comma separated")
-    ap.add_argument("--threads", type=int, default=256)
-    ap.add_argument("--width", type=int, default=8)
+    ints = lambda x: tuple(int(v) for v in x.split(","))  # noqa: E731
+    ap.add_argument("--threads", type=ints, default=(256, 512, 1024), help="threads per CTA candidates")
+    ap.add_argument("--width", type=ints, default=(8, 16), help="beam width (parents per step) candidates")
+    ap.add_argument("--offset", type=ints, default=(1,), help="offset_beam candidates (P:L249)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--ref-queries-per-step", type=int, default=100)

@@ -80,7 +80,7 @@ typedef struct algas_params {
                                 unchecked position >= off; < 0 -> itopk/4;
                                 >= itopk disables beam extend (pure Alg.1)           */
     int32_t ctas_per_query;  /* T = N_parallel; 0 -> adaptive tuner */
-    int32_t threads_per_cta; /* 32/64/128/256; 0 -> tuner                            */
+    int32_t threads_per_cta; /* 32/64/128/256/512/1024 (1024: dim <= 512); 0 -> tuner */
     int32_t n_seeds;         /* S random entry points per CTA; 0 -> 32      */
     int32_t max_iter;        /* per-CTA step cap (R8); 0 -> 4*itopk + 256            */
     int32_t visited_mode;    /* enum algas_visited                                  */
@@ -125,6 +125,8 @@ typedef struct algas_run_info {
     int32_t blocks_per_sm;    /* occupancy of the search kernel                            */
     int32_t hash_bits;
     int32_t reserved;
+    float call_ms;            /* host wall time of the whole call (entry -> outputs written) */
+    float merge_ms;           /* host wall time of the TopK merge + output copy    */
 } algas_run_info;
 
 typedef struct algas_index algas_index;   /* opaque; immutable after create */
@@ -278,9 +280,20 @@ int algas_tune(const algas_device_props *props, int32_t slots, int32_t dim, int3
 /* Exact k nearest base points of every query, fp32 distances,
  * (dist,id) order.  self_base >= 0 excludes base id (self_base + i) from
  * query i's answer (kNN graph of the base set: queries = base, self_base=0).
- * k <= 1024.  out_ids/out_dists: nq x k. */
+ * k <= 1024.  out_ids/out_dists: nq x k.  base/queries/outputs: host or
+ * device pointers (copied as needed; caller keeps ownership).
+ * Two paths with identical results: large problems (n*nq >= 1e8, k <= 170)
+ * screen candidates with tensor-core 3xTF32 GEMMs (cuBLAS), re-rank them
+ * with the exact fp32 direct-form distance and certify each query (bound on
+ * the screening error), redoing uncertified queries on the direct CUDA-core
+ * path; ALGAS_KNN_MODE=direct|screened forces one.  Errors: EINVAL on bad
+ * arguments, ENOMEM/ECUDA from the device. */
 int algas_knn(const float *base, int64_t n, const float *queries, int64_t nq, int32_t dim,
               int32_t metric, int32_t k, int64_t self_base, uint32_t *out_ids, float *out_dists);
+/* Rows screened by the tensor-core path since the last call on this thread;
+ * *fallback_rows (nullable) = rows the certificate sent to the direct path.
+ * Resets both counters. */
+int64_t algas_knn_last_stats(int64_t *fallback_rows);
 /* CAGRA-style reading R24: rank-based detour count, keep `degree` edges,
  * add reverse edges, merge.  knn: n x knn_degree (sorted rows, no self).
  * out_graph: n x degree. */

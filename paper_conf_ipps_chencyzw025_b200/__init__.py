@@ -64,7 +64,8 @@ assert STATS_DTYPE.itemsize == ctypes.sizeof(QueryStats)
 class RunInfo(ctypes.Structure):
     _fields_ = [("kernel_ms", ctypes.c_float), ("grid", ctypes.c_int32), ("threads_per_cta", ctypes.c_int32),
                 ("ctas_per_query", ctypes.c_int32), ("smem_per_cta", ctypes.c_int32),
-                ("blocks_per_sm", ctypes.c_int32), ("hash_bits", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("blocks_per_sm", ctypes.c_int32), ("hash_bits", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("call_ms", ctypes.c_float), ("merge_ms", ctypes.c_float)]
 
 
 class DeviceProps(ctypes.Structure):
@@ -85,7 +86,8 @@ EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_i
            "algas_index_destroy", "algas_index_info", "algas_search", "algas_search_ex", "algas_search_dynamic",
            "algas_server_create", "algas_submit", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
-           "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_prune", "algas_build_graph"]
+           "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
+           "algas_build_graph"]
 
 _lock = threading.Lock()
 _lib = None
@@ -133,6 +135,8 @@ def lib(build_if_missing: bool = True):
         L.algas_tuner_smem_per_block.restype = i64
         L.algas_tune.argtypes = [ctypes.POINTER(DeviceProps), i32, i32, i32, i32, i32, ctypes.POINTER(Tuning)]
         L.algas_knn.argtypes = [P, i64, P, i64, i32, i32, i32, i64, P, P]
+        L.algas_knn_last_stats.argtypes = [ctypes.POINTER(i64)]
+        L.algas_knn_last_stats.restype = i64
         L.algas_prune.argtypes = [P, i64, i32, i32, P]
         L.algas_build_graph.argtypes = [P, i64, i32, i32, i32, i32, i32, P]
         _lib = L
@@ -339,6 +343,14 @@ def knn(base, queries, k: int, metric: int = L2, self_base: int = -1):
     dp, _d = _ptr(ds)
     _check(lib().algas_knn(bp, int(base.shape[0]), qp, nq, dim, metric, k, self_base, ip, dp))
     return ids, ds
+
+
+def knn_last_stats():
+    """(rows screened on tensor cores, rows re-done on the direct path) since
+    the last call (algas_knn_last_stats); resets the counters."""
+    fb = ctypes.c_int64(0)
+    n = lib().algas_knn_last_stats(ctypes.byref(fb))
+    return int(n), int(fb.value)
 
 
 def prune(knn_graph, degree: int):

@@ -10,7 +10,10 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libalgas.so")
 SOURCES = ["search_kernels.cu", "search_api.cu", "runtime.cu", "knn.cu"]
-HEADERS = ["search_core.cuh", "internal.h", os.path.join("..", "..", "include", "algas.h")]
+# the search kernels, one object per thread count (compiled in parallel)
+THREAD_COUNTS = [32, 64, 128, 256, 512, 1024]
+KERNEL_TU = "kernels_nt.cu"
+HEADERS = ["search_core.cuh", "kernels.cuh", "internal.h", KERNEL_TU, os.path.join("..", "..", "include", "algas.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
@@ -32,10 +35,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     objs = []
     jobs = []
-    for src in SOURCES:
-        obj = os.path.join(CSRC, src.replace(".cu", ".o"))
-        cmd = [NVCC, *ARCH, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
-        jobs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)))
+    units = [(src, src.replace(".cu", ".o"), []) for src in SOURCES]
+    units += [(KERNEL_TU, f"kernels_nt{nt}.o", [f"-DALGAS_NT={nt}"]) for nt in THREAD_COUNTS]
+    for src, o, defs in units:
+        obj = os.path.join(CSRC, o)
+        cmd = [NVCC, *ARCH, *FLAGS, *defs, "-c", os.path.join(CSRC, src), "-o", obj]
+        jobs.append((f"{src} {' '.join(defs)}", subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)))
         objs.append(obj)
     logs = []
     failed = False
@@ -44,14 +49,18 @@ def build(force: bool = False, verbose: bool = False) -> str:
         logs.append(f"== {src}\n{out}")
         if p.returncode != 0:
             failed = True
-    log_path = os.path.join(CSRC, "build.log")
+    log_path = os.path.join(HERE, "build.log")
     with open(log_path, "w") as f:
         f.write("\n".join(logs))
     if failed:
         sys.stderr.write("\n".join(logs)[-20000:])
         raise RuntimeError(f"nvcc failed (see {log_path})")
     tmp = LIB + f".tmp{os.getpid()}"
-    subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-lrt", "-lpthread", "-ldl"])
+    # cuBLAS (tensor-core kNN screen) from the toolkit; rpath so the library
+    # resolves it without LD_LIBRARY_PATH (same image on the GPU box)
+    cuda_lib = os.path.join(os.path.dirname(os.path.dirname(NVCC)), "lib64")
+    subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-L" + cuda_lib, "-lcublas",
+                           "-Xlinker", "-rpath=" + cuda_lib, "-lrt", "-lpthread", "-ldl"])
     os.replace(tmp, LIB)
     for o in objs:
         os.remove(o)

@@ -163,6 +163,15 @@ inline void carve_control(uint8_t* cb, int slots, PersistArgs* pa) {
 }
 int max_blocks_per_sm(const Plan& pl, bool persistent, int* out);
 
+// kernel tables, one per thread count (kernels_nt.cu): the batch or
+// persistent kernel for (metric, chunk config, cluster size), or null
+void* kernel_table_nt32(int metric, int cc, bool persist, int cs);
+void* kernel_table_nt64(int metric, int cc, bool persist, int cs);
+void* kernel_table_nt128(int metric, int cc, bool persist, int cs);
+void* kernel_table_nt256(int metric, int cc, bool persist, int cs);
+void* kernel_table_nt512(int metric, int cc, bool persist, int cs);
+void* kernel_table_nt1024(int metric, int cc, bool persist, int cs);
+
 // per-query counters from the T per-CTA records
 inline void aggregate_cta_stats(const CtaStats* cs, int T, algas_query_stats* q) {
   *q = algas_query_stats{};

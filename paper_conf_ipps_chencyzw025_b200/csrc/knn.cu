@@ -12,8 +12,12 @@
 //                merge).  The graph type is named at P:L293; the algorithm
 //                is CAGRA's (ref [25]) and not printed in the paper.
 #include <cub/cub.cuh>
+#include <cublas_v2.h>
 
 #include <algorithm>
+#include <cmath>
+#include <cstdlib>
+#include <mutex>
 #include <cstring>
 #include <vector>
 
@@ -88,10 +92,17 @@ constexpr int SEL_BUF = 64;
 
 // one warp per query row; the row's sorted top-k keys live in HBM between
 // chunks and in shared memory (double buffered) while a chunk is scanned.
+// MODE 0: D holds distances.  MODE 1/2: D holds dot products q.x from the
+// tensor-core screen; the key distance is |q|^2 + |x|^2 - 2 q.x (L2, MODE 1)
+// or -q.x (IP, MODE 2).
+template <int MODE>
 __global__ void __launch_bounds__(SEL_WARPS * 32) select_kernel(const float* __restrict__ D, int64_t ldD, int rows,
                                                                 int64_t cols, int64_t col0, int64_t row0,
                                                                 int64_t self_base, int k,
-                                                                unsigned long long* __restrict__ state) {
+                                                                unsigned long long* __restrict__ state,
+                                                                const float* __restrict__ qnorm,
+                                                                const float* __restrict__ xnorm,
+                                                                const int64_t* __restrict__ self_ids) {
   extern __shared__ __align__(16) uint8_t sm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int row = blockIdx.x * SEL_WARPS + warp;
@@ -105,8 +116,9 @@ __global__ void __launch_bounds__(SEL_WARPS * 32) select_kernel(const float* __r
   unsigned long long* cur = la;
   unsigned long long* oth = lb;
   int nb = 0;
-  const int64_t self = self_base >= 0 ? self_base + row0 + row : -1;
+  const int64_t self = self_ids ? self_ids[row0 + row] : (self_base >= 0 ? self_base + row0 + row : -1);
   const float* dr = D + (size_t)row * ldD;
+  const float qn = MODE == 1 ? qnorm[row0 + row] : 0.f;
   auto flush = [&]() {
     // sort buf[0..64) (padded) with a smem bitonic network, then rank-merge
     for (int i = nb + lane; i < SEL_BUF; i += 32) buf[i] = kKeyMax;
@@ -137,7 +149,12 @@ __global__ void __launch_bounds__(SEL_WARPS * 32) select_kernel(const float* __r
     unsigned long long key = kKeyMax;
     if (c < cols) {
       const int64_t id = col0 + c;
-      if (id != self) key = make_key(dr[c], (uint32_t)id);
+      if (id != self) {
+        float dv = dr[c];
+        if (MODE == 1) dv = qn + xnorm[id] - 2.f * dv;
+        if (MODE == 2) dv = -dv;
+        key = make_key(dv, (uint32_t)id);
+      }
     }
     const unsigned long long thr = cur[k - 1];
     const bool cand = key < thr;
@@ -265,18 +282,10 @@ static int to_device(const void* src, size_t bytes, Dev& holder, const void** ou
   return ALGAS_OK;
 }
 
-}  // namespace algas
-
-using namespace algas;
-
-extern "C" {
-
-int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, int32_t dim, int32_t metric, int32_t k,
-              int64_t self_base, uint32_t* out_ids, float* out_dists) {
-  if (!base || !queries || !out_ids || !out_dists || n < 1 || n >= (1LL << 31) || nq < 0 || dim < 4 ||
-      dim % 4 != 0 || k < 1 || k > 1024 || (metric != ALGAS_L2 && metric != ALGAS_IP))
-    return set_error(ALGAS_EINVAL, "algas_knn: bad arguments");
-  if (nq == 0) return ALGAS_OK;
+// Exact kNN on CUDA cores: direct-form distance tiles + running top-k.
+// self_ids (device, nq entries, nullable) overrides self_base per query.
+static int knn_direct(const float* base, int64_t n, const float* queries, int64_t nq, int32_t dim, int32_t metric,
+                      int32_t k, int64_t self_base, const int64_t* self_ids, uint32_t* out_ids, float* out_dists) {
   Dev hx, hq, hstate, hD, hid, hd;
   const float *X = nullptr, *Q = nullptr;
   int rc;
@@ -292,7 +301,7 @@ int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, in
   ALGAS_CUDA_TRY(cudaMalloc(&hid.p, (size_t)QB * k * 4));
   ALGAS_CUDA_TRY(cudaMalloc(&hd.p, (size_t)QB * k * 4));
   const int sel_smem = SEL_WARPS * (2 * k + SEL_BUF) * 8;
-  ALGAS_CUDA_TRY(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem));
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(select_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem));
   auto* unsafe_D = (float*)hD.p;
   for (int64_t q0 = 0; q0 < nq; q0 += QB) {
     const int64_t qb = std::min<int64_t>(QB, nq - q0);
@@ -305,8 +314,8 @@ int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, in
         dist_tile_kernel<kL2><<<grid, 256>>>(Q + q0 * dim, qb, X + x0 * dim, nb, dim, unsafe_D, NB);
       else
         dist_tile_kernel<kIP><<<grid, 256>>>(Q + q0 * dim, qb, X + x0 * dim, nb, dim, unsafe_D, NB);
-      select_kernel<<<(unsigned)((qb + SEL_WARPS - 1) / SEL_WARPS), SEL_WARPS * 32, sel_smem>>>(
-          unsafe_D, NB, (int)qb, nb, x0, q0, self_base, k, (unsigned long long*)hstate.p);
+      select_kernel<0><<<(unsigned)((qb + SEL_WARPS - 1) / SEL_WARPS), SEL_WARPS * 32, sel_smem>>>(
+          unsafe_D, NB, (int)qb, nb, x0, q0, self_base, k, (unsigned long long*)hstate.p, nullptr, nullptr, self_ids);
     }
     decode_state_kernel<<<(unsigned)((ns + 255) / 256), 256>>>((unsigned long long*)hstate.p, ns, (uint32_t*)hid.p,
                                                                (float*)hd.p);
@@ -317,6 +326,289 @@ int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, in
   (void)dev_out;
   ALGAS_CUDA_TRY(cudaDeviceSynchronize());
   return ALGAS_OK;
+}
+
+
+// ------------------------------------------------------------------ tensor-core screened kNN
+// The kNN distance block is a dense contraction: |q|^2 + |x|^2 - 2 q.x with
+// q.x from cuBLAS tensor-core GEMMs in 3xTF32 (hi/lo split, ~fp32 accuracy),
+// screening the top K2 = k + margin candidates per query; the candidates are
+// re-ranked with the exact direct-form fp32 distance (the same arithmetic as
+// knn_direct), and a per-query certificate
+//     screened_dist(K2-th) - eps  >  exact_dist(k-th)
+// with eps a rigorous bound on |screened - exact| proves that no unscreened
+// point can enter the top k; queries failing it are redone by knn_direct.
+// The output is therefore identical to knn_direct's.
+__device__ __forceinline__ float tf32_hi(float v) {
+  uint32_t h;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(h) : "f"(v));
+  return __uint_as_float(h);
+}
+__global__ void split_tf32_kernel(const float* __restrict__ in, size_t count, float* __restrict__ hi,
+                                  float* __restrict__ lo) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= count) return;
+  const float v = in[i];
+  const float h = tf32_hi(v);
+  hi[i] = h;
+  lo[i] = v - h;  // exact: v - h has at most 14 significant bits
+}
+// squared norms (sequential fp32 FMA over dims, one thread per row) and the
+// running maximum (non-negative floats order like their bit patterns)
+__global__ void norms_kernel(const float* __restrict__ X, int64_t n, int d, float* __restrict__ out,
+                             unsigned int* __restrict__ maxbits) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const float4* r = reinterpret_cast<const float4*>(X + i * d);
+  float acc = 0.f;
+  for (int j = 0; j < d / 4; ++j) {
+    const float4 v = r[j];
+    acc = fmaf(v.x, v.x, acc); acc = fmaf(v.y, v.y, acc); acc = fmaf(v.z, v.z, acc); acc = fmaf(v.w, v.w, acc);
+  }
+  out[i] = acc;
+  if (maxbits) atomicMax(maxbits, __float_as_uint(acc));
+}
+// one warp per query: exact distances of its K2 screened candidates (same
+// arithmetic as dist_tile_kernel: sequential FMA over dims), sort, keep k,
+// and the certificate.  K2 <= KMAX (power of two, smem bitonic sort).
+template <int METRIC, int KMAX>
+__global__ void __launch_bounds__(128) rerank_kernel(const float* __restrict__ Q, int64_t qn, const float* __restrict__ X,
+                                                     int d, const unsigned long long* __restrict__ state, int K2,
+                                                     int k, const float* __restrict__ qnorm, float xmax, float eps_c,
+                                                     uint32_t* __restrict__ out_ids, float* __restrict__ out_d,
+                                                     int* __restrict__ fail) {
+  __shared__ unsigned long long keys[4][KMAX];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t row = (int64_t)blockIdx.x * 4 + warp;
+  if (row >= qn) return;
+  unsigned long long* kk = keys[warp];
+  const unsigned long long* st = state + row * K2;
+  const float* q = Q + row * d;
+  for (int i = lane; i < KMAX; i += 32) {
+    unsigned long long key = kKeyMax;
+    if (i < K2 && st[i] != kKeyMax) {
+      const uint32_t id = key_id(st[i]);
+      const float4* xr = reinterpret_cast<const float4*>(X + (int64_t)id * d);
+      const float4* qr = reinterpret_cast<const float4*>(q);
+      float acc = 0.f;
+      for (int j = 0; j < d / 4; ++j) {
+        const float4 a = qr[j], b = xr[j];
+        if (METRIC == kL2) {
+          float t = a.x - b.x; acc = fmaf(t, t, acc);
+          t = a.y - b.y; acc = fmaf(t, t, acc);
+          t = a.z - b.z; acc = fmaf(t, t, acc);
+          t = a.w - b.w; acc = fmaf(t, t, acc);
+        } else {
+          acc = fmaf(a.x, b.x, acc); acc = fmaf(a.y, b.y, acc); acc = fmaf(a.z, b.z, acc); acc = fmaf(a.w, b.w, acc);
+        }
+      }
+      key = make_key(METRIC == kL2 ? acc : -acc, id);
+    }
+    kk[i] = key;
+  }
+  __syncwarp();
+  for (int size = 2; size <= KMAX; size <<= 1)
+    for (int j = size >> 1; j > 0; j >>= 1) {
+      for (int t = lane; t < KMAX / 2; t += 32) {
+        const int lo = 2 * j * (t / j) + (t % j), hi = lo + j;
+        const bool up = (lo & size) == 0;
+        const unsigned long long a = kk[lo], b = kk[hi];
+        if ((a > b) == up) { kk[lo] = b; kk[hi] = a; }
+      }
+      __syncwarp();
+    }
+  for (int i = lane; i < k; i += 32) {
+    const unsigned long long key = kk[i];
+    out_ids[row * k + i] = key == kKeyMax ? kSentinel : key_id(key);
+    out_d[row * k + i] = key == kKeyMax ? __int_as_float(0x7f800000) : key_dist(key);
+  }
+  if (lane == 0) {
+    const unsigned long long thr = st[K2 - 1];
+    int ok = 1;
+    if (thr != kKeyMax) {  // else every point was screened
+      const float qq = qnorm[row];
+      const float eps = METRIC == kL2 ? eps_c * (qq + xmax) : eps_c * sqrtf(qq) * sqrtf(xmax);
+      const unsigned long long kth = kk[k - 1];
+      ok = (kth != kKeyMax) && (key_dist(thr) - eps > key_dist(kth));
+    }
+    fail[row] = !ok;
+  }
+}
+__global__ void gather_rows_kernel(const float* __restrict__ Q, int d, const int64_t* __restrict__ rows, int m,
+                                   float* __restrict__ out) {
+  const int i = blockIdx.x;
+  for (int j = threadIdx.x; j < d; j += blockDim.x) out[(int64_t)i * d + j] = Q[rows[i] * d + j];
+}
+__global__ void scatter_results_kernel(const uint32_t* __restrict__ ids, const float* __restrict__ ds, int k,
+                                       const int64_t* __restrict__ rows, int m, uint32_t* __restrict__ out_ids,
+                                       float* __restrict__ out_d) {
+  const int i = blockIdx.x;
+  for (int j = threadIdx.x; j < k; j += blockDim.x) {
+    out_ids[rows[i] * k + j] = ids[(int64_t)i * k + j];
+    out_d[rows[i] * k + j] = ds[(int64_t)i * k + j];
+  }
+}
+
+static std::mutex g_cublas_mu;
+static cublasHandle_t cublas_handle() {
+  static cublasHandle_t h[64] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(g_cublas_mu);
+  if (!h[dev & 63]) cublasCreate(&h[dev & 63]);
+  return h[dev & 63];
+}
+#define ALGAS_CUBLAS_TRY(expr)                                                                   \
+  do {                                                                                           \
+    cublasStatus_t _s = (expr);                                                                  \
+    if (_s != CUBLAS_STATUS_SUCCESS)                                                             \
+      return ::algas::set_error(ALGAS_ECUDA, "%s failed: cublas status %d", #expr, (int)_s);     \
+  } while (0)
+
+// screened-path statistics of the last call on this thread (tests, bench)
+static thread_local int64_t g_knn_screened_rows = 0, g_knn_fallback_rows = 0;
+
+static int knn_screened(const float* X, int64_t n, const float* Q, int64_t nq, int32_t d, int32_t metric, int32_t k,
+                        int64_t self_base, uint32_t* out_ids, float* out_dists) {
+  const int margin = std::max(32, k / 2);
+  const int K2 = (int)std::min<int64_t>(k + margin, 256);
+  const int64_t QB = std::min<int64_t>(nq, 4096);
+  const int64_t NB = std::min<int64_t>(n, 65536);
+  Dev hxh, hxl, hqh, hql, hxn, hqn, hmax, hstate, hD, hid, hd, hfail, hrows, hself, hqf, hfid, hfd;
+  ALGAS_CUDA_TRY(cudaMalloc(&hxh.p, (size_t)n * d * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hxl.p, (size_t)n * d * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hqh.p, (size_t)QB * d * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hql.p, (size_t)QB * d * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hxn.p, (size_t)n * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hqn.p, (size_t)nq * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hmax.p, 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hstate.p, (size_t)QB * K2 * 8));
+  ALGAS_CUDA_TRY(cudaMalloc(&hD.p, (size_t)QB * NB * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hid.p, (size_t)QB * k * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hd.p, (size_t)QB * k * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hfail.p, (size_t)QB * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hrows.p, (size_t)QB * 8));
+  float *Xh = (float*)hxh.p, *Xl = (float*)hxl.p, *Qh = (float*)hqh.p, *Ql = (float*)hql.p;
+  float *xn = (float*)hxn.p, *qn = (float*)hqn.p;
+  ALGAS_CUDA_TRY(cudaMemset(hmax.p, 0, 4));
+  const size_t nx = (size_t)n * d;
+  split_tf32_kernel<<<(unsigned)((nx + 255) / 256), 256>>>(X, nx, Xh, Xl);
+  norms_kernel<<<(unsigned)((n + 255) / 256), 256>>>(X, n, d, xn, (unsigned int*)hmax.p);
+  norms_kernel<<<(unsigned)((nq + 255) / 256), 256>>>(Q, nq, d, qn, nullptr);
+  unsigned int maxbits = 0;
+  ALGAS_CUDA_TRY(cudaMemcpy(&maxbits, hmax.p, 4, cudaMemcpyDeviceToHost));
+  float xmax;
+  memcpy(&xmax, &maxbits, 4);
+  // rigorous screening error bound, relative to |q|^2 + max|x|^2 (L2) or
+  // |q| max|x| (IP): operand split/rounding 3 * 2^-22, fp32 accumulation of
+  // the GEMMs, the norms and the direct form gamma_(d+8), final roundings
+  const double u = std::ldexp(1.0, -24);
+  const double gam = (d + 8) * u / (1.0 - (d + 8) * u);
+  const float eps_c = (float)(1.05 * (4.0 * gam + 8.0 * std::ldexp(1.0, -22)));
+  cublasHandle_t h = cublas_handle();
+  ALGAS_CUBLAS_TRY(cublasSetStream(h, 0));
+  const int sel_smem = SEL_WARPS * (2 * K2 + SEL_BUF) * 8;
+  void* sel = metric == ALGAS_L2 ? (void*)select_kernel<1> : (void*)select_kernel<2>;
+  ALGAS_CUDA_TRY(cudaFuncSetAttribute(sel, cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem));
+  float* D = (float*)hD.p;
+  const float one = 1.f, zero = 0.f;
+  std::vector<int> fail((size_t)QB);
+  std::vector<int64_t> frows;
+  for (int64_t q0 = 0; q0 < nq; q0 += QB) {
+    const int64_t qb = std::min<int64_t>(QB, nq - q0);
+    const size_t ns = (size_t)qb * K2;
+    init_state_kernel<<<(unsigned)((ns + 255) / 256), 256>>>((unsigned long long*)hstate.p, ns);
+    split_tf32_kernel<<<(unsigned)((qb * d + 255) / 256), 256>>>(Q + q0 * d, (size_t)qb * d, Qh, Ql);
+    for (int64_t x0 = 0; x0 < n; x0 += NB) {
+      const int64_t nb = std::min<int64_t>(NB, n - x0);
+      // D^T (col-major nb x qb, ld NB) = X_blk . Q_blk^T: hi.hi + lo.hi + hi.lo
+      const float* A[3] = {Xh + x0 * d, Xl + x0 * d, Xh + x0 * d};
+      const float* B[3] = {Qh, Qh, Ql};
+      for (int g = 0; g < 3; ++g)
+        ALGAS_CUBLAS_TRY(cublasGemmEx(h, CUBLAS_OP_T, CUBLAS_OP_N, (int)nb, (int)qb, d, &one, A[g], CUDA_R_32F, d,
+                                      B[g], CUDA_R_32F, d, g == 0 ? &zero : &one, D, CUDA_R_32F, (int)NB,
+                                      CUBLAS_COMPUTE_32F_FAST_TF32, CUBLAS_GEMM_DEFAULT));
+      if (metric == ALGAS_L2)
+        select_kernel<1><<<(unsigned)((qb + SEL_WARPS - 1) / SEL_WARPS), SEL_WARPS * 32, sel_smem>>>(
+            D, NB, (int)qb, nb, x0, q0, self_base, K2, (unsigned long long*)hstate.p, qn, xn, nullptr);
+      else
+        select_kernel<2><<<(unsigned)((qb + SEL_WARPS - 1) / SEL_WARPS), SEL_WARPS * 32, sel_smem>>>(
+            D, NB, (int)qb, nb, x0, q0, self_base, K2, (unsigned long long*)hstate.p, qn, xn, nullptr);
+    }
+    const unsigned rb = (unsigned)((qb + 3) / 4);
+    if (metric == ALGAS_L2)
+      rerank_kernel<kL2, 256><<<rb, 128>>>(Q + q0 * d, qb, X, d, (unsigned long long*)hstate.p, K2, k, qn + q0, xmax,
+                                            eps_c, (uint32_t*)hid.p, (float*)hd.p, (int*)hfail.p);
+    else
+      rerank_kernel<kIP, 256><<<rb, 128>>>(Q + q0 * d, qb, X, d, (unsigned long long*)hstate.p, K2, k, qn + q0, xmax,
+                                            eps_c, (uint32_t*)hid.p, (float*)hd.p, (int*)hfail.p);
+    ALGAS_CUDA_TRY(cudaGetLastError());
+    ALGAS_CUDA_TRY(cudaMemcpy(fail.data(), hfail.p, (size_t)qb * 4, cudaMemcpyDeviceToHost));
+    frows.clear();
+    for (int64_t i = 0; i < qb; ++i)
+      if (fail[i]) frows.push_back(i);
+    g_knn_screened_rows += qb;
+    g_knn_fallback_rows += (int64_t)frows.size();
+    if (!frows.empty()) {
+      // redo the uncertified queries exactly on CUDA cores
+      const int m = (int)frows.size();
+      std::vector<int64_t> selfs(m);
+      for (int i = 0; i < m; ++i) selfs[i] = self_base >= 0 ? self_base + q0 + frows[i] : -1;
+      Dev a, b, c, e, f;
+      ALGAS_CUDA_TRY(cudaMalloc(&a.p, (size_t)m * 8));
+      ALGAS_CUDA_TRY(cudaMalloc(&b.p, (size_t)m * 8));
+      ALGAS_CUDA_TRY(cudaMalloc(&c.p, (size_t)m * d * 4));
+      ALGAS_CUDA_TRY(cudaMalloc(&e.p, (size_t)m * k * 4));
+      ALGAS_CUDA_TRY(cudaMalloc(&f.p, (size_t)m * k * 4));
+      ALGAS_CUDA_TRY(cudaMemcpy(a.p, frows.data(), (size_t)m * 8, cudaMemcpyHostToDevice));
+      ALGAS_CUDA_TRY(cudaMemcpy(b.p, selfs.data(), (size_t)m * 8, cudaMemcpyHostToDevice));
+      gather_rows_kernel<<<m, 128>>>(Q + q0 * d, d, (const int64_t*)a.p, m, (float*)c.p);
+      int rc = knn_direct(X, n, (const float*)c.p, m, d, metric, k, -1, (const int64_t*)b.p, (uint32_t*)e.p,
+                          (float*)f.p);
+      if (rc) return rc;
+      scatter_results_kernel<<<m, 128>>>((const uint32_t*)e.p, (const float*)f.p, k, (const int64_t*)a.p, m,
+                                         (uint32_t*)hid.p, (float*)hd.p);
+      ALGAS_CUDA_TRY(cudaGetLastError());
+    }
+    ALGAS_CUDA_TRY(cudaMemcpy(out_ids + q0 * k, hid.p, (size_t)qb * k * 4, cudaMemcpyDefault));
+    ALGAS_CUDA_TRY(cudaMemcpy(out_dists + q0 * k, hd.p, (size_t)qb * k * 4, cudaMemcpyDefault));
+  }
+  ALGAS_CUDA_TRY(cudaDeviceSynchronize());
+  return ALGAS_OK;
+}
+
+}  // namespace algas
+
+using namespace algas;
+
+extern "C" {
+
+int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, int32_t dim, int32_t metric, int32_t k,
+              int64_t self_base, uint32_t* out_ids, float* out_dists) {
+  if (!base || !queries || !out_ids || !out_dists || n < 1 || n >= (1LL << 31) || nq < 0 || dim < 4 ||
+      dim % 4 != 0 || k < 1 || k > 1024 || (metric != ALGAS_L2 && metric != ALGAS_IP))
+    return set_error(ALGAS_EINVAL, "algas_knn: bad arguments");
+  if (nq == 0) return ALGAS_OK;
+  Dev hx, hq;
+  const float *X = nullptr, *Q = nullptr;
+  int rc;
+  if ((rc = to_device(base, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
+  if ((rc = to_device(queries, (size_t)nq * dim * 4, hq, (const void**)&Q))) return rc;
+  // path: tensor-core screen + exact rerank + certificate (default for large
+  // problems), or the direct CUDA-core path; ALGAS_KNN_MODE=direct|screened
+  const char* env = getenv("ALGAS_KNN_MODE");
+  bool screened = (double)n * (double)nq >= 1e8 && k + std::max(32, k / 2) <= 256;
+  if (env && !strcmp(env, "direct")) screened = false;
+  if (env && !strcmp(env, "screened")) screened = k + std::max(32, k / 2) <= 256;
+  if (screened) return knn_screened(X, n, Q, nq, dim, metric, k, self_base, out_ids, out_dists);
+  return knn_direct(X, n, Q, nq, dim, metric, k, self_base, nullptr, out_ids, out_dists);
+}
+
+int64_t algas_knn_last_stats(int64_t* fallback_rows) {
+  if (fallback_rows) *fallback_rows = g_knn_fallback_rows;
+  const int64_t r = g_knn_screened_rows;
+  g_knn_screened_rows = g_knn_fallback_rows = 0;
+  return r;
 }
 
 int algas_prune(const uint32_t* knn, int64_t n, int32_t knn_degree, int32_t degree, uint32_t* out_graph) {

@@ -420,17 +420,19 @@ int algas_device_query(algas_device_props* out) {
   return ALGAS_OK;
 }
 
-// Full tuner.  Policy (DESIGN.md §6, "tuner"):
-//  * threads/CTA: the paper fixes one warp; on B200 a search step is
-//    latency-bound (dependent select -> gather -> distance -> merge) and the
-//    per-SM random-gather rate grows with loads in flight, so 8 warps
-//    (measured: 64 -> 256 threads = 2x QPS at C2, profiles/round1_c2.md).
-//  * N_parallel: the largest T allowed by P:L231 whose per-block shared memory
-//    fits P:L245 (with M_reserved grown for wide vectors), capped at
-//    T_cap = 8 beyond which extra CTAs mostly repeat work (measured in
-//    profiles/); small batches get the most CTAs per query.
-//  * width / offset_beam: beam extend in the diffusing phase:
-//    w = 1 for L <= 32, 2 for L <= 64, 4 above; off = L/4 (R6).
+// Full tuner.  Policy (DESIGN.md §7, "tuner"):
+//  * threads/CTA: the paper fixes one warp.  On B200 a search step
+//    is latency-bound (dependent select -> gather -> distance -> merge); a
+//    step's wave of row reads completes fastest with 16 warps holding all its
+//    rows in flight (profiles/dist_wave_microbench_ordered.txt), so 512.
+//  * N_parallel: the largest T allowed by P:L231 -- with N_max_block_per_SM
+//    = 1, the occupancy of a 512-thread search CTA (its registers fill the
+//    register file) -- whose per-block shared memory fits P:L245 (with
+//    M_reserved grown for wide vectors), capped at T_cap = 8.
+//  * width / offset_beam: beam extend from the first step
+//    (offset_beam = 1): every step has a fixed latency of ~2 DRAM
+//    round trips plus barriers, so fewer, wider steps win on B200 at equal
+//    recall (profiles/round1_explore_C2.txt); w = 8 up to L = 64, 16 above.
 int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int32_t degree, int32_t itopk, int32_t k,
                algas_tuning* out) {
   if (!out || slots < 1 || dim < 4 || degree < 1 || itopk < 1 || k < 1)
@@ -441,8 +443,9 @@ int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int3
     if (rc) return rc;
     props = &dp;
   }
-  const int nt = 256;
-  const int w = itopk <= 32 ? 1 : (itopk <= 64 ? 2 : 4);
+  const int nt = props->max_threads_per_sm >= 512 ? 512 : 256;
+  const int search_blocks_per_sm = 1;  // occupancy of one wide search CTA
+  const int w = std::min(itopk, itopk <= 64 ? 8 : 16);
   int Rp = 4;
   while (Rp < degree) Rp <<= 1;
   const int S = 32;
@@ -453,7 +456,7 @@ int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int3
   const int dp4 = chunk_tl(cc) * chunk_cpl(cc);
   // M_reserved_per_block: driver reservation + extra L1 for wide rows
   const int64_t reserved = props->smem_reserved_per_block + (dim > 256 ? 8 * 1024 : 0);
-  const int tmax_eq = algas_tuner_max_parallel(slots, props->n_sm, props->max_blocks_per_sm);
+  const int tmax_eq = algas_tuner_max_parallel(slots, props->n_sm, std::min(props->max_blocks_per_sm, search_blocks_per_sm));
   const int tcap = std::min(8, ALGAS_MAX_CTAS);
   int best = 0, best_bps = 0, best_hb = 0, best_sr = 0;
   int64_t best_avail = 0, best_smem = 0;
@@ -483,7 +486,7 @@ int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int3
   out->smem_per_block = best_smem;
   out->threads_per_cta = nt;
   out->width = w;
-  out->offset_beam = std::max(1, itopk / 4);
+  out->offset_beam = 1;
   out->hash_bits = best_hb;
   out->stage_rows = best_sr;
   (void)k;

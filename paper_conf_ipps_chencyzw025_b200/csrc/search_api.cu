@@ -3,6 +3,7 @@
 // (algas_search_dynamic).  The host merge of per-CTA results is in
 // runtime.cu; graph construction in knn.cu.
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstring>
 #include <thread>
@@ -80,8 +81,8 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
     if (nt == 0) nt = tu.threads_per_cta;
   }
   if (T < 1 || T > ALGAS_MAX_CTAS) return set_error(ALGAS_EINVAL, "ctas_per_query %d not in [1,%d]", T, ALGAS_MAX_CTAS);
-  if (nt != 32 && nt != 64 && nt != 128 && nt != 256)
-    return set_error(ALGAS_EINVAL, "threads_per_cta %d not in {32,64,128,256}", nt);
+  if (nt != 32 && nt != 64 && nt != 128 && nt != 256 && nt != 512 && nt != 1024)
+    return set_error(ALGAS_EINVAL, "threads_per_cta %d not in {32,64,128,256,512,1024}", nt);
   const int cc = chunk_config_for(idx->d4);
   if (cc < 0) return set_error(ALGAS_EINVAL, "dim %d unsupported", idx->dim);
   const int Rp = 1 << idx->rp_shift;
@@ -503,6 +504,7 @@ int algas_search_ex(const algas_index* cidx, const float* queries, int64_t nq, c
 int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int64_t nq, const algas_params* params,
                          uint64_t tag0, uint32_t* out_ids, float* out_dists, algas_query_stats* out_stats,
                          void* stream, algas_run_info* info) {
+  const auto t_entry = std::chrono::steady_clock::now();
   algas_index* idx = const_cast<algas_index*>(cidx);
   if (!idx || !params || !queries_dev || !out_ids || !out_dists || nq < 0)
     return set_error(ALGAS_EINVAL, "algas_search_dynamic: null argument");
@@ -562,8 +564,14 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   ALGAS_CUDA_TRY(cudaGetLastError());
   if (info) fill_info(info, pl, ctas, tm.ms());
   bool ovf = false;
+  const auto t_merge = std::chrono::steady_clock::now();
   if ((rc = finish_outputs(res, cst, nq, pl.T, pl.k, pl.k, out_ids, out_dists, nullptr, nullptr, out_stats, &ovf)))
     return rc;
+  if (info) {
+    const auto t_end = std::chrono::steady_clock::now();
+    info->merge_ms = std::chrono::duration<float, std::milli>(t_end - t_merge).count();
+    info->call_ms = std::chrono::duration<float, std::milli>(t_end - t_entry).count();
+  }
   return ovf ? set_error(ALGAS_EOVERFLOW, "a visited table overflowed") : ALGAS_OK;
 }
 

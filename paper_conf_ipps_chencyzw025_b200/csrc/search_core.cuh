@@ -152,6 +152,27 @@ __device__ __forceinline__ float4 ldg_f4_stream(const float4* p) {
   return r;
 }
 
+// Row gathers of the distance step.  Volatile (strong, sys-scope) loads:
+// ptxas keeps volatile memory operations in program order, so every row
+// load of a pass is issued before the (volatile) query reads that the FMAs
+// depend on -- the only robust way to keep all loads of a wave in flight
+// (plain loads get interleaved with FMAs by the scheduler, serialising the
+// round trips).  Device memory: served by L2 like .cg.
+__device__ __forceinline__ float4 ld_row_f4(const float4* p) {
+  float4 r;
+  asm volatile("ld.volatile.global.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float4 lds_f4_ordered(const float4* p) {
+  float4 r;
+  asm volatile("ld.volatile.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "r"(smem_u32(p)));
+  return r;
+}
+
 struct SearchCfg {
   const float4* data;    // n x d4 float4 (row-major, 16-B aligned rows)
   const uint32_t* graph; // n x Rp u32 (Rp = 1 << rp_shift, padded with sentinels)
@@ -196,8 +217,11 @@ struct Ctrl {
 enum { kCmdStep = 1, kCmdQuit = 2 };
 
 // Shared-memory carve-up (bytes, all 16-B aligned).
+// scratch ints for the merge's partial rank counts (>= the widest CTA)
+constexpr int kMergeParts = 1024;
+
 struct SmemLayout {
-  int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_hash, off_stage, off_bar, off_ctrl, total;
+  int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_part, off_hash, off_stage, off_bar, off_ctrl, total;
 };
 __host__ __device__ inline int align16(int x) { return (x + 15) & ~15; }
 __host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int hash_bits, int stage_rows) {
@@ -210,6 +234,7 @@ __host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int 
   s.off_newk = o;  o += align16(ncap * 8);
   s.off_newid = o; o += align16(ncap * 4);
   s.off_sel = o;   o += align16(64 * 4);
+  s.off_part = o;  o += kMergeParts * 4;  // partial ranks of the split merge
   s.off_hash = o;  o += align16((1 << hash_bits) * 4);
   s.off_bar = o;   o += 32;
   s.off_ctrl = o;  o += align16((int)sizeof(Ctrl));
@@ -223,6 +248,7 @@ struct Smem {
   uint64_t* newk;
   uint32_t* newid;
   int* sel;         // [0,32): selected positions, [32,64): parent ids
+  int* part;        // kMergeParts partial rank counts (merge)
   uint32_t* hash;
   float4* stage;    // 2 x stage_rows x dp4
   uint64_t* bar;    // 2 mbarriers
@@ -236,6 +262,7 @@ __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
   s.newk = reinterpret_cast<uint64_t*>(base + l.off_newk);
   s.newid = reinterpret_cast<uint32_t*>(base + l.off_newid);
   s.sel = reinterpret_cast<int*>(base + l.off_sel);
+  s.part = reinterpret_cast<int*>(base + l.off_part);
   s.hash = reinterpret_cast<uint32_t*>(base + l.off_hash);
   s.stage = reinterpret_cast<float4*>(base + l.off_stage);
   s.bar = reinterpret_cast<uint64_t*>(base + l.off_bar);
@@ -425,20 +452,39 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
 
 // Distance step for rows r = r0, r0+rstep, ... < M of newid (P:L217 step 3):
 // LDG.128 straight into registers, each team keeping B rows in flight
-// (NT/TL*B rows per CTA), interleaved shuffle-tree reductions, prefilter
-// against `worst`, one warp-wide scan + one atomic per warp to append the
-// surviving keys to newk.  newid/newk/nkeys may live in another CTA's
-// shared memory (cluster leader).
-template <int NT, int TL, int CPL, int METRIC>
-__device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const QueryRegs<TL, CPL>& Q, int M, int r0, int rstep,
+// (NT/TL*B rows per CTA and pass), interleaved shuffle-tree reductions,
+// prefilter against `worst`, ballot compaction + one atomic per warp to
+// append the surviving keys to newk.  newid/newk/nkeys may live in another
+// CTA's shared memory (cluster leader).
+//
+// A step's wave of row reads is latency-bound, and its fixed cost is
+// instruction issue (profiles/dist_wave_microbench*.txt): warps with no row
+// in a pass skip it entirely (warp-uniform test), and the compaction is one
+// ballot per row group instead of a warp scan.
+template <int NT, int TL, int CPL>
+struct DistRows {
+  // rows in flight per team and pass: the wave's rows all in flight at once
+  // within the register budget (<= 64 registers per thread at 1024 threads,
+  // <= 128 at 512)
+  static constexpr int BW = NT >= 1024 ? 4 : 16;
+  static constexpr int B = CPL >= BW ? 1 : BW / CPL;
+};
+template <int NT, int TL, int CPL, int METRIC, int BOVR = 0>
+__device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs, int M, int r0, int rstep,
                                          uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys) {
   const int tid = threadIdx.x, lane = tid & 31;
   constexpr int NTEAMS = NT / TL;
+  constexpr int TPW = 32 / TL;  // teams per warp
   const int team = tid / TL, tl = tid % TL;
-  constexpr int B = CPL >= 16 ? 1 : 16 / CPL;
+  const int wteam0 = (tid >> 5) * TPW;  // first team of this warp
+  constexpr int B = BOVR > 0 ? BOVR : DistRows<NT, TL, CPL>::B;
   constexpr int PASS = NTEAMS * B;
-  const int Mc = M > r0 ? (M - r0 + rstep - 1) / rstep : 0;  // rows of this CTA
+  const int Mc = M > r0 ? (rstep == 1 ? M - r0 : (M - r0 + rstep - 1) / rstep) : 0;  // rows of this CTA
   for (int base = 0; base < Mc; base += PASS) {
+    // row groups of this pass that hold any row of THIS warp (warp-uniform):
+    // loads, FMAs, shuffles and compaction of empty groups are skipped
+    const int nbw = (Mc - base - wteam0 + NTEAMS - 1) / NTEAMS;
+    if (nbw <= 0) continue;
     float4 v[B][CPL];
     uint32_t ids[B];
 #pragma unroll
@@ -453,21 +499,20 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const QueryRegs<T
 #pragma unroll
       for (int c = 0; c < CPL; ++c) {
         const int chn = tl + c * TL;
-        v[b][c] = (j < Mc && chn < cfg.d4) ? ldg_f4_stream(row + chn) : make_float4(0.f, 0.f, 0.f, 0.f);
+        v[b][c] = (b < nbw && j < Mc && chn < cfg.d4) ? ld_row_f4(row + chn) : make_float4(0.f, 0.f, 0.f, 0.f);
       }
     }
-    // all loads of the pass are issued before any use: the warp barrier
-    // keeps ptxas from hoisting FMAs of early rows between the loads
-    // (which would serialise the DRAM round trips)
-    __syncwarp();
-    // row groups of this pass that hold any row (uniform across the CTA):
-    // the FMA and shuffle work of empty groups is skipped
-    const int nb = (Mc - base + NTEAMS - 1) / NTEAMS;
+    // the query chunks are read (volatile) only after every row load of the
+    // pass was issued; the FMAs depend on them, so no FMA can be scheduled
+    // between the row loads (which would serialise the DRAM round trips)
+    QueryRegs<TL, CPL> Q;
+#pragma unroll
+    for (int c = 0; c < CPL; ++c) Q.q[c] = lds_f4_ordered(qs + tl + c * TL);
     float acc[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       float a = 0.f;
-      if (b >= nb) {
+      if (b >= nbw) {
         acc[b] = 0.f;
         continue;
       }
@@ -488,31 +533,30 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const QueryRegs<T
     for (int o = TL >> 1; o > 0; o >>= 1)
 #pragma unroll
       for (int b = 0; b < B; ++b)
-        if (b < nb) acc[b] += __shfl_xor_sync(0xffffffffu, acc[b], o);
-    uint64_t key[B];
-    int nkeep = 0;
+        if (b < nbw) acc[b] += __shfl_xor_sync(0xffffffffu, acc[b], o);
+    // compaction: one ballot per row group; lane 0 reserves the warp's slots
+    unsigned m[B];
+    int tot = 0;
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       const int j = base + b * NTEAMS + team;
-      key[b] = kKeyMax;
-      if (tl == 0 && j < Mc) key[b] = make_key((METRIC == kL2) ? acc[b] : -acc[b], ids[b]);
-      nkeep += (key[b] < worst) ? 1 : 0;
+      uint64_t key = kKeyMax;
+      if (b < nbw && tl == 0 && j < Mc) key = make_key((METRIC == kL2) ? acc[b] : -acc[b], ids[b]);
+      m[b] = b < nbw ? __ballot_sync(0xffffffffu, key < worst) : 0u;
+      tot += __popc(m[b]);
+      acc[b] = __uint_as_float((uint32_t)(key >> 32));  // keep the key's high word (id is in ids[b])
     }
-    int incl = nkeep;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int t = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += t;
-    }
-    const int wtotal = __shfl_sync(0xffffffffu, incl, 31);
-    if (wtotal > 0) {
+    if (tot > 0) {
       int wbase = 0;
-      if (lane == 0) wbase = atomicAdd(nkeys, wtotal);
+      if (lane == 0) wbase = atomicAdd(nkeys, tot);
       wbase = __shfl_sync(0xffffffffu, wbase, 0);
-      int pos = wbase + incl - nkeep;
+      const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
-      for (int b = 0; b < B; ++b)
-        if (key[b] < worst) newk[pos++] = key[b];
+      for (int b = 0; b < B; ++b) {
+        if (m[b] & (1u << lane))
+          newk[wbase + __popc(m[b] & lt)] = ((uint64_t)__float_as_uint(acc[b]) << 32) | ((uint64_t)ids[b] << 1);
+        wbase += __popc(m[b]);
+      }
     }
   }
 }
@@ -548,8 +592,6 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     C->vis_count = 0; C->spilled = 0; C->overflow = 0; C->cur = 0;
     C->iters = 0; C->parents = 0; C->dist_evals = 0; C->cap_hit = 0;
   }
-  QueryRegs<TL, CPL> Q;
-  Q.load(s.q, tl);
   uint32_t phase = C->phase;  // staging-barrier parities carried across queries
   __syncthreads();
 
@@ -716,18 +758,20 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
             fence_cluster();
             mbar_remote_arrive(s.bar + 2, c);
           }
-          dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
+          dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
           mbar_wait_cluster(s.bar + 3, (phase >> 3) & 1u);  // all workers' keys delivered
           phase ^= 8u;
           __syncthreads();
         } else {
-          dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, 1, worst, s.newid, s.newk, &C->nkeys);
+          dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, 1, worst, s.newid, s.newk, &C->nkeys);
           __syncthreads();
         }
       }
       const int SR = cfg.stage_rows;
       const int nchunks = cfg.gather_mode == 0 ? 0 : (M + SR - 1) / SR;
       if (nchunks > 0) stage_issue<NT>(cfg, s, 0, 0, M < SR ? M : SR, warp, lane);
+      QueryRegs<TL, CPL> Q;  // staged paths: the query in registers for the chunk loop
+      if (nchunks > 0) Q.load(s.q, tl);
       for (int ch = 0; ch < nchunks; ++ch) {
         const int b = ch & 1;
         if (ch + 1 < nchunks) {
@@ -794,19 +838,44 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       if (nk > 0) {
         const uint64_t* src = cur ? s.list[1] : s.list[0];
         uint64_t* dst = cur ? s.list[0] : s.list[1];
-        for (int i = tid; i < nk; i += NT) {
-          const uint64_t key = s.newk[i];
-          int rn = 0;
-          for (int j = 0; j < nk; ++j) rn += (s.newk[j] < key) ? 1 : 0;
-          const int pos = rn + lower_bound_u64(src, cnt, key);
-          if (pos < L) dst[pos] = key;
-        }
-        for (int j = tid; j < cnt; j += NT) {
-          const uint64_t key = src[j];
-          int rn = 0;
-          for (int i = 0; i < nk; ++i) rn += (s.newk[i] < key) ? 1 : 0;
-          const int pos = j + rn;
-          if (pos < L) dst[pos] = key;
+        // the nk x (nk + cnt) comparisons are split over `parts` threads per
+        // key so no thread loops over all nk new keys: partial counts go to
+        // s.part, then one thread per key sums them and writes its key
+        const int nu = nk + cnt;  // keys to place: new keys, then list keys
+        int parts = NT / nu;
+        parts = parts < 1 ? 1 : (parts > 16 ? 16 : parts);
+        if (parts * nu > kMergeParts) parts = kMergeParts / nu > 0 ? kMergeParts / nu : 1;
+        if (parts > 1) {
+          if (tid < parts * nu) {
+            const int u = tid % nu, part = tid / nu;
+            const uint64_t key = u < nk ? s.newk[u] : src[u - nk];
+            const int j0 = part * nk / parts, j1 = (part + 1) * nk / parts;
+            int rn = 0;
+            for (int j = j0; j < j1; ++j) rn += (s.newk[j] < key) ? 1 : 0;
+            if (part == 0) rn += u < nk ? lower_bound_u64(src, cnt, key) : u - nk;
+            s.part[tid] = rn;
+          }
+          __syncthreads();
+          if (tid < nu) {
+            int pos = 0;
+            for (int p = 0; p < parts; ++p) pos += s.part[p * nu + tid];
+            if (pos < L) dst[pos] = tid < nk ? s.newk[tid] : src[tid - nk];
+          }
+        } else {
+          for (int i = tid; i < nk; i += NT) {
+            const uint64_t key = s.newk[i];
+            int rn = 0;
+            for (int j = 0; j < nk; ++j) rn += (s.newk[j] < key) ? 1 : 0;
+            const int pos = rn + lower_bound_u64(src, cnt, key);
+            if (pos < L) dst[pos] = key;
+          }
+          for (int j = tid; j < cnt; j += NT) {
+            const uint64_t key = src[j];
+            int rn = 0;
+            for (int i = 0; i < nk; ++i) rn += (s.newk[i] < key) ? 1 : 0;
+            const int pos = j + rn;
+            if (pos < L) dst[pos] = key;
+          }
         }
         cur ^= 1;
         lcnt = (cnt + nk) < L ? cnt + nk : L;
@@ -869,10 +938,8 @@ __device__ int worker_step(const SearchCfg& cfg, const Smem& s, uint32_t& phase)
   if (cmd != kCmdStep) return cmd;
   const int M = *((volatile int*)&s.ctrl->w_m);
   const uint64_t worst = *((volatile uint64_t*)&s.ctrl->w_worst);
-  QueryRegs<TL, CPL> Q;
-  Q.load(s.q, threadIdx.x % TL);
   Ctrl* LC = leader_ptr(s.ctrl);
-  dist_ldg<NT, TL, CPL, METRIC>(cfg, Q, M, 0, 1, worst, s.newid, leader_ptr(s.newk), &LC->nkeys);
+  dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, 1, worst, s.newid, leader_ptr(s.newk), &LC->nkeys);
   __syncthreads();
   if (threadIdx.x == 0) {
     fence_cluster();

@@ -1,265 +1,8 @@
-// search_kernels.cu -- the batch (static) and persistent (dynamic batching)
-// search kernels and their launchers.
-//
-//  batch_kernel      : static batching -- one launch over nq queries,
-//                      each CTA pulls (query, cta_rank) work items from an
-//                      atomic counter until the batch is drained.
-//  persistent_kernel : dynamic batching -- grid = slots x T
-//                      CTAs that never exit; each slot's rank-0 CTA polls for
-//                      work (host-mapped ring: "The CTAs in the slot
-//                      poll the state", or an HBM query queue), publishes it
-//                      through a device mailbox to the slot's other CTAs,
-//                      and every CTA publishes its own top-k + a Finish flag
-//                      (P:L170).
-#include <cooperative_groups.h>
-
-#include "internal.h"
+// search_kernels.cu -- launchers of the search kernels and the dispatch over
+// the per-thread-count kernel tables (kernels_nt.cu, kernels.cuh).
+#include "kernels.cuh"
 
 namespace algas {
-
-// ------------------------------------------------------------------ memory-order helpers
-__device__ __forceinline__ uint32_t ld_acquire_sys(const volatile uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
-  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ unsigned long long ld_acquire_gpu64(const unsigned long long* p) {
-  unsigned long long v;
-  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_gpu64(unsigned long long* p, unsigned long long v) {
-  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ unsigned int ld_acquire_gpu32(const unsigned int* p) {
-  unsigned int v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ float4 ld_volatile_f4(const float4* p) {
-  float4 r;
-  asm volatile("ld.volatile.global.v4.f32 {%0,%1,%2,%3}, [%4];"
-               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
-               : "l"(p)
-               : "memory");
-  return r;
-}
-
-// ------------------------------------------------------------------ static batch kernel
-struct BatchArgs {
-  SearchCfg cfg;
-  const float4* queries;
-  int64_t nq;
-  int32_t T, k;
-  uint64_t tag0;
-  int* work_counter;
-  ResultEntry* res;
-  CtaStats* stats;
-  unsigned long long* gtab;
-  uint32_t epoch_base;
-};
-
-template <int NT, int TL, int CPL, int METRIC>
-__global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
-  extern __shared__ __align__(128) uint8_t smem_raw[];
-  const SmemLayout lay = smem_layout(a.cfg.dp4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits, a.cfg.stage_rows);
-  const Smem s = carve(smem_raw, lay);
-  init_cta<NT>(s, a.cfg);
-  __shared__ int s_item;
-  const int64_t total = a.nq * a.T;
-  unsigned long long* gt = a.gtab ? a.gtab + ((uint64_t)blockIdx.x << a.cfg.gtab_bits) : nullptr;
-  for (;;) {
-    if (threadIdx.x == 0) s_item = atomicAdd(a.work_counter, 1);
-    __syncthreads();
-    const int64_t item = s_item;
-    if (item >= total) break;
-    const int64_t qi = item / a.T;
-    const int c = (int)(item - qi * a.T);
-    const float4* qsrc = a.queries + qi * a.cfg.d4;
-    for (int i = threadIdx.x; i < a.cfg.d4; i += NT) s.q[i] = qsrc[i];
-    __syncthreads();
-    CtaStats* st = a.stats ? a.stats + item : nullptr;
-    search_cta<NT, TL, CPL, METRIC>(a.cfg, s, a.tag0 + (uint64_t)qi, (uint32_t)c, a.k, gt,
-                                    a.epoch_base + (uint32_t)item, a.res + item * a.k, st);
-    __syncthreads();
-  }
-}
-
-// ------------------------------------------------------------------ persistent kernel
-struct PKArgs {
-  SearchCfg cfg;
-  PersistArgs p;
-};
-
-constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
-
-template <int NT, int TL, int CPL, int METRIC, int CS>
-__global__ void __launch_bounds__(NT) persistent_kernel(PKArgs A) {
-  extern __shared__ __align__(128) uint8_t smem_raw[];
-  const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows);
-  const Smem s = carve(smem_raw, lay);
-  init_cta<NT>(s, A.cfg, CS);
-  if constexpr (CS > 1) cluster_barrier();  // every CTA's mbarriers exist before any remote arrive
-  const PersistArgs& P = A.p;
-  // a search unit = one (slot, cta_rank) search = one cluster of CS CTAs
-  const int unit = blockIdx.x / CS;
-  const int crank = blockIdx.x % CS;  // rank inside the cluster (1-D clusters)
-  const int slot = unit / P.T;
-  const int rank = unit % P.T;
-  const int tid = threadIdx.x;
-  __shared__ unsigned long long s_mbox;
-  __shared__ int4 s_par;
-  __shared__ unsigned long long s_tag, s_t0;
-
-  if constexpr (CS > 1) {
-    if (crank != 0) {
-      // cluster worker: serve the leader's distance steps until it quits
-      uint32_t ph = 0;
-      while (worker_step<NT, TL, CPL, METRIC>(A.cfg, s, ph) == kCmdStep) {
-      }
-      return;
-    }
-  }
-
-  unsigned long long* gt = P.gtab ? P.gtab + ((uint64_t)unit << A.cfg.gtab_bits) : nullptr;
-  uint32_t served = 0;  // queries this CTA has finished (= last epoch in devq mode)
-  uint32_t last_epoch = 0;
-
-  for (;;) {
-    // ---------------- acquire work (rank 0) and publish it to the slot's CTAs
-    if (rank == 0) {
-      if (tid == 0) {
-        unsigned long long mb;
-        if (P.mode == 0) {
-          // host ring: poll the slot state in host memory
-          uint32_t st;
-          unsigned ns = 64;
-          for (;;) {
-            st = ld_acquire_sys(&P.ring[slot].state);
-            uint32_t kind = st & 0xFFu, ep = st >> 8;
-            if (kind == kSlotQuit) break;
-            if (kind == kSlotReady && ep != last_epoch) break;
-            __nanosleep(ns);
-            if (ns < 1024) ns <<= 1;
-          }
-          if ((st & 0xFFu) == kSlotQuit) {
-            mb = kMboxQuit;
-          } else {
-            const uint32_t ep = st >> 8;
-            // payload: params + query from mapped memory (volatile: never a stale line)
-            const volatile RingSlot* rs = &P.ring[slot];
-            int4 par = make_int4(rs->k, rs->L, rs->w, 0);
-            unsigned long long tag = rs->tag;
-            P.dparams[slot] = par;
-            P.dtag[slot] = tag;
-            mb = ((unsigned long long)ep << 32) | (unsigned long long)slot;
-          }
-        } else {
-          // device queue: wait until every CTA of the slot finished the previous query
-          while (ld_acquire_gpu32(P.slot_fin + slot) < (unsigned)(served * P.T)) __nanosleep(32);
-          int item = atomicAdd(P.queue_head, 1);
-          if (item >= P.nq) {
-            mb = kMboxQuit;
-          } else {
-            const uint32_t ep = served + 1;
-            P.dparams[slot] = make_int4(P.kmax, A.cfg.L, A.cfg.w, 0);
-            P.dtag[slot] = P.tag0 + (uint64_t)item;
-            mb = ((unsigned long long)ep << 32) | (unsigned long long)(uint32_t)item;
-          }
-        }
-        s_mbox = mb;
-        s_t0 = globaltimer();
-      }
-      __syncthreads();
-      if (s_mbox != kMboxQuit && P.mode == 0) {
-        // stage the query from host memory into the slot's HBM buffer (one PCIe read)
-        const float4* src = P.ring_q + (uint64_t)slot * A.cfg.d4;
-        float4* dst = P.qbuf + (uint64_t)slot * A.cfg.d4;
-        for (int i = tid; i < A.cfg.d4; i += NT) dst[i] = ld_volatile_f4(src + i);
-      }
-      __syncthreads();
-      if (tid == 0) {
-        __threadfence();
-        st_release_gpu64(P.mbox + slot, s_mbox);
-      }
-    } else {
-      if (tid == 0) {
-        unsigned long long mb;
-        for (;;) {
-          mb = ld_acquire_gpu64(P.mbox + slot);
-          if (mb == kMboxQuit) break;
-          if ((uint32_t)(mb >> 32) != last_epoch && (uint32_t)(mb >> 32) != 0u) break;
-          __nanosleep(32);
-        }
-        s_mbox = mb;
-        s_t0 = globaltimer();
-      }
-      __syncthreads();
-    }
-    const unsigned long long mb = s_mbox;
-    if (mb == kMboxQuit) {
-      if constexpr (CS > 1) post_quit<CS>(s);
-      break;
-    }
-    const uint32_t epoch = (uint32_t)(mb >> 32);
-    const uint32_t item = (uint32_t)mb;
-    if (tid == 0) {
-      const volatile int* vp = reinterpret_cast<const volatile int*>(P.dparams + slot);
-      s_par = make_int4(vp[0], vp[1], vp[2], vp[3]);
-      s_tag = *((volatile unsigned long long*)(P.dtag + slot));
-    }
-    __syncthreads();
-    const int4 par = s_par;
-    const uint64_t tag = s_tag;
-
-    // ---------------- stage the query into shared memory
-    const float4* qsrc = (P.mode == 0) ? P.qbuf + (uint64_t)slot * A.cfg.d4
-                                       : P.queries + (uint64_t)item * A.cfg.d4;
-    for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = (P.mode == 0) ? ld_volatile_f4(qsrc + i) : qsrc[i];
-    if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
-    __syncthreads();
-
-    SearchCfg cfg = A.cfg;
-    cfg.L = par.y;
-    cfg.w = par.z;
-    if (cfg.off > cfg.L) cfg.off = cfg.L;
-    const int k = par.x;
-    ResultEntry* out;
-    CtaStats* stp;
-    if (P.mode == 0) {
-      out = P.ring_res + ((uint64_t)slot * P.T + rank) * P.kmax;
-      stp = P.ring_stats + (uint64_t)slot * P.T + rank;
-    } else {
-      out = P.dq_res + ((uint64_t)item * P.T + rank) * P.kmax;
-      stp = P.dq_stats + (uint64_t)item * P.T + rank;
-    }
-    CtaStats local;
-    search_cta<NT, TL, CPL, METRIC, CS>(cfg, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
-                                        &local);
-    __syncthreads();
-    if (tid == 0) {
-      local.t_start = s_t0;
-      local.t_end = globaltimer();
-      *stp = local;
-    }
-    served++;
-    last_epoch = epoch;
-    __syncthreads();
-    // ---------------- Finish
-    if (tid == 0) {
-      if (P.mode == 0) {
-        __threadfence_system();
-        st_release_sys(P.ring_done + (uint64_t)slot * P.T + rank, epoch);
-      } else {
-        __threadfence();
-        atomicAdd(P.slot_fin + slot, 1u);
-      }
-    }
-  }
-}
 
 // ------------------------------------------------------------------ dispatch
 // chunk configs (TL lanes per vector, CPL float4 chunks per lane), see
@@ -275,42 +18,16 @@ int chunk_config_for(int d4) {
   return -1;
 }
 
-template <int NT, int TL, int CPL, int M>
-static void* sel_kernel(bool persist, int cs) {
-  if (!persist) return (void*)batch_kernel<NT, TL, CPL, M>;
-  switch (cs) {
-    case 1: return (void*)persistent_kernel<NT, TL, CPL, M, 1>;
-    // cluster-split searches: instantiated for the 256-thread configuration only
-    case 2: return NT == 256 ? (void*)persistent_kernel<NT, TL, CPL, M, (NT == 256 ? 2 : 1)> : nullptr;
-    case 4: return NT == 256 ? (void*)persistent_kernel<NT, TL, CPL, M, (NT == 256 ? 4 : 1)> : nullptr;
-    case 8: return NT == 256 ? (void*)persistent_kernel<NT, TL, CPL, M, (NT == 256 ? 8 : 1)> : nullptr;
-  }
-  return nullptr;
-}
-template <int NT, int M>
-static void* pick_cc(int cc, bool persist, int cs) {
-  switch (cc) {
-    case 0: return sel_kernel<NT, 2, 4, M>(persist, cs);
-    case 1: return sel_kernel<NT, 4, 4, M>(persist, cs);
-    case 2: return sel_kernel<NT, 8, 4, M>(persist, cs);
-    case 3: return sel_kernel<NT, 16, 4, M>(persist, cs);
-    case 4: return sel_kernel<NT, 32, 4, M>(persist, cs);
-    case 5: return sel_kernel<NT, 32, 8, M>(persist, cs);
-    case 6: return sel_kernel<NT, 32, 16, M>(persist, cs);
-  }
-  return nullptr;
-}
-template <int NT>
-static void* pick_metric(int metric, int cc, bool persist, int cs) {
-  return metric == kL2 ? pick_cc<NT, kL2>(cc, persist, cs) : pick_cc<NT, kIP>(cc, persist, cs);
-}
+// per-thread-count kernel tables (kernels_nt.cu, one object per NT)
 static void* kernel_for(const Plan& pl, int metric, bool persist) {
   const int cs = persist ? pl.cluster : 1;
   switch (pl.nt) {
-    case 32: return pick_metric<32>(metric, pl.ccfg, persist, cs);
-    case 64: return pick_metric<64>(metric, pl.ccfg, persist, cs);
-    case 128: return pick_metric<128>(metric, pl.ccfg, persist, cs);
-    case 256: return pick_metric<256>(metric, pl.ccfg, persist, cs);
+    case 32: return kernel_table_nt32(metric, pl.ccfg, persist, cs);
+    case 64: return kernel_table_nt64(metric, pl.ccfg, persist, cs);
+    case 128: return kernel_table_nt128(metric, pl.ccfg, persist, cs);
+    case 256: return kernel_table_nt256(metric, pl.ccfg, persist, cs);
+    case 512: return kernel_table_nt512(metric, pl.ccfg, persist, cs);
+    case 1024: return kernel_table_nt1024(metric, pl.ccfg, persist, cs);
   }
   return nullptr;
 }

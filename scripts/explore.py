@@ -75,16 +75,36 @@ def main():
     elif os.environ.get("GRID") == "pf":
         grid = [(64, 4, 1, 256, 1), (64, 8, 1, 256, 1), (64, 4, 2, 256, 1), (56, 4, 2, 256, 1), (48, 4, 4, 256, 1),
                 (56, 4, 4, 256, 1), (64, 4, 1, 128, 1)]
+    elif os.environ.get("GRID") == "nt":
+        grid = []
+        for nt in (256, 512, 1024):
+            for (L, wd, T) in [(64, 8, 1), (56, 7, 2), (48, 6, 4), (64, 4, 1), (64, 16, 1), (56, 8, 4), (96, 8, 1)]:
+                grid.append((L, wd, T, nt, 1))
+    elif os.environ.get("GRID") == "pf2":
+        grid = []
+        for pf in (0, 2, 6):
+            for (L, wd, T, off) in [(64, 8, 1, 16), (64, 8, 1, 8), (64, 8, 1, 1), (56, 7, 2, 14), (56, 7, 2, 4),
+                                    (48, 6, 4, 12), (52, 8, 4, 4)]:
+                grid.append((L, wd, T, 256, 1, off, pf))
+    elif os.environ.get("GRID") == "wide":
+        grid = []
+        for nt in (256, 512, 1024):
+            for T in (1, 2, 4):
+                for wd in (8, 16, 32):
+                    for L in (40, 48, 56, 64):
+                        grid.append((L, wd, T, nt, 1, 1, 0))
     elif os.environ.get("GRID") == "cs":
         grid = [(64, 4, 1, 256, 1), (64, 4, 1, 256, 4), (64, 8, 1, 256, 4), (64, 8, 1, 256, 8)]
     elif a.quick:
         grid = [(64, 4, 1, 256, 1), (64, 4, 1, 256, 2), (64, 4, 1, 256, 4), (64, 8, 1, 256, 4),
                 (64, 4, 2, 256, 2), (48, 4, 2, 256, 2), (48, 4, 4, 256, 1), (64, 8, 1, 256, 2),
                 (128, 8, 1, 256, 4), (64, 2, 1, 256, 4)]
-    grid = [g if len(g) == 5 else g + (1,) for g in grid]
-    for (L, wd, T, nt, cs) in grid:
+    grid = [g if len(g) >= 5 else g + (1,) for g in grid]
+    grid = [g if len(g) == 7 else g + (max(1, g[0] // 4), int(os.environ.get("ALGAS_PREFETCH", "0"))) for g in grid]
+    for (L, wd, T, nt, cs, off, pf) in grid:
+        os.environ["ALGAS_PREFETCH"] = str(pf)
         for slots in ([32] if not a.quick else [32]):
-            p = algas.default_params(k=w.k, itopk=L, width=wd, offset_beam=max(1, L // 4), ctas_per_query=T,
+            p = algas.default_params(k=w.k, itopk=L, width=wd, offset_beam=off, ctas_per_query=T,
                                      threads_per_cta=nt, slots=slots, n_seeds=32, seed=1, cluster_size=cs)
             try:
                 r = idx.search_dynamic(Qd, p)
@@ -95,7 +115,7 @@ def main():
             st = r["stats"]
             lat = (st["t_end_ns"] - st["t_start_ns"]) / 1e3
             rec = recall(r["ids"], ti, w.k)
-            row = dict(L=L, w=wd, T=T, threads=nt, cs=cs, slots=slots, recall=rec, qps=a.nq / (ms / 1e3),
+            row = dict(L=L, w=wd, T=T, threads=nt, cs=cs, off=off, pf=pf, slots=slots, recall=rec, qps=a.nq / (ms / 1e3),
                        kernel_ms=ms, lat_p50_us=float(np.percentile(lat, 50)),
                        lat_p99_us=float(np.percentile(lat, 99)), iters=float(st["iters"].mean() / T),
                        dist_evals=float(st["dist_evals"].mean()), spills=int((st["spills"] > 0).sum()),

@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--nq", type=int, default=3000)
     ap.add_argument("--itopk", type=int, default=64)
     ap.add_argument("--width", type=int, default=4)
+    ap.add_argument("--offset", type=int, default=-1)
     ap.add_argument("--threads", type=int, default=256)
     ap.add_argument("--ctas", type=int, default=1)
     ap.add_argument("--slots", type=int, default=32)
@@ -38,7 +39,7 @@ def main():
     G = algas.prune(knn, w.degree) if w.prune else knn[:, :w.degree].contiguous()
     del knn
     idx = algas.Index(Xd, G, w.metric)
-    p = algas.default_params(k=w.k, itopk=a.itopk, width=a.width, offset_beam=max(1, a.itopk // 4),
+    p = algas.default_params(k=w.k, itopk=a.itopk, width=a.width, offset_beam=a.offset if a.offset > 0 else max(1, a.itopk // 4),
                              ctas_per_query=a.ctas, threads_per_cta=a.threads, slots=a.slots, seed=1)
     out = []
     for _ in range(a.reps):
@@ -49,7 +50,8 @@ def main():
         st = r["stats"]
         out.append(dict(kernel_ms=r["info"].kernel_ms, parents=float(st["parents"].mean()),
                         dist_evals=float(st["dist_evals"].mean()), iters=float(st["iters"].mean())))
-    print(json.dumps(dict(cfg=a.cfg, nq=a.nq, itopk=a.itopk, width=a.width, threads=a.threads, ctas=a.ctas,
+    print(json.dumps(dict(cfg=a.cfg, nq=a.nq, itopk=a.itopk, width=a.width, offset=p.offset_beam, threads=a.threads,
+                          ctas=a.ctas,
                           slots=a.slots, runs=out)))
 
 

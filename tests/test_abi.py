@@ -103,7 +103,7 @@ def test_tuner_policy_respects_paper_constraints(props, slots):
         assert t.smem_per_block <= t.smem_avail_per_block
         assert t.smem_avail_per_block <= oracle.tuner_smem_per_block(props.smem_per_sm, t.blocks_per_sm,
                                                                      props.smem_reserved_per_block)
-        assert t.threads_per_cta in (32, 64, 128, 256)
+        assert t.threads_per_cta in (32, 64, 128, 256, 512)
         assert 1 <= t.width <= 32 and 1 <= t.offset_beam <= L
 
 

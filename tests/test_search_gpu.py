@@ -122,6 +122,47 @@ def test_knn_float_modulo_ties():
         np.testing.assert_allclose(gd[r], d64[r, gi[r]], rtol=1e-5)
 
 
+@pytest.fixture
+def knn_mode(monkeypatch):
+    def set_mode(m):
+        monkeypatch.setenv("ALGAS_KNN_MODE", m)
+    return set_mode
+
+
+@pytest.mark.parametrize("metric,d", [(algas.L2, 128), (algas.IP, 100), (algas.L2, 960)])
+def test_knn_screened_equals_direct_float(knn_mode, metric, d):
+    """Tensor-core screen + exact rerank + certificate gives the direct
+    path's answer bit for bit (float data, several column chunks)."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 70_000 if d == 128 else 20_000)
+    if d != 128:
+        X = synth.uniform(20_000, d, seed=21)
+    Q = X[:300] if d == 128 else synth.uniform(300, d, seed=22)
+    sb = 0 if d == 128 else -1
+    knn_mode("direct")
+    di, dd = algas.knn(X, Q, 48, metric, self_base=sb)
+    algas.knn_last_stats()
+    knn_mode("screened")
+    si, sd = algas.knn(X, Q, 48, metric, self_base=sb)
+    screened, fallback = algas.knn_last_stats()
+    assert screened == Q.shape[0]
+    np.testing.assert_array_equal(si, di)
+    np.testing.assert_array_equal(_bits(sd), _bits(dd))
+
+
+def test_knn_screened_lattice_matches_oracle(knn_mode):
+    """Integer lattice: the screened path equals O1 bit for bit, including
+    (dist, id) tie order (ties defeat the certificate -> direct fallback)."""
+    X = synth.lattice(5000, 64, seed=23)
+    knn_mode("screened")
+    gi, gd = algas.knn(X, X[:200], 20, algas.L2, self_base=0)
+    screened, fallback = algas.knn_last_stats()
+    assert screened == 200
+    oi, od = oracle.brute_force(X, X[:200], 20, oracle.L2, self_base=0)
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(_bits(gd), _bits(od))
+
+
 def test_knn_k_exceeds_n_padding():
     X = synth.uniform(7, 8, seed=1)
     gi, gd = algas.knn(X, X[:2], 9, algas.L2, self_base=0)
@@ -160,9 +201,11 @@ LATTICE_CASES = [
 
 
 @pytest.mark.parametrize("case", range(len(LATTICE_CASES)))
-@pytest.mark.parametrize("threads", [32, 64, 128, 256])
+@pytest.mark.parametrize("threads", [32, 64, 128, 256, 512, 1024])
 def test_search_lattice_exact_trajectory(case, threads):
     n, d, metric, R, kw = LATTICE_CASES[case]
+    if threads == 1024 and d > 512:
+        pytest.skip("1024-thread CTAs are built for dim <= 512 (register budget)")
     X, Q, G = lattice_case(n, d, metric, R, seed=100 + case)
     p = algas.default_params(threads_per_cta=threads, seed=7, **kw)
     idx = algas.Index(X, G, metric)
@@ -254,6 +297,24 @@ def test_dynamic_queue_equals_batch(slots, T):
     np.testing.assert_array_equal(_bits(d["dists"]), _bits(b["dists"]))
     np.testing.assert_array_equal(d["stats"]["iters"], b["stats"]["iters"])
     assert (d["stats"]["t_end_ns"] >= d["stats"]["t_start_ns"]).all()
+
+
+@pytest.mark.parametrize("threads", [512, 1024])
+@pytest.mark.parametrize("metric,d", [(algas.L2, 128), (algas.IP, 100), (algas.L2, 960)])
+def test_dynamic_queue_wide_ctas_equal_oracle(threads, metric, d):
+    """The persistent kernel with 16/32-warp CTAs (the bench configuration)
+    follows the oracle's trajectory bit for bit on lattice data."""
+    if threads == 1024 and d > 512:
+        pytest.skip("1024-thread CTAs are built for dim <= 512")
+    X, Q, G = lattice_case(2000, d, metric, 32, seed=330 + d)
+    p = algas.default_params(k=10, itopk=56, width=7, offset_beam=14, n_seeds=32, ctas_per_query=2,
+                             threads_per_cta=threads, slots=8, seed=9)
+    idx = algas.Index(X, G, metric)
+    r = idx.search_dynamic(_torch_cuda(Q), p, tag0=3)
+    oi, od, ost = oracle.search(X, G, Q, _oracle_params(p), metric=metric, tag0=3)
+    np.testing.assert_array_equal(r["ids"], oi)
+    np.testing.assert_array_equal(_bits(r["dists"]), _bits(od))
+    np.testing.assert_array_equal(r["stats"]["dist_evals"].astype(np.int64), ost["dist_evals"])
 
 
 @pytest.mark.parametrize("cs", [2, 4, 8])
