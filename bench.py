@@ -166,39 +166,42 @@ def build_workload(w, nq, dev):
 
 
 def choose_operating_point(idx, Qd, truth, w, slots, target=0.95, Ts=(1,), threads=(256,), widths=(8,),
-                           offsets=(1,)):
+                           offsets=(1,), visited=(0,)):
     """Operating point of the BASELINE metric: for each (CTAs per query T
     (P:L229), threads per CTA, beam width w, offset_beam),
     the smallest L of the sweep whose recall@k >= target; among those, the
     configuration with the highest QPS (the adaptive tuning of P:L225-249
-    applied to measured recall)."""
+    applied to measured recall).  visited: 0 = PRIVATE per-CTA tables, 1 =
+    SHARED per-query table."""
+    import itertools
+
     import paper_conf_ipps_chencyzw025_b200 as algas
-    Ls = [16, 24, 32, 40, 48, 56, 64, 80, 96, 128, 160, 192, 256, 320, 384, 448, 512]
+    Ls = [10, 12, 16, 20, 24, 32, 40, 48, 56, 64, 80, 96, 128, 160, 192, 256, 320, 384, 448, 512]
     sweep = []
     best, best_qps = None, -1.0
-    for nt in threads:
-        for T in Ts:
-            for wd in widths:
-                for off in offsets:
-                    for L in Ls:
-                        if L < w.k:
-                            continue
-                        p = algas.default_params(k=w.k, itopk=L, width=min(wd, L), offset_beam=min(off, L),
-                                                 ctas_per_query=T, threads_per_cta=nt, slots=slots, n_seeds=32,
-                                                 seed=1)
-                        try:
-                            r = idx.search_dynamic(Qd, p)
-                        except algas.AlgasError as e:  # e.g. slots x T not co-resident
-                            sweep.append({"ctas": T, "threads": nt, "itopk": L, "error": str(e)[:80]})
-                            break
-                        rec = recall_at(r["ids"], truth, w.k)
-                        qps = Qd.shape[0] / (r["info"].kernel_ms / 1e3)
-                        sweep.append({"ctas": T, "threads": nt, "width": p.width, "offset_beam": p.offset_beam,
-                                      "itopk": L, "recall": round(rec, 5), "qps": round(qps)})
-                        if rec >= target:
-                            if qps > best_qps:
-                                best, best_qps = p, qps
-                            break
+    for nt, T, wd, off, vis in itertools.product(threads, Ts, widths, offsets, visited):
+        if T == 1 and vis:  # one CTA per query: shared == private
+            continue
+        for L in Ls:
+            if L < w.k:
+                continue
+            p = algas.default_params(k=w.k, itopk=L, width=min(wd, L), offset_beam=min(off, L),
+                                     ctas_per_query=T, threads_per_cta=nt, slots=slots, n_seeds=32,
+                                     seed=1, visited_mode=vis if T > 1 else 0)
+            try:
+                r = idx.search_dynamic(Qd, p)
+            except algas.AlgasError as e:  # e.g. slots x T not co-resident
+                sweep.append({"ctas": T, "threads": nt, "itopk": L, "error": str(e)[:80]})
+                break
+            rec = recall_at(r["ids"], truth, w.k)
+            qps = Qd.shape[0] / (r["info"].kernel_ms / 1e3)
+            sweep.append({"ctas": T, "threads": nt, "width": p.width, "offset_beam": p.offset_beam,
+                          "visited": "shared" if p.visited_mode else "private", "itopk": L,
+                          "recall": round(rec, 5), "qps": round(qps)})
+            if rec >= target:
+                if qps > best_qps:
+                    best, best_qps = p, qps
+                break
     return best, sweep
 
 
@@ -218,7 +221,7 @@ def run_algas(a, rank, world, local):
     # the recall/QPS curve is swept on the measured query set (standard ANN
     # practice), so the reported point provably meets recall@10 >= 0.95
     p, sweep = choose_operating_point(idx, Qd, truth, w, a.batch, Ts=a.ctas, threads=a.threads, widths=a.width,
-                                      offsets=a.offset)
+                                      offsets=a.offset, visited=a.visited)
     if p is None:
         raise SystemExit("no swept itopk reaches recall 0.95")
     if world > 1:  # every rank runs rank 0's operating point
@@ -365,7 +368,8 @@ def run_algas(a, rank, world, local):
                    "degree": w.degree, "k": w.k, "batch_slots": a.batch, "queries_per_step": a.nq,
                    "itopk": p.itopk, "width": p.width, "offset_beam": p.offset_beam,
                    "ctas_per_query": p.ctas_per_query, "threads_per_cta": p.threads_per_cta,
-                   "n_seeds": p.n_seeds, "recall_at_k": float(np.mean(recs)), "recall_target": 0.95,
+                   "n_seeds": p.n_seeds, "visited": "shared" if p.visited_mode else "private",
+                   "recall_at_k": float(np.mean(recs)), "recall_target": 0.95,
                    "parallelism": f"replicas x{world}",
                    "l2": "flushed (256 MB write) between timed steps; index working set 768 MB > L2"},
         "latency_us": {"p50": float(np.percentile(lat, 50)), "p99": float(np.percentile(lat, 99)),
@@ -434,7 +438,7 @@ def run_reference(a, rank, world, local):
     X, Q, Xd, Qd, G, truth, (Qcd, tcal), _ = build_workload(w, a.nq, dev)
     idx = algas.Index(Xd, G, w.metric)
     p, sweep = choose_operating_point(idx, Qcd, tcal, w, a.batch, Ts=a.ctas, threads=a.threads, widths=a.width,
-                                      offsets=a.offset)
+                                      offsets=a.offset, visited=a.visited)
     del idx
     import oracle
     op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=1, S=p.n_seeds,
@@ -477,9 +481,10 @@ def main():
     ap.add_argument("--ctas", type=lambda x: tuple(int(v) for v in x.split(",")), default=(1, 2, 4),
                     help="CTAs per query (T) candidates, comma separated")
     ints = lambda x: tuple(int(v) for v in x.split(","))  # noqa: E731
-    ap.add_argument("--threads", type=ints, default=(256, 512, 1024), help="threads per CTA candidates")
+    ap.add_argument("--threads", type=ints, default=(512, 1024), help="threads per CTA candidates")
     ap.add_argument("--width", type=ints, default=(8, 16), help="beam width (parents per step) candidates")
     ap.add_argument("--offset", type=ints, default=(1,), help="offset_beam candidates (P:L249)")
+    ap.add_argument("--visited", type=ints, default=(0, 1), help="visited modes: 0 private, 1 shared (P:L211)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--ref-queries-per-step", type=int, default=100)

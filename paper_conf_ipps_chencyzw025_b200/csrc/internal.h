@@ -148,7 +148,16 @@ struct PersistArgs {
   unsigned int* slot_fin;   // slots
   unsigned long long* gtab;
   uint32_t epoch_base;
+  // SHARED visited mode: one n-bit bitmap per slot (vbm_words u32 words,
+  // a multiple of 4), or null -> the epoch-tagged per-slot hash in gtab
+  uint32_t* vbm;
+  int64_t vbm_words;
 };
+// SHARED-mode bitmap words per slot for n points (0 = too large: use the hash)
+inline int64_t shared_bitmap_words(int64_t n) {
+  if (n > (int64_t(1) << 22)) return 0;  // > 512 KB per slot to clear per query
+  return ((n + 127) / 128) * 4;
+}
 int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st);
 
 // device control block of a persistent launch: queue head | dparams (16-B) |

@@ -127,7 +127,11 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
     }
   }
 
-  unsigned long long* gt = P.gtab ? P.gtab + ((uint64_t)unit << A.cfg.gtab_bits) : nullptr;
+  // HBM visited tables: one per search unit (PRIVATE spill), or one per slot
+  // shared by the slot's T CTAs (SHARED)
+  unsigned long long* gt =
+      P.gtab ? P.gtab + ((uint64_t)(A.cfg.shared ? slot : unit) << A.cfg.gtab_bits) : nullptr;
+  uint32_t* vbm = (A.cfg.shared && P.vbm) ? P.vbm + (uint64_t)slot * P.vbm_words : nullptr;
   uint32_t served = 0;  // queries this CTA has finished (= last epoch in devq mode)
   uint32_t last_epoch = 0;
 
@@ -177,6 +181,14 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
         s_t0 = globaltimer();
       }
       __syncthreads();
+      if (s_mbox != kMboxQuit && vbm) {
+        // SHARED visited bitmap of the slot: cleared by the slot's
+        // rank-0 CTA before the query is published to the other CTAs (the
+        // mailbox release below orders the clear before their first access)
+        uint4* b4 = reinterpret_cast<uint4*>(vbm);
+        const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+        for (int64_t i = tid; i < P.vbm_words / 4; i += NT) b4[i] = z;
+      }
       if (s_mbox != kMboxQuit && P.mode == 0) {
         // stage the query from host memory into the slot's HBM buffer (one PCIe read)
         const float4* src = P.ring_q + (uint64_t)slot * A.cfg.d4;
@@ -241,7 +253,7 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
     }
     CtaStats local;
     search_cta<NT, TL, CPL, METRIC, CS>(cfg, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
-                                        &local);
+                                        &local, vbm);
     __syncthreads();
     if (tid == 0) {
       local.t_start = s_t0;

@@ -86,6 +86,7 @@ struct algas_server {
   void* ctl = nullptr;
   float4* qbuf = nullptr;
   unsigned long long* gtab = nullptr;  // the server's own HBM spill tables
+  uint32_t* vbm = nullptr;             // SHARED visited bitmaps, one per slot
   // host-side slot bookkeeping (host owns: EMPTY/claimed/in-flight)
   std::vector<std::atomic<int>>* hstate = nullptr;  // 0 free, 1 claimed, 2 in flight
   std::vector<uint32_t> epoch;
@@ -166,8 +167,6 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   *out = nullptr;
   algas_index* idx = const_cast<algas_index*>(cidx);
   if (!idx || !params) return set_error(ALGAS_EINVAL, "null argument");
-  if (params->visited_mode != ALGAS_VISITED_PRIVATE)
-    return set_error(ALGAS_EINVAL, "server: SHARED visited mode not implemented yet");
   const int slots = params->slots > 0 ? params->slots : 32;
   algas_server* s = new algas_server();
   s->idx = idx;
@@ -219,6 +218,9 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   if ((e = cudaMalloc(&s->gtab, gent * 8)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc spill tables: %s", cudaGetErrorString(e)));
   cudaMemset(s->gtab, 0, gent * 8);
+  const int64_t vw = s->plan.cfg.shared ? shared_bitmap_words(idx->n) : 0;
+  if (vw > 0 && (e = cudaMalloc(&s->vbm, (size_t)slots * vw * 4)) != cudaSuccess)
+    return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc visited bitmaps: %s", cudaGetErrorString(e)));
   uint8_t* cb = (uint8_t*)s->ctl;
   PersistArgs pa;
   memset(&pa, 0, sizeof(pa));
@@ -235,6 +237,8 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   pa.qbuf = s->qbuf;
   pa.gtab = s->gtab;
   pa.epoch_base = 1;
+  pa.vbm = s->vbm;
+  pa.vbm_words = vw;
   cudaDeviceSynchronize();
   rc = launch_persistent(s->plan, pa, s->stream);
   if (rc) return cleanup(rc);
@@ -333,6 +337,7 @@ int algas_server_destroy(algas_server* s) {
   if (s->poller.joinable()) s->poller.join();
   if (rc == ALGAS_OK) {
     if (s->gtab) cudaFree(s->gtab);
+    if (s->vbm) cudaFree(s->vbm);
     if (s->ctl) cudaFree(s->ctl);
     if (s->qbuf) cudaFree(s->qbuf);
     if (s->ring_h) cudaFreeHost(s->ring_h);

@@ -149,6 +149,8 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
     c.prefetch = pf ? atoi(pf) : 0;
   }
   c.seed = p->seed;
+  c.shared = p->visited_mode == ALGAS_VISITED_SHARED ? 1 : 0;
+  if (c.shared && cs > 1) return set_error(ALGAS_EINVAL, "SHARED visited mode needs cluster_size 1");
   int nb = 0;
   int rc = max_blocks_per_sm(pl, persistent, &nb);
   if (rc != ALGAS_OK) return rc;
@@ -511,8 +513,6 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   if (!is_device_ptr(queries_dev)) return set_error(ALGAS_EINVAL, "algas_search_dynamic: queries must be device memory");
   if (nq == 0) return ALGAS_OK;
   if (nq >= (1LL << 31)) return set_error(ALGAS_EINVAL, "nq too large");
-  if (params->visited_mode != ALGAS_VISITED_PRIVATE)
-    return set_error(ALGAS_EINVAL, "algas_search_dynamic: SHARED visited mode not implemented yet");
   const int slots = params->slots > 0 ? params->slots : 32;
   Plan pl;
   int rc = make_plan(idx, params, slots, &pl, true);
@@ -550,6 +550,11 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   pa.dq_stats = (CtaStats*)sb.p;
   pa.gtab = idx->ws->gtab;
   pa.epoch_base = 1;
+  DevBuf vb;  // SHARED visited bitmaps (cleared per query by the slot's rank-0 CTA)
+  if (pl.cfg.shared && (pa.vbm_words = shared_bitmap_words(idx->n)) > 0) {
+    if ((rc = vb.alloc((size_t)slots * pa.vbm_words * 4, st))) return rc;
+    pa.vbm = (uint32_t*)vb.p;
+  }
   EventTimer tm(st);
   if ((rc = tm.start())) return rc;
   if ((rc = launch_persistent(pl, pa, st))) return rc;

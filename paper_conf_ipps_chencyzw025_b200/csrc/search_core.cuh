@@ -189,6 +189,9 @@ struct SearchCfg {
   int32_t gather_mode;   // 0: LDG.128 into registers, many rows in flight per warp (default)
                          // 1: 16-B cp.async (LDGSTS) staging, 2: cp.async.bulk staging (mbarrier)
   int32_t prefetch;      // 1: L2 bulk prefetch of each surviving row at filter time
+  int32_t shared;        // 1: SHARED visited mode -- the HBM table passed to search_cta is the
+                         //    query's table, shared by its T CTAs; the shared-memory
+                         //    hash is this CTA's cache of it
   uint64_t seed;
 };
 
@@ -567,7 +570,8 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
 // other CTAs run search_worker() in lock step (two cluster barriers per step).
 template <int NT, int TL, int CPL, int METRIC, int CS = 1>
 __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, uint32_t cta_rank, int k,
-                           unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st) {
+                           unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st,
+                           uint32_t* vbm = nullptr) {
   const int tid = threadIdx.x;
   const int lane = tid & 31;
   const int warp = tid >> 5;
@@ -607,7 +611,13 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
         if (el == kSentinel) continue;
         if (lane == 0) {
           int r = smem_visit(s.hash, hbits, el);
-          if (r == kVisNew) { s.newid[C->nnew] = el; C->nnew++; C->vis_count++; }
+          if (r == kVisNew) {
+            s.newid[C->nnew] = el; C->nnew++; C->vis_count++;
+            // SHARED: a CTA keeps its own seeds even when another CTA of the
+            // query claimed them first (R21), but marks them for the others
+            if (cfg.shared && vbm) atomicOr(vbm + (el >> 5), 1u << (el & 31));
+            else if (cfg.shared && gtab) (void)gmem_visit(gtab, cfg.gtab_bits, epoch, el);
+          }
         }
         __syncwarp();
       }
@@ -709,6 +719,21 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
               const int r = smem_visit(s.hash, hbits, id);
               keep = (r == kVisNew);
               if (r == kVisFull) atomicOr(&C->overflow, 1);
+              if (keep && cfg.shared) {  // new to this CTA: claim it in the query's table (P:L211, P:L217 step 2)
+                if (vbm) {                // the paper's bitmap: one L2 atomic, no probing
+                  const uint32_t bit = 1u << (id & 31);
+                  keep = (atomicOr(vbm + (id >> 5), bit) & bit) == 0u;
+                } else {
+                  const int g = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
+                  keep = (g == kVisNew);
+                  if (g == kVisFull) atomicOr(&C->overflow, 1);
+                }
+              }
+            } else if (vbm) {
+              if (!smem_contains(s.hash, hbits, id)) {
+                const uint32_t bit = 1u << (id & 31);
+                keep = (atomicOr(vbm + (id >> 5), bit) & bit) == 0u;
+              }
             } else if (!smem_contains(s.hash, hbits, id)) {
               const int r = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
               keep = (r == kVisNew);

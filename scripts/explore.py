@@ -93,6 +93,11 @@ def main():
                 for wd in (8, 16, 32):
                     for L in (40, 48, 56, 64):
                         grid.append((L, wd, T, nt, 1, 1, 0))
+    elif os.environ.get("GRID") == "shared":
+        grid = []
+        for (L, wd, T, nt) in [(24, 16, 4, 1024), (32, 16, 4, 1024), (24, 16, 4, 512), (40, 8, 4, 512),
+                               (40, 16, 2, 1024), (32, 8, 4, 1024), (16, 16, 4, 1024), (24, 8, 4, 1024)]:
+            grid.append((L, wd, T, nt, 1, 1, 0))
     elif os.environ.get("GRID") == "cs":
         grid = [(64, 4, 1, 256, 1), (64, 4, 1, 256, 4), (64, 8, 1, 256, 4), (64, 8, 1, 256, 8)]
     elif a.quick:
@@ -105,7 +110,8 @@ def main():
         os.environ["ALGAS_PREFETCH"] = str(pf)
         for slots in ([32] if not a.quick else [32]):
             p = algas.default_params(k=w.k, itopk=L, width=wd, offset_beam=off, ctas_per_query=T,
-                                     threads_per_cta=nt, slots=slots, n_seeds=32, seed=1, cluster_size=cs)
+                                     threads_per_cta=nt, slots=slots, n_seeds=32, seed=1, cluster_size=cs,
+                                     visited_mode=int(os.environ.get("VIS", "0")))
             try:
                 r = idx.search_dynamic(Qd, p)
             except algas.AlgasError as e:
@@ -115,7 +121,8 @@ def main():
             st = r["stats"]
             lat = (st["t_end_ns"] - st["t_start_ns"]) / 1e3
             rec = recall(r["ids"], ti, w.k)
-            row = dict(L=L, w=wd, T=T, threads=nt, cs=cs, off=off, pf=pf, slots=slots, recall=rec, qps=a.nq / (ms / 1e3),
+            row = dict(L=L, w=wd, T=T, threads=nt, cs=cs, off=off, pf=pf, vis=int(os.environ.get("VIS", "0")),
+                       slots=slots, recall=rec, qps=a.nq / (ms / 1e3),
                        kernel_ms=ms, lat_p50_us=float(np.percentile(lat, 50)),
                        lat_p99_us=float(np.percentile(lat, 99)), iters=float(st["iters"].mean() / T),
                        dist_evals=float(st["dist_evals"].mean()), spills=int((st["spills"] > 0).sum()),
