@@ -198,7 +198,10 @@ def choose_operating_point(idx, Qd, truth, w, slots, target=0.95, Ts=(1,), threa
             sweep.append({"ctas": T, "threads": nt, "width": p.width, "offset_beam": p.offset_beam,
                           "visited": "shared" if p.visited_mode else "private", "itopk": L,
                           "recall": round(rec, 5), "qps": round(qps)})
-            if rec >= target:
+            # SHARED mode is nondeterministic (which CTA claims a point): its
+            # recall varies run to run by ~1e-3, so it must clear the target
+            # with a margin to stay >= target in the timed steps
+            if rec >= target + (0.003 if p.visited_mode else 0.0):
                 if qps > best_qps:
                     best, best_qps = p, qps
                 break
@@ -287,7 +290,7 @@ def run_algas(a, rank, world, local):
         try:
             tj = json.load(open(tp))
             same = all(tj.get("params", {}).get(f) == getattr(p, f)
-                       for f in ("itopk", "width", "ctas_per_query", "threads_per_cta", "slots"))
+                       for f in ("itopk", "width", "ctas_per_query", "threads_per_cta", "slots", "visited_mode"))
             if same and tj.get("dram_bytes_per_launch_per_query") is not None:
                 traffic = float(tj["dram_bytes_per_launch_per_query"]) * a.nq
         except Exception:
@@ -305,8 +308,9 @@ def run_algas(a, rank, world, local):
                 pending = 0
                 t0 = time.perf_counter()
                 while done < nq:
-                    while pending < nq and srv.submit(Q[pending % Q.shape[0]], tag=pending):
-                        pending += 1
+                    if pending < nq:  # one library crossing per batch of free slots
+                        s0 = pending % Q.shape[0]
+                        pending += srv.submit_many(Q[s0:min(Q.shape[0], s0 + nq - pending)], tag0=pending)
                     tags, ids, ds, st = srv.poll(256)
                     done += len(tags)
                     lats.append(st["latency_ns"])
@@ -324,7 +328,7 @@ def run_algas(a, rank, world, local):
                    "h2d_bytes_per_step": int(a.nq * (w.dim * 4 + 32)),
                    "d2h_bytes_per_step": int(a.nq * (p.ctas_per_query * (w.k * 8 + 32) + 4)),
                    "p50_us": float(np.percentile(le / 1e3, 50)), "p99_us": float(np.percentile(le / 1e3, 99)),
-                   "path": "algas_submit/algas_poll (host-mapped slot ring, persistent kernel, host merge)"}
+                   "path": "algas_submit_many/algas_poll (host-mapped slot ring, persistent kernel, host merge)"}
         finally:
             srv.close()
 
@@ -334,7 +338,7 @@ def run_algas(a, rank, world, local):
         for B in (1, 8, 16, 32):
             pb = algas.default_params(k=p.k, itopk=p.itopk, width=p.width, offset_beam=p.offset_beam,
                                       ctas_per_query=p.ctas_per_query, threads_per_cta=p.threads_per_cta,
-                                      slots=B, n_seeds=p.n_seeds, seed=p.seed)
+                                      slots=B, n_seeds=p.n_seeds, seed=p.seed, visited_mode=p.visited_mode)
             nqb = min(a.nq, 400 * B)
             rb = idx.search_dynamic(Qd[:nqb], pb, stream=stream)
             lb = (rb["stats"]["t_end_ns"] - rb["stats"]["t_start_ns"]) / 1e3

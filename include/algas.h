@@ -206,6 +206,13 @@ int algas_server_create(const algas_index *idx, const algas_params *params, alga
  * k <= server k, itopk <= server itopk, width <= 32 (0 -> server value). */
 int algas_submit(algas_server *s, const float *query, uint64_t tag, int32_t k, int32_t itopk,
                  int32_t width);
+/* Non-blocking batched submit: queries i = 0.. (n x dim fp32, HOST,
+ * row-major) with tags tag0 + i are submitted in order until every slot is
+ * busy; *n_accepted (required) = how many were (0 when the ring is full --
+ * not an error).  Same semantics per query as algas_submit; one library
+ * crossing for many queries (the host side of dynamic batching). */
+int algas_submit_many(algas_server *s, const float *queries, int64_t n, uint64_t tag0, int32_t k,
+                      int32_t itopk, int32_t width, int64_t *n_accepted);
 /* Non-blocking.  Moves up to max_results completed queries into caller
  * HOST buffers: tags[i], ids[i*kmax .. ), dists[i*kmax .. ) where kmax is
  * the server's k (rows padded with SENTINEL / +inf), stats[i] (nullable).

@@ -84,7 +84,7 @@ class Tuning(ctypes.Structure):
 # every symbol include/algas.h declares (checked by tests/test_abi.py)
 EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_index_create",
            "algas_index_destroy", "algas_index_info", "algas_search", "algas_search_ex", "algas_search_dynamic",
-           "algas_server_create", "algas_submit", "algas_poll", "algas_server_inflight", "algas_server_destroy",
+           "algas_server_create", "algas_submit", "algas_submit_many", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
            "algas_build_graph"]
@@ -120,6 +120,7 @@ def lib(build_if_missing: bool = True):
                                            ctypes.POINTER(RunInfo)]
         L.algas_server_create.argtypes = [P, ctypes.POINTER(Params), ctypes.POINTER(P)]
         L.algas_submit.argtypes = [P, P, u64, i32, i32, i32]
+        L.algas_submit_many.argtypes = [P, P, i64, u64, i32, i32, i32, ctypes.POINTER(i64)]
         L.algas_poll.argtypes = [P, P, P, P, P, i32, ctypes.POINTER(i32)]
         L.algas_server_inflight.argtypes = [P, ctypes.POINTER(i64)]
         L.algas_server_destroy.argtypes = [P]
@@ -297,6 +298,14 @@ class Server:
         rc = lib().algas_submit(self._h, qp, tag, k, itopk, width)
         _check(rc, allow=(EAGAIN,))
         return rc == OK
+
+    def submit_many(self, queries: np.ndarray, tag0: int, k: int = 0, itopk: int = 0, width: int = 0) -> int:
+        """Submit rows of a contiguous HOST fp32 array with tags tag0 + i until
+        the ring is full; returns how many were accepted."""
+        n = ctypes.c_int64(0)
+        qp, _a = _ptr(queries)
+        _check(lib().algas_submit_many(self._h, qp, int(queries.shape[0]), tag0, k, itopk, width, ctypes.byref(n)))
+        return n.value
 
     def poll(self, max_results: int = 64):
         tags = np.empty(max_results, np.uint64)

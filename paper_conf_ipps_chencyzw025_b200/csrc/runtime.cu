@@ -281,6 +281,24 @@ int algas_submit(algas_server* s, const float* query, uint64_t tag, int32_t k, i
   return ALGAS_EAGAIN;
 }
 
+int algas_submit_many(algas_server* s, const float* queries, int64_t n, uint64_t tag0, int32_t k, int32_t itopk,
+                      int32_t width, int64_t* n_accepted) {
+  if (!n_accepted) return set_error(ALGAS_EINVAL, "null n_accepted");
+  *n_accepted = 0;
+  if (!s || (!queries && n > 0) || n < 0) return set_error(ALGAS_EINVAL, "null argument");
+  int64_t i = 0;
+  for (; i < n; ++i) {
+    const int rc = algas_submit(s, queries + i * (int64_t)s->dim, tag0 + (uint64_t)i, k, itopk, width);
+    if (rc == ALGAS_EAGAIN) break;
+    if (rc != ALGAS_OK) {
+      *n_accepted = i;
+      return rc;
+    }
+  }
+  *n_accepted = i;
+  return ALGAS_OK;
+}
+
 int algas_poll(algas_server* s, uint64_t* tags, uint32_t* ids, float* dists, algas_query_stats* stats,
                int32_t max_results, int32_t* n_out) {
   if (!s || !n_out) return set_error(ALGAS_EINVAL, "null argument");

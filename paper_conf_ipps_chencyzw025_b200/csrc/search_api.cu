@@ -145,8 +145,8 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   c.stage_rows = sr;
   c.gather_mode = gather_mode;
   {
-    const char* pf = getenv("ALGAS_PREFETCH");  // experiment switch (DESIGN.md §5)
-    c.prefetch = pf ? atoi(pf) : 0;
+    const char* pf = getenv("ALGAS_PREFETCH");  // experiment switch (DESIGN.md §6)
+    c.prefetch = pf ? atoi(pf) : 8;
   }
   c.seed = p->seed;
   c.shared = p->visited_mode == ALGAS_VISITED_SHARED ? 1 : 0;

@@ -188,7 +188,9 @@ struct SearchCfg {
   int32_t stage_rows;    // vectors per shared-memory staging buffer (2 buffers)
   int32_t gather_mode;   // 0: LDG.128 into registers, many rows in flight per warp (default)
                          // 1: 16-B cp.async (LDGSTS) staging, 2: cp.async.bulk staging (mbarrier)
-  int32_t prefetch;      // 1: L2 bulk prefetch of each surviving row at filter time
+  int32_t prefetch;      // bits: 1 L2 prefetch of each surviving row at filter time, 2 of the
+                         // likely next parents' graph rows at select, 4 evict_last graph loads,
+                         // 8 (default) graph rows of keys entering the list, at distance time
   int32_t shared;        // 1: SHARED visited mode -- the HBM table passed to search_cta is the
                          //    query's table, shared by its T CTAs; the shared-memory
                          //    hash is this CTA's cache of it
@@ -547,6 +549,13 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
       if (b < nbw && tl == 0 && j < Mc) key = make_key((METRIC == kL2) ? acc[b] : -acc[b], ids[b]);
       m[b] = b < nbw ? __ballot_sync(0xffffffffu, key < worst) : 0u;
       tot += __popc(m[b]);
+      // a key that enters the list is a likely parent of the next step(s):
+      // pull its graph row into L2 now (prefetch bit 8, on by default;
+      // results unaffected)
+      if ((cfg.prefetch & 8) && key < worst)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)ids[b] << cfg.rp_shift)),
+                     "r"(4u << cfg.rp_shift)
+                     : "memory");
       acc[b] = __uint_as_float((uint32_t)(key >> 32));  // keep the key's high word (id is in ids[b])
     }
     if (tot > 0) {

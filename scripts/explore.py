@@ -98,6 +98,11 @@ def main():
         for (L, wd, T, nt) in [(24, 16, 4, 1024), (32, 16, 4, 1024), (24, 16, 4, 512), (40, 8, 4, 512),
                                (40, 16, 2, 1024), (32, 8, 4, 1024), (16, 16, 4, 1024), (24, 8, 4, 1024)]:
             grid.append((L, wd, T, nt, 1, 1, 0))
+    elif os.environ.get("GRID") == "pf8":
+        grid = []
+        for pf in (0, 8):
+            for (L, wd, T, nt) in [(12, 8, 4, 512), (12, 8, 4, 1024), (16, 16, 4, 1024), (20, 16, 4, 1024)]:
+                grid.append((L, wd, T, nt, 1, 1, pf))
     elif os.environ.get("GRID") == "cs":
         grid = [(64, 4, 1, 256, 1), (64, 4, 1, 256, 4), (64, 8, 1, 256, 4), (64, 8, 1, 256, 8)]
     elif a.quick:

@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--itopk", type=int, default=64)
     ap.add_argument("--width", type=int, default=4)
     ap.add_argument("--offset", type=int, default=-1)
+    ap.add_argument("--visited", default="private", choices=["private", "shared"])
     ap.add_argument("--threads", type=int, default=256)
     ap.add_argument("--ctas", type=int, default=1)
     ap.add_argument("--slots", type=int, default=32)
@@ -40,7 +41,8 @@ def main():
     del knn
     idx = algas.Index(Xd, G, w.metric)
     p = algas.default_params(k=w.k, itopk=a.itopk, width=a.width, offset_beam=a.offset if a.offset > 0 else max(1, a.itopk // 4),
-                             ctas_per_query=a.ctas, threads_per_cta=a.threads, slots=a.slots, seed=1)
+                             ctas_per_query=a.ctas, threads_per_cta=a.threads, slots=a.slots, seed=1,
+                             visited_mode=1 if a.visited == "shared" else 0)
     out = []
     for _ in range(a.reps):
         if a.batch_kernel:

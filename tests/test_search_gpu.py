@@ -501,3 +501,25 @@ def test_shared_visited_server():
     ds = np.stack([got[t][1] for t in range(Q.shape[0])])
     _check_invariants(X, Q, ids, ds, algas.L2, 10)
     assert oracle.recall(ids, ti, 10) > 0.5
+
+
+def test_server_submit_many_equals_batch():
+    """algas_submit_many (batched host submit) reproduces the static batch
+    path bit for bit (tags = query index)."""
+    X, Q, G = lattice_case(2000, 128, algas.L2, 32, seed=410)
+    kw = dict(k=10, itopk=32, width=8, offset_beam=1, n_seeds=16, ctas_per_query=2, threads_per_cta=512, seed=8)
+    idx = algas.Index(X, G)
+    b = idx.search(Q, params=algas.default_params(**kw), tag0=0)
+    got = {}
+    with algas.Server(idx, algas.default_params(slots=5, **kw)) as srv:
+        pending = 0
+        t0 = time.time()
+        while (pending < Q.shape[0] or srv.inflight() > 0) and time.time() - t0 < 60:
+            if pending < Q.shape[0]:
+                pending += srv.submit_many(np.ascontiguousarray(Q[pending:]), tag0=pending)
+            for t, i, dd, st in zip(*srv.poll(64)):
+                got[int(t)] = (i.copy(), dd.copy())
+    assert len(got) == Q.shape[0]
+    for t in range(Q.shape[0]):
+        np.testing.assert_array_equal(got[t][0], b["ids"][t])
+        np.testing.assert_array_equal(_bits(got[t][1]), _bits(b["dists"][t]))
