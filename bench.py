@@ -17,7 +17,7 @@ Multi-GPU (torchrun, one process per GPU): replicas only -- every rank holds
 the full index and serves its own query stream; no data-path collective
 (DESIGN.md §7).  value = all ranks' queries / max-over-ranks time.
 
---impl reference: the CPU oracle (oracle/, O2 reference search, T=1, same
+--impl reference: the CPU oracle (oracle/, O2 reference search, the same
 graph and parameters) timed on the host cores, rank 0 only.
 """
 from __future__ import annotations
@@ -244,7 +244,7 @@ def run_algas(a, rank, world, local):
         dist.barrier()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
     kern_ms, call_ms, merge_ms, lat, evals, parents, recs = [], [], [], [], [], [], []
-    with ClockSampler(local) as clk:
+    with ClockSampler(local, period_s=float(os.environ.get("ALGAS_BENCH_CLOCK_PERIOD", "0.05"))) as clk:
         for i in range(a.steps):
             flush.zero_()                       # L2 flush between timed steps (untimed)
             torch.cuda.synchronize()
@@ -400,11 +400,12 @@ def run_algas(a, rank, world, local):
 
 
 def cpu_baseline(X, G, Q, truth, w, p, budget_s=15.0):
-    """O2 (oracle/) single-threaded on the host, same graph and parameters
-    with T=1, on a bounded sample of the query stream."""
+    """O2 (oracle/) single-threaded on the host, same graph and the same
+    parameters (itopk, width, offset_beam, T CTAs per query run one after
+    another, visited mode), on a bounded sample of the query stream."""
     import oracle
-    op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=1, S=p.n_seeds,
-                            max_iter=4 * p.itopk + 256, seed=p.seed)
+    op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=p.ctas_per_query, S=p.n_seeds,
+                            max_iter=4 * p.itopk + 256, shared_visited=p.visited_mode, seed=p.seed)
     done = 0
     lats = []
     ids_all = []
@@ -419,7 +420,8 @@ def cpu_baseline(X, G, Q, truth, w, p, budget_s=15.0):
     ids_all = np.concatenate(ids_all)
     return {"value": done / el, "unit": "queries/s", "cores": 1, "kind": "oracle",
             "sample": f"first {done} queries of the step's query set, one query at a time, "
-                      f"O2 with T=1 (itopk={p.itopk}, width={p.width}), {el:.1f} s",
+                      f"O2 (itopk={p.itopk}, width={p.width}, T={p.ctas_per_query}, "
+                      f"{'shared' if p.visited_mode else 'private'} visited), {el:.1f} s",
             "p50_us": float(np.percentile(np.array(lats) * 1e6, 50)),
             "p99_us": float(np.percentile(np.array(lats) * 1e6, 99)),
             "recall_at_k": recall_at(ids_all, truth[:done], w.k)}
@@ -445,8 +447,8 @@ def run_reference(a, rank, world, local):
                                       offsets=a.offset, visited=a.visited)
     del idx
     import oracle
-    op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=1, S=p.n_seeds,
-                            max_iter=4 * p.itopk + 256, seed=p.seed)
+    op = oracle.make_params(k=p.k, L=p.itopk, w=p.width, off=p.offset_beam, T=p.ctas_per_query, S=p.n_seeds,
+                            max_iter=4 * p.itopk + 256, shared_visited=p.visited_mode, seed=p.seed)
     per_step = max(1, a.ref_queries_per_step)
     for i in range(a.warmup):
         oracle.search(X, G, Q[:per_step], op, metric=w.metric)
@@ -464,7 +466,8 @@ def run_reference(a, rank, world, local):
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": tot * 1e3 / a.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": w.name, "n": w.n, "dim": w.dim, "degree": w.degree, "k": w.k,
-                       "itopk": p.itopk, "width": p.width, "ctas_per_query": 1, "queries_per_step": per_step},
+                       "itopk": p.itopk, "width": p.width, "ctas_per_query": p.ctas_per_query,
+                       "visited": "shared" if p.visited_mode else "private", "queries_per_step": per_step},
             "cpu_baseline": {"value": value, "unit": "queries/s", "cores": 1, "kind": "oracle",
                              "sample": f"{per_step} queries per step, single-threaded O2"},
             "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},

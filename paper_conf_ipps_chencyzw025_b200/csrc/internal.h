@@ -37,6 +37,10 @@ struct Workspace {
   size_t h_res_bytes = 0;
   void* h_st = nullptr;                // pinned staging of per-CTA counters
   size_t h_st_bytes = 0;
+  // grow-only device scratch of the dynamic-batching path (per-CTA results,
+  // counters, control block, SHARED bitmaps): no allocation per call
+  void* d_scratch[4] = {nullptr, nullptr, nullptr, nullptr};
+  size_t d_scratch_bytes[4] = {0, 0, 0, 0};
 };
 
 }  // namespace algas

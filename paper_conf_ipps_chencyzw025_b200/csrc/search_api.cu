@@ -48,6 +48,24 @@ int ensure_gtab(algas_index* idx, size_t entries) {
   return ALGAS_OK;
 }
 
+// grow-only device scratch buffer `i` of the workspace (caller holds ws->mu;
+// every user synchronizes its stream before releasing the lock)
+static int ensure_scratch(Workspace* ws, int i, size_t bytes, void** out) {
+  bytes = std::max<size_t>(bytes, 256);
+  if (ws->d_scratch_bytes[i] < bytes) {
+    if (ws->d_scratch[i]) {
+      ALGAS_CUDA_TRY(cudaDeviceSynchronize());
+      cudaFree(ws->d_scratch[i]);
+    }
+    ws->d_scratch[i] = nullptr;
+    ws->d_scratch_bytes[i] = 0;
+    ALGAS_CUDA_TRY(cudaMalloc(&ws->d_scratch[i], bytes));
+    ws->d_scratch_bytes[i] = bytes;
+  }
+  *out = ws->d_scratch[i];
+  return ALGAS_OK;
+}
+
 // Reserve `count` consecutive spill-table epochs; clears the tables on wrap.
 static int take_epochs(algas_index* idx, uint64_t count, uint32_t* base, cudaStream_t st) {
   Workspace* ws = idx->ws;
@@ -415,6 +433,8 @@ int algas_index_destroy(algas_index* idx) {
     if (idx->ws->counters) cudaFree(idx->ws->counters);
     if (idx->ws->h_res) cudaFreeHost(idx->ws->h_res);
     if (idx->ws->h_st) cudaFreeHost(idx->ws->h_st);
+    for (void* p : idx->ws->d_scratch)
+      if (p) cudaFree(p);
     delete idx->ws;
   }
   delete idx;
@@ -507,6 +527,12 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
                          uint64_t tag0, uint32_t* out_ids, float* out_dists, algas_query_stats* out_stats,
                          void* stream, algas_run_info* info) {
   const auto t_entry = std::chrono::steady_clock::now();
+  static const bool trace = getenv("ALGAS_TRACE") != nullptr;
+  auto mark = [&](const char* what) {
+    if (trace)
+      fprintf(stderr, "[algas] %-10s %8.3f ms\n", what,
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_entry).count());
+  };
   algas_index* idx = const_cast<algas_index*>(cidx);
   if (!idx || !params || !queries_dev || !out_ids || !out_dists || nq < 0)
     return set_error(ALGAS_EINVAL, "algas_search_dynamic: null argument");
@@ -518,24 +544,29 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   int rc = make_plan(idx, params, slots, &pl, true);
   if (rc) return rc;
   if ((rc = check_coresident(pl, slots))) return rc;
+  mark("plan");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   const int ctas = slots * pl.T * pl.cluster;
   const int64_t items = nq * pl.T;
 
   std::lock_guard<std::mutex> lk(idx->ws->mu);
   if ((rc = ensure_gtab(idx, (size_t)ctas << pl.cfg.gtab_bits))) return rc;
-  // per-CTA tables restart at epoch 1 for this launch: clear the used region
-  ALGAS_CUDA_TRY(cudaMemsetAsync(idx->ws->gtab, 0, ((size_t)ctas << pl.cfg.gtab_bits) * 8, st));
-  idx->ws->epoch = 1;
+  // epoch-tagged spill tables: every query of this call gets an epoch above
+  // all earlier ones (base + queries served by its CTA), so nothing is cleared
+  uint32_t ebase = 1;
+  if ((rc = take_epochs(idx, (uint64_t)nq + 1, &ebase, st))) return rc;
 
-  DevBuf rb, sb, ctl;
-  if ((rc = rb.alloc((size_t)items * pl.k * sizeof(ResultEntry), st))) return rc;
-  if ((rc = sb.alloc((size_t)items * sizeof(CtaStats), st))) return rc;
+  Workspace* ws = idx->ws;
+  void* rbp = nullptr;
+  void* sbp = nullptr;
+  void* ctlp = nullptr;
+  if ((rc = ensure_scratch(ws, 0, (size_t)items * pl.k * sizeof(ResultEntry), &rbp))) return rc;
+  if ((rc = ensure_scratch(ws, 1, (size_t)items * sizeof(CtaStats), &sbp))) return rc;
   // control block: queue head | mbox[slots] | dparams[slots] | dtag[slots] | slot_fin[slots] | qbuf unused
   const size_t ctl_bytes = control_bytes(slots);
-  if ((rc = ctl.alloc(ctl_bytes, st))) return rc;
-  ALGAS_CUDA_TRY(cudaMemsetAsync(ctl.p, 0, ctl_bytes, st));
-  uint8_t* cb = (uint8_t*)ctl.p;
+  if ((rc = ensure_scratch(ws, 2, ctl_bytes, &ctlp))) return rc;
+  ALGAS_CUDA_TRY(cudaMemsetAsync(ctlp, 0, ctl_bytes, st));
+  uint8_t* cb = (uint8_t*)ctlp;
   PersistArgs pa;
   memset(&pa, 0, sizeof(pa));
   pa.mode = 1;
@@ -546,32 +577,37 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   pa.nq = nq;
   pa.tag0 = tag0;
   carve_control(cb, slots, &pa);
-  pa.dq_res = (ResultEntry*)rb.p;
-  pa.dq_stats = (CtaStats*)sb.p;
-  pa.gtab = idx->ws->gtab;
-  pa.epoch_base = 1;
-  DevBuf vb;  // SHARED visited bitmaps (cleared per query by the slot's rank-0 CTA)
+  pa.dq_res = (ResultEntry*)rbp;
+  pa.dq_stats = (CtaStats*)sbp;
+  pa.gtab = ws->gtab;
+  pa.epoch_base = ebase;
+  // SHARED visited bitmaps: cleared per query by the slot's rank-0 CTA
   if (pl.cfg.shared && (pa.vbm_words = shared_bitmap_words(idx->n)) > 0) {
-    if ((rc = vb.alloc((size_t)slots * pa.vbm_words * 4, st))) return rc;
-    pa.vbm = (uint32_t*)vb.p;
+    void* vbp = nullptr;
+    if ((rc = ensure_scratch(ws, 3, (size_t)slots * pa.vbm_words * 4, &vbp))) return rc;
+    pa.vbm = (uint32_t*)vbp;
   }
+  mark("alloc");
   EventTimer tm(st);
   if ((rc = tm.start())) return rc;
   if ((rc = launch_persistent(pl, pa, st))) return rc;
   if ((rc = tm.stop())) return rc;
+  mark("launch");
   const size_t res_bytes = (size_t)items * pl.k * sizeof(ResultEntry), st_bytes = (size_t)items * sizeof(CtaStats);
   if ((rc = ensure_pinned(idx->ws, res_bytes, st_bytes))) return rc;
   ResultEntry* res = (ResultEntry*)idx->ws->h_res;
   CtaStats* cst = (CtaStats*)idx->ws->h_st;
-  ALGAS_CUDA_TRY(cudaMemcpyAsync(res, rb.p, res_bytes, cudaMemcpyDeviceToHost, st));
-  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst, sb.p, st_bytes, cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(res, rbp, res_bytes, cudaMemcpyDeviceToHost, st));
+  ALGAS_CUDA_TRY(cudaMemcpyAsync(cst, sbp, st_bytes, cudaMemcpyDeviceToHost, st));
   ALGAS_CUDA_TRY(cudaStreamSynchronize(st));
   ALGAS_CUDA_TRY(cudaGetLastError());
+  mark("sync");
   if (info) fill_info(info, pl, ctas, tm.ms());
   bool ovf = false;
   const auto t_merge = std::chrono::steady_clock::now();
   if ((rc = finish_outputs(res, cst, nq, pl.T, pl.k, pl.k, out_ids, out_dists, nullptr, nullptr, out_stats, &ovf)))
     return rc;
+  mark("merge");
   if (info) {
     const auto t_end = std::chrono::steady_clock::now();
     info->merge_ms = std::chrono::duration<float, std::milli>(t_end - t_merge).count();
