@@ -485,7 +485,7 @@ def main():
     ap.add_argument("--config", default="C2")
     ap.add_argument("--nq", type=int, default=10000, help="queries per step")
     ap.add_argument("--batch", type=int, default=32, help="query slots in flight (B)")
-    ap.add_argument("--ctas", type=lambda x: tuple(int(v) for v in x.split(",")), default=(1, 2, 4),
+    ap.add_argument("--ctas", type=lambda x: tuple(int(v) for v in x.split(",")), default=(1, 2, 4, 6, 8),
                     help="CTAs per query (T) candidates, comma separated")
     ints = lambda x: tuple(int(v) for v in x.split(","))  # noqa: E731
     ap.add_argument("--threads", type=ints, default=(512, 1024), help="threads per CTA candidates")

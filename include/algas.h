@@ -113,6 +113,13 @@ typedef struct algas_query_stats {
     uint64_t cyc_gather;  /* neighbour-id gather + visited filter (steps 1-2)    */
     uint64_t cyc_dist;    /* vector gathers + distances (step 3)                 */
     uint64_t cyc_sort;    /* sort + merge into the candidate list (step 4)       */
+    /* device globaltimer (persistent/dynamic path): the first / last of the
+     * query's CTAs to enter its search loop (after pickup, query staging,
+     * visited reset and seeding), and the last to leave it */
+    uint64_t t_loop_first_ns;
+    uint64_t t_loop_last_ns;
+    uint64_t t_loop_end_ns;
+    uint64_t t_entry_last_ns;  /* the last CTA to start its search (query staged) */
 } algas_query_stats;
 
 /* Optional per-call timing filled by the search entry points. */

@@ -50,14 +50,18 @@ class QueryStats(ctypes.Structure):
                 ("dist_evals", ctypes.c_uint32), ("cap_hits", ctypes.c_uint32), ("spills", ctypes.c_uint32),
                 ("overflows", ctypes.c_uint32), ("ctas", ctypes.c_uint32), ("t_start_ns", ctypes.c_uint64),
                 ("t_end_ns", ctypes.c_uint64), ("latency_ns", ctypes.c_uint64), ("cyc_select", ctypes.c_uint64),
-                ("cyc_gather", ctypes.c_uint64), ("cyc_dist", ctypes.c_uint64), ("cyc_sort", ctypes.c_uint64)]
+                ("cyc_gather", ctypes.c_uint64), ("cyc_dist", ctypes.c_uint64), ("cyc_sort", ctypes.c_uint64),
+                ("t_loop_first_ns", ctypes.c_uint64), ("t_loop_last_ns", ctypes.c_uint64),
+                ("t_loop_end_ns", ctypes.c_uint64), ("t_entry_last_ns", ctypes.c_uint64)]
 
 
 STATS_DTYPE = np.dtype([("iters", np.uint32), ("max_iters", np.uint32), ("parents", np.uint32),
                         ("dist_evals", np.uint32), ("cap_hits", np.uint32), ("spills", np.uint32),
                         ("overflows", np.uint32), ("ctas", np.uint32), ("t_start_ns", np.uint64),
                         ("t_end_ns", np.uint64), ("latency_ns", np.uint64), ("cyc_select", np.uint64),
-                        ("cyc_gather", np.uint64), ("cyc_dist", np.uint64), ("cyc_sort", np.uint64)])
+                        ("cyc_gather", np.uint64), ("cyc_dist", np.uint64), ("cyc_sort", np.uint64),
+                        ("t_loop_first_ns", np.uint64), ("t_loop_last_ns", np.uint64), ("t_loop_end_ns", np.uint64),
+                        ("t_entry_last_ns", np.uint64)])
 assert STATS_DTYPE.itemsize == ctypes.sizeof(QueryStats)
 
 

@@ -69,6 +69,7 @@ struct Plan {
   int visited_mode;
   int metric;
   int cluster;     // CTAs per search (thread-block cluster), persistent paths
+  int occ;         // resident CTAs per SM the persistent kernel is built for (1 or 2)
 };
 int max_active_clusters(const Plan& pl, int* out);
 int check_coresident(const Plan& pl, int slots);
@@ -152,14 +153,15 @@ struct PersistArgs {
   unsigned int* slot_fin;   // slots
   unsigned long long* gtab;
   uint32_t epoch_base;
-  // SHARED visited mode: one n-bit bitmap per slot (vbm_words u32 words,
-  // a multiple of 4), or null -> the epoch-tagged per-slot hash in gtab
+  // SHARED visited mode: two n-bit bitmaps per slot (vbm_words u32 words
+  // each, a multiple of 4; zero at launch), or null -> the epoch-tagged
+  // per-slot hash in gtab
   uint32_t* vbm;
   int64_t vbm_words;
 };
 // SHARED-mode bitmap words per slot for n points (0 = too large: use the hash)
 inline int64_t shared_bitmap_words(int64_t n) {
-  if (n > (int64_t(1) << 22)) return 0;  // > 512 KB per slot to clear per query
+  if (n > (int64_t(1) << 22)) return 0;  // > 512 KB per slot and query to clear
   return ((n + 127) / 128) * 4;
 }
 int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st);
@@ -178,12 +180,12 @@ int max_blocks_per_sm(const Plan& pl, bool persistent, int* out);
 
 // kernel tables, one per thread count (kernels_nt.cu): the batch or
 // persistent kernel for (metric, chunk config, cluster size), or null
-void* kernel_table_nt32(int metric, int cc, bool persist, int cs);
-void* kernel_table_nt64(int metric, int cc, bool persist, int cs);
-void* kernel_table_nt128(int metric, int cc, bool persist, int cs);
-void* kernel_table_nt256(int metric, int cc, bool persist, int cs);
-void* kernel_table_nt512(int metric, int cc, bool persist, int cs);
-void* kernel_table_nt1024(int metric, int cc, bool persist, int cs);
+void* kernel_table_nt32(int metric, int cc, bool persist, int cs, int occ);
+void* kernel_table_nt64(int metric, int cc, bool persist, int cs, int occ);
+void* kernel_table_nt128(int metric, int cc, bool persist, int cs, int occ);
+void* kernel_table_nt256(int metric, int cc, bool persist, int cs, int occ);
+void* kernel_table_nt512(int metric, int cc, bool persist, int cs, int occ);
+void* kernel_table_nt1024(int metric, int cc, bool persist, int cs, int occ);
 
 // per-query counters from the T per-CTA records
 inline void aggregate_cta_stats(const CtaStats* cs, int T, algas_query_stats* q) {
@@ -204,6 +206,10 @@ inline void aggregate_cta_stats(const CtaStats* cs, int T, algas_query_stats* q)
     q->cyc_sort += cs[c].cyc_sort;
     if (cs[c].t_start < t0) t0 = cs[c].t_start;
     if (cs[c].t_end > t1) t1 = cs[c].t_end;
+    if (c == 0 || cs[c].t_loop0 < q->t_loop_first_ns) q->t_loop_first_ns = cs[c].t_loop0;
+    if (cs[c].t_loop0 > q->t_loop_last_ns) q->t_loop_last_ns = cs[c].t_loop0;
+    if (cs[c].t_loop1 > q->t_loop_end_ns) q->t_loop_end_ns = cs[c].t_loop1;
+    if (cs[c].t_entry > q->t_entry_last_ns) q->t_entry_last_ns = cs[c].t_entry;
   }
   q->t_start_ns = t0 == ~0ull ? 0 : t0;
   q->t_end_ns = t1;

@@ -99,8 +99,10 @@ struct PKArgs {
 
 constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
 
-template <int NT, int TL, int CPL, int METRIC, int CS>
-__global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
+// MINB = resident CTAs per SM the build is for (1, or 2 when a persistent
+// grid of slots x T searches exceeds the SM count: half the registers)
+template <int NT, int TL, int CPL, int METRIC, int CS, int MINB = 1>
+__global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows);
   const Smem s = carve(smem_raw, lay);
@@ -131,7 +133,9 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
   // shared by the slot's T CTAs (SHARED)
   unsigned long long* gt =
       P.gtab ? P.gtab + ((uint64_t)(A.cfg.shared ? slot : unit) << A.cfg.gtab_bits) : nullptr;
-  uint32_t* vbm = (A.cfg.shared && P.vbm) ? P.vbm + (uint64_t)slot * P.vbm_words : nullptr;
+  // SHARED visited bitmaps: two per slot, query number e (served count) of
+  // the slot uses buffer e & 1 (see the clear below)
+  uint32_t* vbm2 = (A.cfg.shared && P.vbm) ? P.vbm + (uint64_t)slot * 2 * P.vbm_words : nullptr;
   uint32_t served = 0;  // queries this CTA has finished (= last epoch in devq mode)
   uint32_t last_epoch = 0;
 
@@ -181,14 +185,6 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
         s_t0 = globaltimer();
       }
       __syncthreads();
-      if (s_mbox != kMboxQuit && vbm) {
-        // SHARED visited bitmap of the slot: cleared by the slot's
-        // rank-0 CTA before the query is published to the other CTAs (the
-        // mailbox release below orders the clear before their first access)
-        uint4* b4 = reinterpret_cast<uint4*>(vbm);
-        const uint4 z = make_uint4(0u, 0u, 0u, 0u);
-        for (int64_t i = tid; i < P.vbm_words / 4; i += NT) b4[i] = z;
-      }
       if (s_mbox != kMboxQuit && P.mode == 0) {
         // stage the query from host memory into the slot's HBM buffer (one PCIe read)
         const float4* src = P.ring_q + (uint64_t)slot * A.cfg.d4;
@@ -234,6 +230,21 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
     const float4* qsrc = (P.mode == 0) ? P.qbuf + (uint64_t)slot * A.cfg.d4
                                        : P.queries + (uint64_t)item * A.cfg.d4;
     for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = (P.mode == 0) ? ld_volatile_f4(qsrc + i) : qsrc[i];
+    uint32_t* vbm = nullptr;
+    if (vbm2) {
+      // SHARED visited bitmap ("each CTA initializes a part of the
+      // visited table"): this query uses buffer served & 1, and
+      // every CTA clears its 1/T share of the OTHER buffer now, for the
+      // slot's next query, off the critical path of this one.  That buffer's last user (the previous query)
+      // is complete in every CTA (pickup waits for all T Finish signals),
+      // and these stores are ordered before the next query's first claim by
+      // this CTA's Finish release -> rank 0's acquire -> mailbox release.
+      vbm = vbm2 + (uint64_t)(served & 1u) * P.vbm_words;
+      uint4* o4 = reinterpret_cast<uint4*>(vbm2 + (uint64_t)((served & 1u) ^ 1u) * P.vbm_words);
+      const int64_t n4 = P.vbm_words / 4, lo = n4 * rank / P.T, hi = n4 * (rank + 1) / P.T;
+      const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+      for (int64_t i = lo + tid; i < hi; i += NT) o4[i] = z;
+    }
     if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
     __syncthreads();
 
@@ -252,8 +263,8 @@ __global__ void __launch_bounds__(NT, 1) persistent_kernel(PKArgs A) {
       stp = P.dq_stats + (uint64_t)item * P.T + rank;
     }
     CtaStats local;
-    search_cta<NT, TL, CPL, METRIC, CS>(cfg, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
-                                        &local, vbm);
+    search_cta<NT, TL, CPL, METRIC, CS, MINB>(cfg, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
+                                              &local, vbm);
     __syncthreads();
     if (tid == 0) {
       local.t_start = s_t0;

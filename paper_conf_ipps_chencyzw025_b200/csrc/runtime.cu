@@ -86,7 +86,7 @@ struct algas_server {
   void* ctl = nullptr;
   float4* qbuf = nullptr;
   unsigned long long* gtab = nullptr;  // the server's own HBM spill tables
-  uint32_t* vbm = nullptr;             // SHARED visited bitmaps, one per slot
+  uint32_t* vbm = nullptr;             // SHARED visited bitmaps, two per slot
   // host-side slot bookkeeping (host owns: EMPTY/claimed/in-flight)
   std::vector<std::atomic<int>>* hstate = nullptr;  // 0 free, 1 claimed, 2 in flight
   std::vector<uint32_t> epoch;
@@ -219,8 +219,9 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc spill tables: %s", cudaGetErrorString(e)));
   cudaMemset(s->gtab, 0, gent * 8);
   const int64_t vw = s->plan.cfg.shared ? shared_bitmap_words(idx->n) : 0;
-  if (vw > 0 && (e = cudaMalloc(&s->vbm, (size_t)slots * vw * 4)) != cudaSuccess)
+  if (vw > 0 && (e = cudaMalloc(&s->vbm, (size_t)slots * 2 * vw * 4)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc visited bitmaps: %s", cudaGetErrorString(e)));
+  if (vw > 0) cudaMemset(s->vbm, 0, (size_t)slots * 2 * vw * 4);
   uint8_t* cb = (uint8_t*)s->ctl;
   PersistArgs pa;
   memset(&pa, 0, sizeof(pa));

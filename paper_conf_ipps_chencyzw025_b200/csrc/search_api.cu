@@ -144,6 +144,9 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   pl.visited_mode = p->visited_mode;
   pl.metric = idx->metric;
   pl.cluster = cs;
+  // a persistent grid of more searches than SMs runs two 256/512-thread CTAs
+  // per SM (the build with half the registers per thread)
+  pl.occ = (persistent && cs == 1 && (nt == 256 || nt == 512) && (int64_t)slots * T > nsm) ? 2 : 1;
   SearchCfg& c = pl.cfg;
   c.data = reinterpret_cast<const float4*>(idx->d_data);
   c.graph = idx->d_graph;
@@ -581,10 +584,11 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   pa.dq_stats = (CtaStats*)sbp;
   pa.gtab = ws->gtab;
   pa.epoch_base = ebase;
-  // SHARED visited bitmaps: cleared per query by the slot's rank-0 CTA
+  // SHARED visited bitmaps: two per slot (zeroed here; each query's CTAs clear the other one)
   if (pl.cfg.shared && (pa.vbm_words = shared_bitmap_words(idx->n)) > 0) {
     void* vbp = nullptr;
-    if ((rc = ensure_scratch(ws, 3, (size_t)slots * pa.vbm_words * 4, &vbp))) return rc;
+    if ((rc = ensure_scratch(ws, 3, (size_t)slots * 2 * pa.vbm_words * 4, &vbp))) return rc;
+    ALGAS_CUDA_TRY(cudaMemsetAsync(vbp, 0, (size_t)slots * 2 * pa.vbm_words * 4, st));
     pa.vbm = (uint32_t*)vbp;
   }
   mark("alloc");

@@ -201,6 +201,8 @@ struct CtaStats {
   uint32_t iters, parents, dist_evals, cap_hit, spilled, overflow;
   unsigned long long t_start, t_end;  // globaltimer (persistent paths)
   unsigned long long cyc_select, cyc_gather, cyc_dist, cyc_sort;  // SM cycles per phase
+  unsigned long long t_loop0, t_loop1;  // globaltimer: search loop entered / left
+  unsigned long long t_entry;           // globaltimer: search_cta entered (query staged)
 };
 
 struct ResultEntry {
@@ -466,12 +468,13 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
 // instruction issue (profiles/dist_wave_microbench*.txt): warps with no row
 // in a pass skip it entirely (warp-uniform test), and the compaction is one
 // ballot per row group instead of a warp scan.
-template <int NT, int TL, int CPL>
+template <int NT, int TL, int CPL, int MINB = 1>
 struct DistRows {
   // rows in flight per team and pass: the wave's rows all in flight at once
-  // within the register budget (<= 64 registers per thread at 1024 threads,
-  // <= 128 at 512)
-  static constexpr int BW = NT >= 1024 ? 4 : 16;
+  // within the register budget (<= 64 registers per thread at 1024 resident
+  // threads per SM -- one 1024-thread CTA or two 512-thread CTAs -- <= 128
+  // at 512)
+  static constexpr int BW = NT * MINB >= 1024 ? 4 : 16;
   static constexpr int B = CPL >= BW ? 1 : BW / CPL;
 };
 template <int NT, int TL, int CPL, int METRIC, int BOVR = 0>
@@ -577,7 +580,7 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
 // Writes min(k, |list|) results to out[0..k) (rest padded) and the CTA's
 // counters to *st.  CS > 1: this CTA is the leader of a cluster whose
 // other CTAs run search_worker() in lock step (two cluster barriers per step).
-template <int NT, int TL, int CPL, int METRIC, int CS = 1>
+template <int NT, int TL, int CPL, int METRIC, int CS = 1, int MINB = 1>
 __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, uint32_t cta_rank, int k,
                            unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st,
                            uint32_t* vbm = nullptr) {
@@ -594,6 +597,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   const int Rp = 1 << cfg.rp_shift;
   const int step_max_new = cfg.w * Rp;
 
+  if (tid == 0 && st) st->t_entry = globaltimer();
   // ---- reset per-query state (16-B stores)
   {
     uint4* h4 = reinterpret_cast<uint4*>(s.hash);
@@ -609,31 +613,33 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   __syncthreads();
 
   // ---- entry points (Alg.1 l.5): S seeds, duplicates dropped.
-  // Lane 0 of warp 0 inserts them in j order so the visited set holds
-  // exactly the deduplicated seed set.
-  if (warp == 0) {
-    for (int j0 = 0; j0 < cfg.S; j0 += 32) {
-      int j = j0 + lane;
-      uint32_t e = (j < cfg.S) ? entry_point(cfg.seed, tag, cta_rank, (uint32_t)j, cfg.n) : kSentinel;
-      for (int l = 0; l < 32; ++l) {
-        uint32_t el = __shfl_sync(0xffffffffu, e, l);
-        if (el == kSentinel) continue;
-        if (lane == 0) {
-          int r = smem_visit(s.hash, hbits, el);
-          if (r == kVisNew) {
-            s.newid[C->nnew] = el; C->nnew++; C->vis_count++;
-            // SHARED: a CTA keeps its own seeds even when another CTA of the
-            // query claimed them first (R21), but marks them for the others
-            if (cfg.shared && vbm) atomicOr(vbm + (el >> 5), 1u << (el & 31));
-            else if (cfg.shared && gtab) (void)gmem_visit(gtab, cfg.gtab_bits, epoch, el);
-          }
-        }
-        __syncwarp();
-      }
+  // One thread per seed, all inserted at once: the shared-memory hash's
+  // test-and-set lets exactly one copy of a repeated id through, so the
+  // visited set and the new-id list hold the deduplicated seed set (its
+  // order in newid is irrelevant: the merge places keys by value).
+  for (int j = tid; j < ((cfg.S + 31) & ~31); j += NT) {
+    bool keep = false;
+    uint32_t e = kSentinel;
+    if (j < cfg.S) {
+      e = entry_point(cfg.seed, tag, cta_rank, (uint32_t)j, cfg.n);
+      keep = smem_visit(s.hash, hbits, e) == kVisNew;
+      // SHARED: a CTA keeps its own seeds even when another CTA of the
+      // query claimed them first (R21), but marks them for the others
+      if (keep && cfg.shared && vbm) atomicOr(vbm + (e >> 5), 1u << (e & 31));
+      else if (keep && cfg.shared && gtab) (void)gmem_visit(gtab, cfg.gtab_bits, epoch, e);
+    }
+    const unsigned m = __ballot_sync(0xffffffffu, keep);
+    if (m) {
+      int wbase = 0;
+      if (lane == 0) wbase = atomicAdd(&C->nnew, __popc(m));
+      wbase = __shfl_sync(0xffffffffu, wbase, 0);
+      if (keep) s.newid[wbase + __popc(m & ((1u << lane) - 1u))] = e;
     }
   }
   __syncthreads();
+  if (tid == 0) C->vis_count = C->nnew;
 
+  if (tid == 0 && st) st->t_loop0 = globaltimer();
   // per-phase SM cycles (thread 0; the paper's calc/sort split, Fig. 3/17)
   long long tp = clock64();
   unsigned long long cyc[4] = {0, 0, 0, 0};  // select, gather+filter, distance, merge
@@ -792,12 +798,13 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
             fence_cluster();
             mbar_remote_arrive(s.bar + 2, c);
           }
-          dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
+          dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
           mbar_wait_cluster(s.bar + 3, (phase >> 3) & 1u);  // all workers' keys delivered
           phase ^= 8u;
           __syncthreads();
         } else {
-          dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, 1, worst, s.newid, s.newk, &C->nkeys);
+          dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, 1, worst, s.newid, s.newk,
+                                                                      &C->nkeys);
           __syncthreads();
         }
       }
@@ -922,6 +929,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
 
   // ================= publish the first k =================
   if (tid == 0) {
+    if (st) st->t_loop1 = globaltimer();
     C->cnt = lcnt;
     C->iters = liters;
   }

@@ -22,12 +22,12 @@ int chunk_config_for(int d4) {
 static void* kernel_for(const Plan& pl, int metric, bool persist) {
   const int cs = persist ? pl.cluster : 1;
   switch (pl.nt) {
-    case 32: return kernel_table_nt32(metric, pl.ccfg, persist, cs);
-    case 64: return kernel_table_nt64(metric, pl.ccfg, persist, cs);
-    case 128: return kernel_table_nt128(metric, pl.ccfg, persist, cs);
-    case 256: return kernel_table_nt256(metric, pl.ccfg, persist, cs);
-    case 512: return kernel_table_nt512(metric, pl.ccfg, persist, cs);
-    case 1024: return kernel_table_nt1024(metric, pl.ccfg, persist, cs);
+    case 32: return kernel_table_nt32(metric, pl.ccfg, persist, cs, persist ? pl.occ : 1);
+    case 64: return kernel_table_nt64(metric, pl.ccfg, persist, cs, persist ? pl.occ : 1);
+    case 128: return kernel_table_nt128(metric, pl.ccfg, persist, cs, persist ? pl.occ : 1);
+    case 256: return kernel_table_nt256(metric, pl.ccfg, persist, cs, persist ? pl.occ : 1);
+    case 512: return kernel_table_nt512(metric, pl.ccfg, persist, cs, persist ? pl.occ : 1);
+    case 1024: return kernel_table_nt1024(metric, pl.ccfg, persist, cs, persist ? pl.occ : 1);
   }
   return nullptr;
 }
