@@ -190,7 +190,9 @@ struct SearchCfg {
                          // 1: 16-B cp.async (LDGSTS) staging, 2: cp.async.bulk staging (mbarrier)
   int32_t prefetch;      // bits: 1 L2 prefetch of each surviving row at filter time, 2 of the
                          // likely next parents' graph rows at select, 4 evict_last graph loads,
-                         // 8 (default) graph rows of keys entering the list, at distance time
+                         // 8 (default) graph rows of keys entering the list, at distance time,
+                         // 16 each row new to the CTA, before the shared claim;
+                         // 64 (experiment switch) disables the fused warp merge+select
   int32_t shared;        // 1: SHARED visited mode -- the HBM table passed to search_cta is the
                          //    query's table, shared by its T CTAs; the shared-memory
                          //    hash is this CTA's cache of it
@@ -211,7 +213,11 @@ struct ResultEntry {
 };
 
 struct Ctrl {
-  int cnt, nnew, nkeys, np, done, diffusing, vis_count, spilled, overflow, cur;
+  int cnt, np, done, diffusing, vis_count, spilled, overflow, cur;
+  // per-step counters, double-buffered by step parity so that the fused
+  // merge+select of warp 0 can reset the next step's while the other warps
+  // still read this step's
+  int nnew[2], nkeys[2];
   uint32_t iters, parents, dist_evals, cap_hit;
   uint32_t phase;  // bit b: parity of staging barrier b (b=2: step-ready, b=3: keys)
   uint64_t worst;  // prefilter key of the current step
@@ -576,6 +582,39 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
   }
 }
 
+// Warp-level bitonic merge ("parallel-friendly bitonic sort", the
+// beam-extend candidate update of BASELINE north_star (2)): the sorted list
+// (cnt <= 32 keys, one per lane) absorbs nk unsorted new keys 32 at a time --
+// bitonic sort of the block in registers, reversed, lane-wise min against
+// the list (the 32 smallest of the union, a bitonic sequence), 5-stage
+// bitonic merge.  Writes the first L (<= 32) keys to dst.  Warp-uniform.
+constexpr int kWarpMergeMax = 64;
+__device__ __forceinline__ void warp_bitonic_merge(const uint64_t* src, int cnt, const uint64_t* newk, int nk,
+                                                   uint64_t* dst, int L, int lane) {
+  uint64_t mine = lane < cnt ? src[lane] : kKeyMax;
+  for (int c0 = 0; c0 < nk; c0 += 32) {
+    uint64_t x = (c0 + lane < nk) ? newk[c0 + lane] : kKeyMax;
+#pragma unroll
+    for (int kk = 2; kk <= 32; kk <<= 1) {
+#pragma unroll
+      for (int j = kk >> 1; j > 0; j >>= 1) {
+        const uint64_t y = __shfl_xor_sync(0xffffffffu, x, j);
+        const bool keep_min = ((lane & j) == 0) == ((lane & kk) == 0);
+        x = keep_min ? (x < y ? x : y) : (x < y ? y : x);
+      }
+    }
+    const uint64_t xr = __shfl_sync(0xffffffffu, x, 31 - lane);
+    uint64_t m = mine < xr ? mine : xr;
+#pragma unroll
+    for (int j = 16; j > 0; j >>= 1) {
+      const uint64_t y = __shfl_xor_sync(0xffffffffu, m, j);
+      m = ((lane & j) == 0) ? (m < y ? m : y) : (m < y ? y : m);
+    }
+    mine = m;
+  }
+  if (lane < L) dst[lane] = mine;
+}
+
 // Preconditions: s.q holds the query (d4 float4, zero tail); init_cta() ran.
 // Writes min(k, |list|) results to out[0..k) (rest padded) and the CTA's
 // counters to *st.  CS > 1: this CTA is the leader of a cluster whose
@@ -605,7 +644,8 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     for (int i = tid; i < (hcap >> 2); i += NT) h4[i] = e;
   }
   if (tid == 0) {
-    C->cnt = 0; C->nnew = 0; C->nkeys = 0; C->np = 0; C->done = 0; C->diffusing = 0;
+    C->cnt = 0; C->nnew[0] = C->nnew[1] = 0; C->nkeys[0] = C->nkeys[1] = 0; C->np = 0; C->done = 0;
+    C->diffusing = 0;
     C->vis_count = 0; C->spilled = 0; C->overflow = 0; C->cur = 0;
     C->iters = 0; C->parents = 0; C->dist_evals = 0; C->cap_hit = 0;
   }
@@ -631,13 +671,13 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     const unsigned m = __ballot_sync(0xffffffffu, keep);
     if (m) {
       int wbase = 0;
-      if (lane == 0) wbase = atomicAdd(&C->nnew, __popc(m));
+      if (lane == 0) wbase = atomicAdd(&C->nnew[0], __popc(m));
       wbase = __shfl_sync(0xffffffffu, wbase, 0);
       if (keep) s.newid[wbase + __popc(m & ((1u << lane) - 1u))] = e;
     }
   }
   __syncthreads();
-  if (tid == 0) C->vis_count = C->nnew;
+  if (tid == 0) C->vis_count = C->nnew[0];
 
   if (tid == 0 && st) st->t_loop0 = globaltimer();
   // per-phase SM cycles (thread 0; the paper's calc/sort split, Fig. 3/17)
@@ -655,69 +695,83 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   int lcnt = 0;            // list length (uniform register copy in every thread)
   uint32_t liters = 0;     // steps taken
   bool first = true;
+  int sp = 0;              // step parity: which nnew/nkeys counters this step uses (0 for clusters)
+  bool pre = false;        // the next step's parents were already selected (fused path)
+  int np_step = 0;         // parents of the current step
+
+  // ---- select (warp 0, P:L217 step 1): the first w unchecked candidates of
+  // the list (one under greedy search), marked checked; resets the step
+  // counters [ri] of the step it selects for
+  auto select_parents = [&](int ri) {
+    const int cnt = lcnt;
+    uint64_t* list = cur ? s.list[1] : s.list[0];
+    // also look past the parents: the next few unchecked candidates are
+    // the likely parents of the next step, whose graph rows are
+    // prefetched into L2 now (prefetch bit 1; results are unaffected)
+    const int pf = (cfg.prefetch & 2) ? (cfg.w < 16 ? cfg.w : 32 - cfg.w) : 0;
+    const int want = cfg.w + pf;
+    int found = 0;
+    for (int base = 0; base < cnt && found < want; base += 32) {
+      int i = base + lane;
+      bool un = (i < cnt) && !(list[i] & 1ull);
+      unsigned m = __ballot_sync(0xffffffffu, un);
+      int rank = found + __popc(m & ((1u << lane) - 1u));
+      if (un && rank < want) s.sel[rank] = i;
+      found += __popc(m);
+    }
+    const int found_all = found < want ? found : want;
+    if (found > cfg.w) found = cfg.w;
+    __syncwarp();
+    int done = 0, np = 0;
+    if (found == 0) {
+      done = 1;
+    } else if ((int)liters >= cfg.max_iter) {
+      done = 1;
+      if (lane == 0) C->cap_hit = 1;
+    } else {
+      int diff = C->diffusing;
+      if (s.sel[0] >= cfg.off) diff = 1;          // P:L249 (sticky, R6)
+      np = diff ? found : 1;
+      if (lane < np) {
+        int pos = s.sel[lane];
+        uint64_t kk = list[pos];
+        list[pos] = kk | 1ull;                    // mark checked (Alg.1 l.7)
+        s.sel[32 + lane] = (int)key_id(kk);
+      } else if (lane < found_all) {
+        const uint32_t nid = key_id(list[s.sel[lane]]);
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)nid << cfg.rp_shift)),
+                     "r"(4u << cfg.rp_shift)
+                     : "memory");
+      }
+      if (lane == 0) C->diffusing = diff;
+    }
+    if (lane == 0) {
+      C->done = done;
+      C->np = np;
+      C->nnew[ri] = 0;
+      C->nkeys[ri] = 0;
+      if (!done) { C->parents += np; }
+      // switch to the HBM spill table before the shared one gets too full
+      if (!C->spilled && gtab != nullptr && C->vis_count + step_max_new > (hcap * 3) / 4) C->spilled = 1;
+    }
+  };
+
   for (;;) {
     // ================= select (warp 0) =================
     if (!first) {
-      if (warp == 0) {
-        const int cnt = lcnt;
-        uint64_t* list = cur ? s.list[1] : s.list[0];
-        // also look past the parents: the next few unchecked candidates are
-        // the likely parents of the next step, whose graph rows are
-        // prefetched into L2 now (prefetch bit 1; results are unaffected)
-        const int pf = (cfg.prefetch & 2) ? (cfg.w < 16 ? cfg.w : 32 - cfg.w) : 0;
-        const int want = cfg.w + pf;
-        int found = 0;
-        for (int base = 0; base < cnt && found < want; base += 32) {
-          int i = base + lane;
-          bool un = (i < cnt) && !(list[i] & 1ull);
-          unsigned m = __ballot_sync(0xffffffffu, un);
-          int rank = found + __popc(m & ((1u << lane) - 1u));
-          if (un && rank < want) s.sel[rank] = i;
-          found += __popc(m);
-        }
-        const int found_all = found < want ? found : want;
-        if (found > cfg.w) found = cfg.w;
-        __syncwarp();
-        int done = 0, np = 0;
-        if (found == 0) {
-          done = 1;
-        } else if ((int)liters >= cfg.max_iter) {
-          done = 1;
-          if (lane == 0) C->cap_hit = 1;
-        } else {
-          int diff = C->diffusing;
-          if (s.sel[0] >= cfg.off) diff = 1;          // P:L249 (sticky, R6)
-          np = diff ? found : 1;
-          if (lane < np) {
-            int pos = s.sel[lane];
-            uint64_t kk = list[pos];
-            list[pos] = kk | 1ull;                    // mark checked (Alg.1 l.7)
-            s.sel[32 + lane] = (int)key_id(kk);
-          } else if (lane < found_all) {
-            const uint32_t nid = key_id(list[s.sel[lane]]);
-            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)nid << cfg.rp_shift)),
-                         "r"(4u << cfg.rp_shift)
-                         : "memory");
-          }
-          if (lane == 0) C->diffusing = diff;
-        }
-        if (lane == 0) {
-          C->done = done;
-          C->np = np;
-          C->nnew = 0;
-          C->nkeys = 0;
-          if (!done) { C->parents += np; }
-          // switch to the HBM spill table before the shared one gets too full
-          if (!C->spilled && gtab != nullptr && C->vis_count + step_max_new > (hcap * 3) / 4) C->spilled = 1;
-        }
+      if (CS == 1) sp ^= 1;
+      if (!pre) {
+        if (warp == 0) select_parents(sp);
+        __syncthreads();
       }
-      __syncthreads();
+      pre = false;
       lap(0);
       if (C->done) break;
 
       // ================= gather + visited filter (P:L217 steps 1-2) =================
       {
         const int np = C->np;
+        np_step = np;
         const int spilled = C->spilled;
         const int total = np << cfg.rp_shift;  // one neighbour id per thread and pass
         for (int base = 0; base < total; base += NT) {
@@ -734,6 +788,18 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
               const int r = smem_visit(s.hash, hbits, id);
               keep = (r == kVisNew);
               if (r == kVisFull) atomicOr(&C->overflow, 1);
+              // bit 16: the row of an id new to this CTA is pulled into L2
+              // now, so its DRAM fetch overlaps the shared claim, the
+              // compaction and the barrier (wasted only if another CTA
+              // claimed it first)
+              if (keep && (cfg.prefetch & 16))
+                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.data + (uint64_t)id * cfg.d4),
+                             "r"((uint32_t)cfg.d4 * 16u)
+                             : "memory");
+              if (keep && (cfg.prefetch & 32)) {  // same with plain per-line L2 prefetches
+                const char* rp = reinterpret_cast<const char*>(cfg.data + (uint64_t)id * cfg.d4);
+                for (int o = 0; o < cfg.d4 * 16; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rp + o));
+              }
               if (keep && cfg.shared) {  // new to this CTA: claim it in the query's table (P:L211, P:L217 step 2)
                 if (vbm) {                // the paper's bitmap: one L2 atomic, no probing
                   const uint32_t bit = 1u << (id & 31);
@@ -763,13 +829,13 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           const unsigned m = __ballot_sync(0xffffffffu, keep);
           if (m) {
             int wbase = 0;
-            if (lane == 0) wbase = atomicAdd(&C->nnew, __popc(m));
+            if (lane == 0) wbase = atomicAdd(&C->nnew[sp], __popc(m));
             wbase = __shfl_sync(0xffffffffu, wbase, 0);
             if (keep) s.newid[wbase + __popc(m & ((1u << lane) - 1u))] = id;
           }
         }
         __syncthreads();
-        if (tid == 0 && !spilled) C->vis_count += C->nnew;
+        if (tid == 0 && !spilled) C->vis_count += C->nnew[sp];
         lap(1);
       }
     }
@@ -777,7 +843,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
 
     // ================= distances (P:L217 step 3) + prefilter =================
     {
-      const int M = C->nnew;
+      const int M = C->nnew[sp];
       const int cnt = lcnt;
       const uint64_t worst = (cnt >= L) ? (cur ? s.list[1] : s.list[0])[L - 1] : kKeyMax;
       if (cfg.gather_mode == 0) {
@@ -798,13 +864,14 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
             fence_cluster();
             mbar_remote_arrive(s.bar + 2, c);
           }
-          dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, CS, worst, s.newid, s.newk, &C->nkeys);
+          dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, CS, worst, s.newid, s.newk,
+                                                                        &C->nkeys[0]);
           mbar_wait_cluster(s.bar + 3, (phase >> 3) & 1u);  // all workers' keys delivered
           phase ^= 8u;
           __syncthreads();
         } else {
           dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, 1, worst, s.newid, s.newk,
-                                                                      &C->nkeys);
+                                                                      &C->nkeys[sp]);
           __syncthreads();
         }
       }
@@ -855,7 +922,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
             const unsigned m = __ballot_sync(0xffffffffu, keep);
             if (m) {
               int wbase = 0;
-              if (lane == 0) wbase = atomicAdd(&C->nkeys, __popc(m));
+              if (lane == 0) wbase = atomicAdd(&C->nkeys[sp], __popc(m));
               wbase = __shfl_sync(0xffffffffu, wbase, 0);
               if (keep) s.newk[wbase + __popc(m & ((1u << lane) - 1u))] = key;
             }
@@ -873,9 +940,30 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     // of new keys below it.  Keys are unique, so positions are unique; the
     // first L positions form the new list (a merge, not a re-sort).
     {
-      const int nk = C->nkeys;
-      const int npv = C->np;  // read before warp 0 may start the next select
+      const int nk = C->nkeys[sp];
       const int cnt = lcnt;
+      if (CS == 1 && L <= 32 && nk <= kWarpMergeMax && !(cfg.prefetch & 64)) {
+        // fused path (short lists): warp 0 merges with a warp-level bitonic
+        // merge and selects the next step's parents right away, so
+        // a step costs one CTA barrier here instead of three
+        if (warp == 0) {
+          if (nk > 0) {
+            warp_bitonic_merge(cur ? s.list[1] : s.list[0], cnt, s.newk, nk, cur ? s.list[0] : s.list[1], L, lane);
+            cur ^= 1;
+            lcnt = (cnt + nk) < L ? cnt + nk : L;
+          }
+          liters += np_step > 0 ? 1 : 0;
+          __syncwarp();
+          select_parents(sp ^ 1);
+          if (lane == 0) { C->cur = cur; C->cnt = lcnt; }
+        }
+        __syncthreads();
+        cur = C->cur;
+        lcnt = C->cnt;
+        pre = true;
+        lap(3);
+        continue;
+      }
       if (nk > 0) {
         const uint64_t* src = cur ? s.list[1] : s.list[0];
         uint64_t* dst = cur ? s.list[0] : s.list[1];
@@ -921,7 +1009,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
         cur ^= 1;
         lcnt = (cnt + nk) < L ? cnt + nk : L;
       }
-      liters += npv > 0 ? 1 : 0;
+      liters += np_step > 0 ? 1 : 0;
       __syncthreads();
       lap(3);
     }
@@ -981,7 +1069,7 @@ __device__ int worker_step(const SearchCfg& cfg, const Smem& s, uint32_t& phase)
   const int M = *((volatile int*)&s.ctrl->w_m);
   const uint64_t worst = *((volatile uint64_t*)&s.ctrl->w_worst);
   Ctrl* LC = leader_ptr(s.ctrl);
-  dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, 1, worst, s.newid, leader_ptr(s.newk), &LC->nkeys);
+  dist_ldg<NT, TL, CPL, METRIC>(cfg, s.q, M, 0, 1, worst, s.newid, leader_ptr(s.newk), &LC->nkeys[0]);
   __syncthreads();
   if (threadIdx.x == 0) {
     fence_cluster();
