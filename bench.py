@@ -300,25 +300,30 @@ def run_algas(a, rank, world, local):
     e2e = None
     lat_e2e = None
     if not a.no_e2e:
-        srv = algas.Server(idx, p)
+        ps = algas.default_params(**{f: getattr(p, f) for f, _ in p._fields_})
+        ps.host_threads = a.host_threads
+        srv = algas.Server(idx, ps)
         try:
             def serve(nq):
+                # the whole stream goes into the server's host FIFO at once;
+                # the poller thread feeds slots as they free up (algas_enqueue)
+                lats, qw = [], []
                 done = 0
-                lats = []
-                pending = 0
                 t0 = time.perf_counter()
+                for s0 in range(0, nq, Q.shape[0]):
+                    m = min(Q.shape[0], nq - s0)
+                    srv.enqueue(Q[:m], tag0=s0)
                 while done < nq:
-                    if pending < nq:  # one library crossing per batch of free slots
-                        s0 = pending % Q.shape[0]
-                        pending += srv.submit_many(Q[s0:min(Q.shape[0], s0 + nq - pending)], tag0=pending)
                     tags, ids, ds, st = srv.poll(256)
                     done += len(tags)
                     lats.append(st["latency_ns"])
-                return time.perf_counter() - t0, np.concatenate(lats) if lats else np.zeros(0)
+                    qw.append(st["queue_ns"])
+                el = time.perf_counter() - t0
+                return el, np.concatenate(lats), np.concatenate(qw)
             serve(min(2000, a.nq))  # warm-up
             if world > 1:
                 dist.barrier()
-            el, le = serve(a.nq * a.e2e_steps)
+            el, le, qw = serve(a.nq * a.e2e_steps)
             if world > 1:
                 t = torch.tensor([el], device=dev)
                 dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -328,7 +333,10 @@ def run_algas(a, rank, world, local):
                    "h2d_bytes_per_step": int(a.nq * (w.dim * 4 + 32)),
                    "d2h_bytes_per_step": int(a.nq * (p.ctas_per_query * (w.k * 8 + 32) + 4)),
                    "p50_us": float(np.percentile(le / 1e3, 50)), "p99_us": float(np.percentile(le / 1e3, 99)),
-                   "path": "algas_submit_many/algas_poll (host-mapped slot ring, persistent kernel, host merge)"}
+                   "latency_definition": "host: query written into its slot -> merged result ready",
+                   "fifo_wait_us_mean": float(np.mean(qw) / 1e3),
+                   "path": "algas_enqueue/algas_poll (host FIFO -> host-mapped slot ring, persistent kernel, "
+                           "host merge by the poller thread)"}
         finally:
             srv.close()
 
@@ -493,6 +501,7 @@ def main():
     ap.add_argument("--offset", type=ints, default=(1,), help="offset_beam candidates (P:L249)")
     ap.add_argument("--visited", type=ints, default=(0, 1), help="visited modes: 0 private, 1 shared (P:L211)")
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--host-threads", type=int, default=0, help="server poller threads (0: library default)")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--ref-queries-per-step", type=int, default=100)
     ap.add_argument("--no-e2e", action="store_true")

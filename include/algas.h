@@ -90,7 +90,10 @@ typedef struct algas_params {
     int32_t cluster_size;    /* persistent paths: CTAs (SMs) per search as a thread-block
                                 cluster sharing the distance gathers through DSMEM;
                                 1 = off, 2/4/8 (needs threads_per_cta = 256); 0 -> 1 */
-    int32_t reserved1;
+    int32_t host_threads;    /* persistent server: host poller threads, each watching
+                                slots q with q % host_threads == its index, merging
+                                and refilling them (Fig. 18); 0 -> 1 (measured best on
+                                the B200 box: more threads contend for the FIFO/queue locks) */
     uint64_t seed;           /* entry-point generator seed (R5)                      */
 } algas_params;
 
@@ -120,6 +123,7 @@ typedef struct algas_query_stats {
     uint64_t t_loop_last_ns;
     uint64_t t_loop_end_ns;
     uint64_t t_entry_last_ns;  /* the last CTA to start its search (query staged) */
+    uint64_t queue_ns;    /* host: algas_enqueue -> into a slot (0 for algas_submit) */
 } algas_query_stats;
 
 /* Optional per-call timing filled by the search entry points. */
@@ -224,6 +228,16 @@ int algas_submit_many(algas_server *s, const float *queries, int64_t n, uint64_t
  * HOST buffers: tags[i], ids[i*kmax .. ), dists[i*kmax .. ) where kmax is
  * the server's k (rows padded with SENTINEL / +inf), stats[i] (nullable).
  * *n_out = number returned. */
+/* Non-blocking, never refuses: queries i = 0.. (n x dim fp32, HOST,
+ * row-major; copied) with tags tag0 + i join a host FIFO; as many as there
+ * are free slots go in now, the rest enter slots in order as the poller
+ * thread recycles them (Done -> None -> Work without a library crossing by
+ * the caller: the host side of dynamic batching).
+ * Results arrive through algas_poll like submitted ones (stats.queue_ns =
+ * FIFO wait, stats.latency_ns = slot in -> merged result).  Queries still in
+ * the FIFO at algas_server_destroy are dropped. */
+int algas_enqueue(algas_server *s, const float *queries, int64_t n, uint64_t tag0, int32_t k, int32_t itopk,
+                  int32_t width);
 int algas_poll(algas_server *s, uint64_t *tags, uint32_t *ids, float *dists,
                algas_query_stats *stats, int32_t max_results, int32_t *n_out);
 /* Number of submitted-but-not-yet-polled queries. */

@@ -42,7 +42,7 @@ class Params(ctypes.Structure):
                 ("threads_per_cta", ctypes.c_int32), ("n_seeds", ctypes.c_int32),
                 ("max_iter", ctypes.c_int32), ("visited_mode", ctypes.c_int32), ("slots", ctypes.c_int32),
                 ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32),
-                ("cluster_size", ctypes.c_int32), ("reserved1", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("cluster_size", ctypes.c_int32), ("host_threads", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class QueryStats(ctypes.Structure):
@@ -52,7 +52,8 @@ class QueryStats(ctypes.Structure):
                 ("t_end_ns", ctypes.c_uint64), ("latency_ns", ctypes.c_uint64), ("cyc_select", ctypes.c_uint64),
                 ("cyc_gather", ctypes.c_uint64), ("cyc_dist", ctypes.c_uint64), ("cyc_sort", ctypes.c_uint64),
                 ("t_loop_first_ns", ctypes.c_uint64), ("t_loop_last_ns", ctypes.c_uint64),
-                ("t_loop_end_ns", ctypes.c_uint64), ("t_entry_last_ns", ctypes.c_uint64)]
+                ("t_loop_end_ns", ctypes.c_uint64), ("t_entry_last_ns", ctypes.c_uint64),
+                ("queue_ns", ctypes.c_uint64)]
 
 
 STATS_DTYPE = np.dtype([("iters", np.uint32), ("max_iters", np.uint32), ("parents", np.uint32),
@@ -61,7 +62,7 @@ STATS_DTYPE = np.dtype([("iters", np.uint32), ("max_iters", np.uint32), ("parent
                         ("t_end_ns", np.uint64), ("latency_ns", np.uint64), ("cyc_select", np.uint64),
                         ("cyc_gather", np.uint64), ("cyc_dist", np.uint64), ("cyc_sort", np.uint64),
                         ("t_loop_first_ns", np.uint64), ("t_loop_last_ns", np.uint64), ("t_loop_end_ns", np.uint64),
-                        ("t_entry_last_ns", np.uint64)])
+                        ("t_entry_last_ns", np.uint64), ("queue_ns", np.uint64)])
 assert STATS_DTYPE.itemsize == ctypes.sizeof(QueryStats)
 
 
@@ -88,7 +89,7 @@ class Tuning(ctypes.Structure):
 # every symbol include/algas.h declares (checked by tests/test_abi.py)
 EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_index_create",
            "algas_index_destroy", "algas_index_info", "algas_search", "algas_search_ex", "algas_search_dynamic",
-           "algas_server_create", "algas_submit", "algas_submit_many", "algas_poll", "algas_server_inflight", "algas_server_destroy",
+           "algas_server_create", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
            "algas_build_graph"]
@@ -125,6 +126,7 @@ def lib(build_if_missing: bool = True):
         L.algas_server_create.argtypes = [P, ctypes.POINTER(Params), ctypes.POINTER(P)]
         L.algas_submit.argtypes = [P, P, u64, i32, i32, i32]
         L.algas_submit_many.argtypes = [P, P, i64, u64, i32, i32, i32, ctypes.POINTER(i64)]
+        L.algas_enqueue.argtypes = [P, P, i64, u64, i32, i32, i32]
         L.algas_poll.argtypes = [P, P, P, P, P, i32, ctypes.POINTER(i32)]
         L.algas_server_inflight.argtypes = [P, ctypes.POINTER(i64)]
         L.algas_server_destroy.argtypes = [P]
@@ -310,6 +312,13 @@ class Server:
         qp, _a = _ptr(queries)
         _check(lib().algas_submit_many(self._h, qp, int(queries.shape[0]), tag0, k, itopk, width, ctypes.byref(n)))
         return n.value
+
+    def enqueue(self, queries: np.ndarray, tag0: int, k: int = 0, itopk: int = 0, width: int = 0) -> None:
+        """Append rows of a contiguous HOST fp32 array (tags tag0 + i) to the
+        server's host FIFO; the poller thread feeds them into slots as they
+        free up (never refuses)."""
+        qp, _a = _ptr(queries)
+        _check(lib().algas_enqueue(self._h, qp, int(queries.shape[0]), tag0, k, itopk, width))
 
     def poll(self, max_results: int = 64):
         tags = np.empty(max_results, np.uint64)

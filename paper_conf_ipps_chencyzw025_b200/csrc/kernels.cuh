@@ -42,6 +42,14 @@ __device__ __forceinline__ unsigned int ld_acquire_gpu32(const unsigned int* p) 
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ int4 ld_volatile_i4(const int4* p) {
+  int4 r;
+  asm volatile("ld.volatile.global.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p)
+               : "memory");
+  return r;
+}
 __device__ __forceinline__ float4 ld_volatile_f4(const float4* p) {
   float4 r;
   asm volatile("ld.volatile.global.v4.f32 {%0,%1,%2,%3}, [%4];"
@@ -154,18 +162,12 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
             if (kind == kSlotQuit) break;
             if (kind == kSlotReady && ep != last_epoch) break;
             __nanosleep(ns);
-            if (ns < 1024) ns <<= 1;
+            if (ns < 256) ns <<= 1;
           }
           if ((st & 0xFFu) == kSlotQuit) {
             mb = kMboxQuit;
           } else {
             const uint32_t ep = st >> 8;
-            // payload: params + query from mapped memory (volatile: never a stale line)
-            const volatile RingSlot* rs = &P.ring[slot];
-            int4 par = make_int4(rs->k, rs->L, rs->w, 0);
-            unsigned long long tag = rs->tag;
-            P.dparams[slot] = par;
-            P.dtag[slot] = tag;
             mb = ((unsigned long long)ep << 32) | (unsigned long long)slot;
           }
         } else {
@@ -176,8 +178,6 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
             mb = kMboxQuit;
           } else {
             const uint32_t ep = served + 1;
-            P.dparams[slot] = make_int4(P.kmax, A.cfg.L, A.cfg.w, 0);
-            P.dtag[slot] = P.tag0 + (uint64_t)item;
             mb = ((unsigned long long)ep << 32) | (unsigned long long)(uint32_t)item;
           }
         }
@@ -186,10 +186,23 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       }
       __syncthreads();
       if (s_mbox != kMboxQuit && P.mode == 0) {
-        // stage the query from host memory into the slot's HBM buffer (one PCIe read)
+        // payload from mapped host memory in ONE PCIe round trip: the query
+        // chunks, {state, k, L, w} and the tag are read by different threads
+        // at once (volatile: never a stale line; ordered after thread 0's
+        // acquire of the state by the barrier), staged into the slot's HBM
+        // buffer for the other CTAs and into this CTA's shared memory
         const float4* src = P.ring_q + (uint64_t)slot * A.cfg.d4;
         float4* dst = P.qbuf + (uint64_t)slot * A.cfg.d4;
-        for (int i = tid; i < A.cfg.d4; i += NT) dst[i] = ld_volatile_f4(src + i);
+        for (int i = tid; i < A.cfg.d4; i += NT) {
+          const float4 v = ld_volatile_f4(src + i);
+          dst[i] = v;
+          s.q[i] = v;
+        }
+        if (tid == NT - 1) {
+          const int4 sp4 = ld_volatile_i4(reinterpret_cast<const int4*>(&P.ring[slot]));
+          P.dparams[slot] = make_int4(sp4.y, sp4.z, sp4.w, 0);
+        }
+        if (tid == NT - 2) P.dtag[slot] = *((const volatile unsigned long long*)&P.ring[slot].tag);
       }
       __syncthreads();
       if (tid == 0) {
@@ -217,19 +230,33 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     }
     const uint32_t epoch = (uint32_t)(mb >> 32);
     const uint32_t item = (uint32_t)mb;
-    if (tid == 0) {
-      const volatile int* vp = reinterpret_cast<const volatile int*>(P.dparams + slot);
-      s_par = make_int4(vp[0], vp[1], vp[2], vp[3]);
-      s_tag = *((volatile unsigned long long*)(P.dtag + slot));
+    int4 par;
+    uint64_t tag;
+    if (P.mode == 0) {
+      // host ring: per-query params published by rank 0 with the mailbox
+      if (tid == 0) {
+        const volatile int* vp = reinterpret_cast<const volatile int*>(P.dparams + slot);
+        s_par = make_int4(vp[0], vp[1], vp[2], vp[3]);
+        s_tag = *((volatile unsigned long long*)(P.dtag + slot));
+      }
+      __syncthreads();
+      par = s_par;
+      tag = s_tag;
+    } else {
+      // device queue: the launch's params; the tag follows from the item
+      par = make_int4(P.kmax, A.cfg.L, A.cfg.w, 0);
+      tag = P.tag0 + (uint64_t)item;
     }
-    __syncthreads();
-    const int4 par = s_par;
-    const uint64_t tag = s_tag;
 
-    // ---------------- stage the query into shared memory
-    const float4* qsrc = (P.mode == 0) ? P.qbuf + (uint64_t)slot * A.cfg.d4
-                                       : P.queries + (uint64_t)item * A.cfg.d4;
-    for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = (P.mode == 0) ? ld_volatile_f4(qsrc + i) : qsrc[i];
+    // ---------------- stage the query into shared memory (rank 0 of a ring
+    // slot already holds it from the PCIe read)
+    if (P.mode == 1) {
+      const float4* qsrc = P.queries + (uint64_t)item * A.cfg.d4;
+      for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = qsrc[i];
+    } else if (rank != 0) {
+      const float4* qsrc = P.qbuf + (uint64_t)slot * A.cfg.d4;
+      for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = ld_volatile_f4(qsrc + i);
+    }
     uint32_t* vbm = nullptr;
     if (vbm2) {
       // SHARED visited bitmap ("each CTA initializes a part of the

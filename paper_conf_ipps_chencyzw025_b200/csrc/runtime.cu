@@ -4,7 +4,7 @@
 //     filtered out;
 //   * adaptive tuning;
 //   * the persistent server: host-mapped slot ring with per-slot state
-//     machine, one poller thread that watches the per-CTA
+//     machine, host poller threads that watch the per-CTA
 //     Finish flags in host memory (local polling), merges and
 //     recycles the slot (Done -> None).
 #include <algorithm>
@@ -94,7 +94,7 @@ struct algas_server {
   std::vector<int> kq;
   std::vector<std::chrono::steady_clock::time_point> t_submit;
   std::atomic<int> next_slot{0};
-  std::thread poller;
+  std::vector<std::thread> pollers;
   std::atomic<bool> stop{false};
   std::atomic<bool> kernel_ok{true};
   std::mutex cq_mu;
@@ -106,16 +106,73 @@ struct algas_server {
   };
   std::deque<Done> cq;
   std::atomic<int64_t> inflight{0};
+  // host FIFO of enqueued queries not yet in a slot (algas_enqueue): the
+  // poller thread moves the head into a slot the moment one is recycled
+  struct Pending {
+    uint64_t tag;
+    int32_t k, L, w;
+    std::chrono::steady_clock::time_point t_enq;
+    std::vector<float> q;
+  };
+  std::mutex pq_mu;
+  std::deque<Pending> pending;
+  std::atomic<int64_t> n_pending{0};
+  std::vector<uint64_t> queue_ns;  // per slot: FIFO wait of its current query
 };
 
-static void poller_main(algas_server* s) {
+namespace {
+// None -> Work of a claimed slot q: payload first, state word last (release)
+void write_slot(algas_server* s, int q, const float* query, uint64_t tag, int32_t k, int32_t itopk, int32_t width) {
+  memcpy(s->ringq_h + (size_t)q * s->dim, query, (size_t)s->dim * 4);
+  RingSlot* rs = &s->ring_h[q];
+  rs->k = k;
+  rs->L = itopk;
+  rs->w = width;
+  rs->tag = tag;
+  s->tags[q] = tag;
+  s->kq[q] = k;
+  const uint32_t ep = (s->epoch[q] + 1) & 0xFFFFFFu;
+  s->epoch[q] = ep == 0 ? 1 : ep;
+  s->t_submit[q] = std::chrono::steady_clock::now();
+  (*s->hstate)[q].store(2, std::memory_order_release);
+  __atomic_store_n(&rs->state, (s->epoch[q] << 8) | kSlotReady, __ATOMIC_RELEASE);
+}
+// claim a free slot (host state 0 -> 1), scanning from `start`; -1 if none
+int claim_slot(algas_server* s, int start) {
+  for (int i = 0; i < s->slots; ++i) {
+    const int q = (start + i) % s->slots;
+    int expect = 0;
+    if ((*s->hstate)[q].compare_exchange_strong(expect, 1, std::memory_order_acq_rel)) return q;
+  }
+  return -1;
+}
+// move FIFO heads into free slots (caller thread or poller)
+void drain_pending(algas_server* s, int start) {
+  if (s->n_pending.load(std::memory_order_acquire) == 0) return;
+  std::lock_guard<std::mutex> lk(s->pq_mu);
+  while (!s->pending.empty()) {
+    const int q = claim_slot(s, start);
+    if (q < 0) break;
+    algas_server::Pending& p = s->pending.front();
+    s->queue_ns[q] = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+                         std::chrono::steady_clock::now() - p.t_enq).count();
+    write_slot(s, q, p.q.data(), p.tag, p.k, p.L, p.w);
+    s->pending.pop_front();
+    s->n_pending.fetch_sub(1, std::memory_order_acq_rel);
+    start = q + 1;
+  }
+}
+}  // namespace
+
+// poller thread `me` of `nth`: watches slots q = me, me + nth, ...
+static void poller_main(algas_server* s, int me, int nth) {
   const int T = s->T;
   std::vector<uint32_t> ids(s->kmax);
   std::vector<float> ds(s->kmax);
   int idle = 0;
   while (!s->stop.load(std::memory_order_acquire)) {
     bool any = false;
-    for (int q = 0; q < s->slots; ++q) {
+    for (int q = me; q < s->slots; q += nth) {
       if ((*s->hstate)[q].load(std::memory_order_acquire) != 2) continue;
       const uint32_t ep = s->epoch[q];
       bool all = true;
@@ -141,13 +198,19 @@ static void poller_main(algas_server* s) {
       d.st.latency_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
                             std::chrono::steady_clock::now() - s->t_submit[q])
                             .count();
+      d.st.queue_ns = s->queue_ns[q];
+      // Done -> None: host owns the slot again, and the next
+      // enqueued query (if any) goes straight into it -- before the result
+      // is handed to the caller's completion queue (whose lock a polling
+      // caller may hold)
+      __atomic_store_n(&s->ring_h[q].state, (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
+      s->queue_ns[q] = 0;
+      (*s->hstate)[q].store(0, std::memory_order_release);
+      drain_pending(s, q);
       {
         std::lock_guard<std::mutex> lk(s->cq_mu);
         s->cq.push_back(std::move(d));
       }
-      // Done -> None: host owns the slot again
-      __atomic_store_n(&s->ring_h[q].state, (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
-      (*s->hstate)[q].store(0, std::memory_order_release);
     }
     if (!any) {
       if (++idle > 64) {
@@ -205,6 +268,7 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   s->tags.assign(slots, 0);
   s->kq.assign(slots, s->kmax);
   s->t_submit.resize(slots);
+  s->queue_ns.assign(slots, 0);
   const size_t ctl_bytes = control_bytes(slots);
   if ((e = cudaMalloc(&s->ctl, ctl_bytes)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc: %s", cudaGetErrorString(e)));
@@ -243,7 +307,8 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   cudaDeviceSynchronize();
   rc = launch_persistent(s->plan, pa, s->stream);
   if (rc) return cleanup(rc);
-  s->poller = std::thread(poller_main, s);
+  const int nth = std::max(1, std::min(params->host_threads > 0 ? params->host_threads : 1, slots));
+  for (int t = 0; t < nth; ++t) s->pollers.emplace_back(poller_main, s, t, nth);
   *out = s;
   return ALGAS_OK;
 }
@@ -258,28 +323,12 @@ int algas_submit(algas_server* s, const float* query, uint64_t tag, int32_t k, i
     return set_error(ALGAS_EINVAL, "submit: k=%d itopk=%d width=%d exceed server limits (%d,%d,%d)", k, itopk, width,
                      s->kmax, s->plan.cfg.L, s->plan.cfg.w);
   const int start = s->next_slot.fetch_add(1, std::memory_order_relaxed);
-  for (int i = 0; i < s->slots; ++i) {
-    const int q = (start + i) % s->slots;
-    int expect = 0;
-    if (!(*s->hstate)[q].compare_exchange_strong(expect, 1, std::memory_order_acq_rel)) continue;
-    // None -> Work: payload first, state word last (release)
-    memcpy(s->ringq_h + (size_t)q * s->dim, query, (size_t)s->dim * 4);
-    RingSlot* rs = &s->ring_h[q];
-    rs->k = k;
-    rs->L = itopk;
-    rs->w = width;
-    rs->tag = tag;
-    s->tags[q] = tag;
-    s->kq[q] = k;
-    const uint32_t ep = (s->epoch[q] + 1) & 0xFFFFFFu;
-    s->epoch[q] = ep == 0 ? 1 : ep;
-    s->t_submit[q] = std::chrono::steady_clock::now();
-    s->inflight.fetch_add(1);
-    (*s->hstate)[q].store(2, std::memory_order_release);
-    __atomic_store_n(&rs->state, (s->epoch[q] << 8) | kSlotReady, __ATOMIC_RELEASE);
-    return ALGAS_OK;
-  }
-  return ALGAS_EAGAIN;
+  const int q = claim_slot(s, start);
+  if (q < 0) return ALGAS_EAGAIN;
+  s->queue_ns[q] = 0;
+  s->inflight.fetch_add(1);
+  write_slot(s, q, query, tag, k, itopk, width);
+  return ALGAS_OK;
 }
 
 int algas_submit_many(algas_server* s, const float* queries, int64_t n, uint64_t tag0, int32_t k, int32_t itopk,
@@ -297,6 +346,37 @@ int algas_submit_many(algas_server* s, const float* queries, int64_t n, uint64_t
     }
   }
   *n_accepted = i;
+  return ALGAS_OK;
+}
+
+int algas_enqueue(algas_server* s, const float* queries, int64_t n, uint64_t tag0, int32_t k, int32_t itopk,
+                  int32_t width) {
+  if (!s || (!queries && n > 0) || n < 0) return set_error(ALGAS_EINVAL, "null argument");
+  if (s->stop.load()) return set_error(ALGAS_ESTATE, "server is shutting down");
+  if (k <= 0) k = s->kmax;
+  if (itopk <= 0) itopk = s->plan.cfg.L;
+  if (width <= 0) width = s->plan.cfg.w;
+  if (k > s->kmax || itopk > s->plan.cfg.L || k > itopk || width > s->plan.cfg.w)
+    return set_error(ALGAS_EINVAL, "enqueue: k=%d itopk=%d width=%d exceed server limits (%d,%d,%d)", k, itopk, width,
+                     s->kmax, s->plan.cfg.L, s->plan.cfg.w);
+  if (n == 0) return ALGAS_OK;
+  const auto now = std::chrono::steady_clock::now();
+  {
+    std::lock_guard<std::mutex> lk(s->pq_mu);
+    for (int64_t i = 0; i < n; ++i) {
+      algas_server::Pending p;
+      p.tag = tag0 + (uint64_t)i;
+      p.k = k;
+      p.L = itopk;
+      p.w = width;
+      p.t_enq = now;
+      p.q.assign(queries + i * (int64_t)s->dim, queries + (i + 1) * (int64_t)s->dim);
+      s->pending.push_back(std::move(p));
+    }
+    s->inflight.fetch_add(n);
+    s->n_pending.fetch_add(n, std::memory_order_acq_rel);
+  }
+  drain_pending(s, s->next_slot.fetch_add(1, std::memory_order_relaxed));
   return ALGAS_OK;
 }
 
@@ -353,7 +433,8 @@ int algas_server_destroy(algas_server* s) {
     }
   }
   s->stop.store(true);
-  if (s->poller.joinable()) s->poller.join();
+  for (auto& th : s->pollers)
+    if (th.joinable()) th.join();
   if (rc == ALGAS_OK) {
     if (s->gtab) cudaFree(s->gtab);
     if (s->vbm) cudaFree(s->vbm);

@@ -1,3 +1,4 @@
 # ad-hoc GPU diagnostics (one gpurun call)
-timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc=$?; tail -3 gpurun_out/pytest_gpu.log
-for PF in 8 72 8 72; do echo "== ALGAS_PREFETCH=$PF"; ALGAS_PREFETCH=$PF timeout 300 python scripts/probe_call.py C2 12,12,1,4,1024,1 10,8,1,6,512,1 32,8,1,2,1024,1 64,8,1,1,512,0 2>&1 | grep -E "^====|^recall|^latency|last in loop ->|^per query"; done > gpurun_out/pf.log 2>&1
+for H in 1 1; do timeout 900 python bench.py --ctas 4 --threads 1024 --width 12 --visited 1 --no-cpu --no-sweep --host-threads $H > gpurun_out/bench_e2e_h$H.json 2> gpurun_out/bench_e2e.err; echo bench rc=$?; python -c "
+import json;l=json.load(open('gpurun_out/bench_e2e_h$H.json'))
+print($H, l['value'], json.dumps(l['e2e']))"; done

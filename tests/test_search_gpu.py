@@ -523,3 +523,34 @@ def test_server_submit_many_equals_batch():
     for t in range(Q.shape[0]):
         np.testing.assert_array_equal(got[t][0], b["ids"][t])
         np.testing.assert_array_equal(_bits(got[t][1]), _bits(b["dists"][t]))
+
+
+@pytest.mark.parametrize("slots,T,shared", [(3, 2, False), (8, 4, True)])
+def test_server_enqueue_fifo_equals_batch(slots, T, shared):
+    """algas_enqueue (host FIFO fed into slots by the poller thread) returns
+    every query exactly once; PRIVATE mode reproduces the static batch path
+    bit for bit, SHARED mode satisfies the invariants."""
+    X, Q, G = lattice_case(2000, 128, algas.L2, 32, seed=420)
+    kw = dict(k=10, itopk=32, width=8, offset_beam=1, n_seeds=16, ctas_per_query=T, threads_per_cta=512, seed=9)
+    idx = algas.Index(X, G)
+    b = idx.search(Q, params=algas.default_params(**kw), tag0=0)
+    got = {}
+    qn = 0
+    with algas.Server(idx, algas.default_params(slots=slots, visited_mode=1 if shared else 0, **kw)) as srv:
+        srv.enqueue(np.ascontiguousarray(Q), tag0=0)
+        t0 = time.time()
+        while len(got) < Q.shape[0] and time.time() - t0 < 60:
+            for t, i, dd, st in zip(*srv.poll(64)):
+                assert int(t) not in got
+                got[int(t)] = (i.copy(), dd.copy())
+                qn += int(st["queue_ns"] > 0)
+        assert srv.inflight() == 0
+    assert len(got) == Q.shape[0]
+    assert qn > 0  # more queries than slots: some waited in the FIFO
+    ids = np.stack([got[t][0] for t in range(Q.shape[0])])
+    ds = np.stack([got[t][1] for t in range(Q.shape[0])])
+    if not shared:
+        np.testing.assert_array_equal(ids, b["ids"])
+        np.testing.assert_array_equal(_bits(ds), _bits(b["dists"]))
+    else:
+        _check_invariants(X, Q, ids, ds, algas.L2, 10)
