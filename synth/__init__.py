@@ -51,8 +51,13 @@ WORKLOADS = {
                    100, 12, 4.0, 0.05, 1.0, 0.0, False, False, 1001, 1002, 0.5),
     "C2": Workload("C2-SIFT1M-shaped-1Mx128-L2", 1_000_000, 128, L2, 64, 10, 10_000, 128, True,
                    1000, 24, 4.0, 0.3, 12.0, 40.0, True, False, 2001, 2002, 0.5),
+    # C3 calibrated on the B200 box (scripts/sweep_cfg.py): with 1000 points
+    # per cluster, well-separated 960-d clusters make the kNN graph split into
+    # per-cluster components (recall ~0.03 from random seeds); overlapping
+    # centres (0.15) and a rank-16 subspace give a connected, GIST-hard graph:
+    # recall@10 0.85 / 0.95 at L = 128 / 256 with one CTA per query
     "C3": Workload("C3-GIST1M-shaped-1Mx960-L2", 1_000_000, 960, L2, 64, 10, 1_000, 128, True,
-                   1000, 32, 4.0, 0.5, 0.08, 0.3, True, False, 3001, 3002, 0.5),
+                   1000, 16, 4.0, 0.3, 0.08, 0.3, True, False, 3001, 3002, 0.15),
     "C4": Workload("C4-GloVe100-shaped-1.2Mx100-IP", 1_200_000, 100, IP, 64, 100, 10_000, 128, True,
                    1000, 24, 4.0, 0.3, 1.0, 0.0, False, True, 4001, 4002, 0.5),
     "C5": Workload("C5-DEEP100M-shaped-100Mx96-L2", 100_000_000, 96, L2, 64, 10, 10_000, 128, True,
