@@ -383,7 +383,8 @@ def run_algas(a, rank, world, local):
                    "n_seeds": p.n_seeds, "visited": "shared" if p.visited_mode else "private",
                    "recall_at_k": float(np.mean(recs)), "recall_target": 0.95,
                    "parallelism": f"replicas x{world}",
-                   "l2": "flushed (256 MB write) between timed steps; index working set 768 MB > L2"},
+                   "l2": f"flushed (256 MB write) between timed steps; index working set "
+                         f"{(w.n * w.dim * 4 + w.n * Rp * 4) / 1e6:.0f} MB > L2"},
         "latency_us": {"p50": float(np.percentile(lat, 50)), "p99": float(np.percentile(lat, 99)),
                        "definition": "device globaltimer, slot pickup -> last CTA published"},
         "clocks": clk.summary(),
