@@ -8,7 +8,10 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libalgas.so")
+# ALGAS_LIB: load / build an alternative library file (A/B builds of the
+# same sources with extra -D flags from ALGAS_BUILD_DEFS, e.g. build/*.so)
+LIB = os.environ.get("ALGAS_LIB") or os.path.join(HERE, "libalgas.so")
+EXTRA_DEFS = os.environ.get("ALGAS_BUILD_DEFS", "").split()
 SOURCES = ["search_kernels.cu", "search_api.cu", "runtime.cu", "knn.cu"]
 # the search kernels, one object per thread count (compiled in parallel)
 THREAD_COUNTS = [32, 64, 128, 256, 512, 1024]
@@ -35,11 +38,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     objs = []
     jobs = []
-    units = [(src, src.replace(".cu", ".o"), []) for src in SOURCES]
-    units += [(KERNEL_TU, f"kernels_nt{nt}.o", [f"-DALGAS_NT={nt}"]) for nt in THREAD_COUNTS]
+    tag = f".{os.getpid()}" if EXTRA_DEFS else ""
+    units = [(src, src.replace(".cu", f"{tag}.o"), []) for src in SOURCES]
+    units += [(KERNEL_TU, f"kernels_nt{nt}{tag}.o", [f"-DALGAS_NT={nt}"]) for nt in THREAD_COUNTS]
     for src, o, defs in units:
         obj = os.path.join(CSRC, o)
-        cmd = [NVCC, *ARCH, *FLAGS, *defs, "-c", os.path.join(CSRC, src), "-o", obj]
+        cmd = [NVCC, *ARCH, *FLAGS, *EXTRA_DEFS, *defs, "-c", os.path.join(CSRC, src), "-o", obj]
         jobs.append((f"{src} {' '.join(defs)}", subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)))
         objs.append(obj)
     logs = []
@@ -49,7 +53,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         logs.append(f"== {src}\n{out}")
         if p.returncode != 0:
             failed = True
-    log_path = os.path.join(HERE, "build.log")
+    log_path = LIB[:-3] + ".build.log" if EXTRA_DEFS else os.path.join(HERE, "build.log")
     with open(log_path, "w") as f:
         f.write("\n".join(logs))
     if failed:

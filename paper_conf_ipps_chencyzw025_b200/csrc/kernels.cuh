@@ -76,7 +76,8 @@ struct BatchArgs {
 template <int NT, int TL, int CPL, int METRIC>
 __global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
-  const SmemLayout lay = smem_layout(a.cfg.dp4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits, a.cfg.stage_rows);
+  const SmemLayout lay = smem_layout(a.cfg.dp4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits, a.cfg.stage_rows,
+                                       gc_bytes(a.cfg.gc_bits, a.cfg.rp_shift));
   const Smem s = carve(smem_raw, lay);
   init_cta<NT>(s, a.cfg);
   __shared__ int s_item;
@@ -112,7 +113,8 @@ constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
 template <int NT, int TL, int CPL, int METRIC, int CS, int MINB = 1>
 __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
-  const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows);
+  const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows,
+                                       gc_bytes(A.cfg.gc_bits, A.cfg.rp_shift));
   const Smem s = carve(smem_raw, lay);
   init_cta<NT>(s, A.cfg, CS);
   if constexpr (CS > 1) cluster_barrier();  // every CTA's mbarriers exist before any remote arrive

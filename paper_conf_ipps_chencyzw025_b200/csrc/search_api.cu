@@ -127,12 +127,27 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   const int gather_mode = gm_env ? atoi(gm_env) : 0;
   if (gather_mode < 0 || gather_mode > 2) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0, 1 or 2");
   if (cs > 1 && gather_mode != 0) return set_error(ALGAS_EINVAL, "cluster_size > 1 needs the register gather path");
+  const char* pf_env = getenv("ALGAS_PREFETCH");  // experiment switch
+  const int prefetch = pf_env ? atoi(pf_env) : 8;
+  // graph-row cache (prefetch bit 128; 64 rows of <= 64 ids, 32 of 128):
+  // reserved first, if the visited hash can still have its minimum size next
+  // to it.  Off by default: measured -4 % at the C2 point (the cp.async issue
+  // in the distance step costs more than the L2 read it saves)
+  int gcbits = (gather_mode == 0 && cs == 1 && (prefetch & 128)) ? (Rp <= 64 ? 6 : 5) : 0;
   int hb = p->hash_bits, sr = gather_mode == 0 ? -1 : p->stage_rows;
-  choose_smem(dp4, L, ncap, S, w, Rp, budget, &hb, &sr);
+  {
+    int hb_min = 6;
+    while ((1LL << hb_min) < 2LL * (S + w * Rp)) ++hb_min;
+    if (gcbits && smem_layout(dp4, L, ncap, hb > 0 ? hb : hb_min, sr < 0 ? 0 : sr, gc_bytes(gcbits, idx->rp_shift))
+                          .total > budget)
+      gcbits = 0;
+  }
+  const int gcb = gc_bytes(gcbits, idx->rp_shift);
+  choose_smem(dp4, L, ncap, S, w, Rp, budget - gcb, &hb, &sr);
   if (hb < 6 || hb > 16) return set_error(ALGAS_EINVAL, "hash_bits %d not in [6,16]", hb);
   if ((1 << hb) < 2 * (S + w * Rp))
     return set_error(ALGAS_EINVAL, "visited hash 2^%d too small for seeds + one step (%d)", hb, S + w * Rp);
-  SmemLayout lay = smem_layout(dp4, L, ncap, hb, sr);
+  SmemLayout lay = smem_layout(dp4, L, ncap, hb, sr, gcb);
   if (lay.total + reserved > optin)
     return set_error(ALGAS_EINVAL, "search needs %d B shared memory per CTA, device allows %d", lay.total, optin);
 
@@ -165,10 +180,8 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   c.ncap = ncap;
   c.stage_rows = sr;
   c.gather_mode = gather_mode;
-  {
-    const char* pf = getenv("ALGAS_PREFETCH");  // experiment switch
-    c.prefetch = pf ? atoi(pf) : 8;
-  }
+  c.prefetch = prefetch;
+  c.gc_bits = gcbits;
   c.seed = p->seed;
   c.shared = p->visited_mode == ALGAS_VISITED_SHARED ? 1 : 0;
   if (c.shared && cs > 1) return set_error(ALGAS_EINVAL, "SHARED visited mode needs cluster_size 1");

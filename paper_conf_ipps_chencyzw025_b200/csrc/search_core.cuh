@@ -158,11 +158,28 @@ __device__ __forceinline__ float4 ldg_f4_stream(const float4* p) {
 // depend on -- the only robust way to keep all loads of a wave in flight
 // (plain loads get interleaved with FMAs by the scheduler, serialising the
 // round trips).  Device memory: served by L2 like .cg.
+#ifndef ALGAS_ROWLOAD
+#define ALGAS_ROWLOAD 0  // A/B builds: 1 = ld.relaxed.gpu, 2 = ld.relaxed.cta, 3 = ld.global.nc (asm volatile)
+#endif
 __device__ __forceinline__ float4 ld_row_f4(const float4* p) {
   float4 r;
+#if ALGAS_ROWLOAD == 1
+  asm volatile("ld.relaxed.gpu.global.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+#elif ALGAS_ROWLOAD == 2
+  asm volatile("ld.relaxed.cta.global.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+#elif ALGAS_ROWLOAD == 3
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+#else
   asm volatile("ld.volatile.global.v4.f32 {%0,%1,%2,%3}, [%4];"
                : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
                : "l"(p));
+#endif
   return r;
 }
 __device__ __forceinline__ float4 lds_f4_ordered(const float4* p) {
@@ -192,7 +209,12 @@ struct SearchCfg {
                          // likely next parents' graph rows at select, 4 evict_last graph loads,
                          // 8 (default) graph rows of keys entering the list, at distance time,
                          // 16 each row new to the CTA, before the shared claim;
-                         // 64 (experiment switch) disables the fused warp merge+select
+                         // 64 (experiment switch) disables the fused warp merge+select;
+                         // 128 enables the shared-memory graph-row cache (gc_bits)
+  int32_t gc_bits;       // log2 entries of the shared-memory graph-row cache (0: off): rows of
+                         //    keys entering the list are copied (cp.async) into it during the
+                         //    distance step, so the next step's parents' neighbour ids are
+                         //    read from shared memory instead of L2
   int32_t shared;        // 1: SHARED visited mode -- the HBM table passed to search_cta is the
                          //    query's table, shared by its T CTAs; the shared-memory
                          //    hash is this CTA's cache of it
@@ -218,6 +240,7 @@ struct Ctrl {
   // merge+select of warp 0 can reset the next step's while the other warps
   // still read this step's
   int nnew[2], nkeys[2];
+  uint32_t gc_stamp;  // step stamp of the graph-row cache (claims one copy per slot and step)
   uint32_t iters, parents, dist_evals, cap_hit;
   uint32_t phase;  // bit b: parity of staging barrier b (b=2: step-ready, b=3: keys)
   uint64_t worst;  // prefilter key of the current step
@@ -234,10 +257,16 @@ enum { kCmdStep = 1, kCmdQuit = 2 };
 constexpr int kMergeParts = 1024;
 
 struct SmemLayout {
-  int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_part, off_hash, off_stage, off_bar, off_ctrl, total;
+  int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_part, off_hash, off_stage, off_bar, off_ctrl,
+      off_gc, total;
 };
+// bytes of a graph-row cache of 2^gc_bits rows of Rp ids + tag + stamp per row
+__host__ __device__ inline int gc_bytes(int gc_bits, int rp_shift) {
+  return gc_bits > 0 ? (1 << gc_bits) * ((4 << rp_shift) + 8) : 0;
+}
 __host__ __device__ inline int align16(int x) { return (x + 15) & ~15; }
-__host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int hash_bits, int stage_rows) {
+__host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int hash_bits, int stage_rows,
+                                                   int gcb = 0) {
   SmemLayout s;
   int o = 0;
   s.off_stage = o; o += 2 * stage_rows * dp4 * 16;  // 128-B aligned at offset 0
@@ -251,6 +280,7 @@ __host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int 
   s.off_hash = o;  o += align16((1 << hash_bits) * 4);
   s.off_bar = o;   o += 32;
   s.off_ctrl = o;  o += align16((int)sizeof(Ctrl));
+  s.off_gc = o;    o += align16(gcb);
   s.total = o;
   return s;
 }
@@ -266,6 +296,7 @@ struct Smem {
   float4* stage;    // 2 x stage_rows x dp4
   uint64_t* bar;    // 2 mbarriers
   Ctrl* ctrl;
+  uint32_t* gcache; // graph-row cache: rows [2^gc_bits][Rp], then tags, then stamps
 };
 __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
   Smem s;
@@ -279,6 +310,7 @@ __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
   s.hash = reinterpret_cast<uint32_t*>(base + l.off_hash);
   s.stage = reinterpret_cast<float4*>(base + l.off_stage);
   s.bar = reinterpret_cast<uint64_t*>(base + l.off_bar);
+  s.gcache = reinterpret_cast<uint32_t*>(base + l.off_gc);
   s.ctrl = reinterpret_cast<Ctrl*>(base + l.off_ctrl);
   return s;
 }
@@ -299,6 +331,11 @@ __device__ __forceinline__ void init_cta(const Smem& s, const SearchCfg& cfg, in
     mbar_init(s.bar + 3, cs > 1 ? cs - 1 : 1);
     mbar_fence_init();
     s.ctrl->phase = 0;
+    s.ctrl->gc_stamp = 0;
+  }
+  if (cfg.gc_bits > 0) {  // rows are immutable: the cache stays valid across queries
+    uint32_t* tags = s.gcache + ((1u << cfg.gc_bits) << cfg.rp_shift);
+    for (int i = threadIdx.x; i < (2 << cfg.gc_bits); i += NT) tags[i] = i < (1 << cfg.gc_bits) ? 0xFFFFFFFFu : 0u;
   }
   __syncthreads();
 }
@@ -485,7 +522,8 @@ struct DistRows {
 };
 template <int NT, int TL, int CPL, int METRIC, int BOVR = 0>
 __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs, int M, int r0, int rstep,
-                                         uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys) {
+                                         uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys,
+                                         uint32_t* gcache = nullptr, uint32_t gc_stamp = 0) {
   const int tid = threadIdx.x, lane = tid & 31;
   constexpr int NTEAMS = NT / TL;
   constexpr int TPW = 32 / TL;  // teams per warp
@@ -561,7 +599,20 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
       // a key that enters the list is a likely parent of the next step(s):
       // pull its graph row into L2 now (prefetch bit 8, on by default;
       // results unaffected)
-      if ((cfg.prefetch & 8) && key < worst)
+      if (gcache != nullptr && key < worst) {
+        // graph-row cache: the row of a key entering the list goes to shared
+        // memory now (16-B cp.async by this lane, waited for before the
+        // step's last barrier), one copy per cache slot and step
+        const uint32_t slot = hash_slot(ids[b], cfg.gc_bits);
+        uint32_t* tags = gcache + ((1u << cfg.gc_bits) << cfg.rp_shift);
+        if (atomicExch(tags + (1u << cfg.gc_bits) + slot, gc_stamp) != gc_stamp) {
+          tags[slot] = ids[b];
+          const uint32_t* src = cfg.graph + ((uint64_t)ids[b] << cfg.rp_shift);
+          uint32_t* dst = gcache + (slot << cfg.rp_shift);
+          for (int c = 0; c < (1 << cfg.rp_shift); c += 4) cp_async16(dst + c, src + c);
+          asm volatile("cp.async.commit_group;" ::: "memory");
+        }
+      } else if ((cfg.prefetch & 8) && key < worst)
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)ids[b] << cfg.rp_shift)),
                      "r"(4u << cfg.rp_shift)
                      : "memory");
@@ -698,6 +749,9 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   int sp = 0;              // step parity: which nnew/nkeys counters this step uses (0 for clusters)
   bool pre = false;        // the next step's parents were already selected (fused path)
   int np_step = 0;         // parents of the current step
+  // graph-row cache (single-CTA searches on the register gather path)
+  uint32_t* const gcache = (CS == 1 && cfg.gc_bits > 0 && cfg.gather_mode == 0) ? s.gcache : nullptr;
+  uint32_t gstamp = C->gc_stamp;  // read after the seeding barrier; advanced per step
 
   // ---- select (warp 0, P:L217 step 1): the first w unchecked candidates of
   // the list (one under greedy search), marked checked; resets the step
@@ -779,8 +833,13 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           uint32_t id = kSentinel;
           if (idx < total) {
             const uint32_t parent = (uint32_t)s.sel[32 + (idx >> cfg.rp_shift)];
-            const uint32_t* gp = cfg.graph + ((uint64_t)parent << cfg.rp_shift) + (idx & (Rp - 1));
-            id = (cfg.prefetch & 4) ? ldg_u32_hint(gp, l2_evict_last_policy()) : __ldg(gp);
+            const uint32_t slot = gcache ? hash_slot(parent, cfg.gc_bits) : 0u;
+            if (gcache && gcache[((1u << cfg.gc_bits) << cfg.rp_shift) + slot] == parent) {
+              id = gcache[(slot << cfg.rp_shift) + (idx & (Rp - 1))];  // cached row (shared memory)
+            } else {
+              const uint32_t* gp = cfg.graph + ((uint64_t)parent << cfg.rp_shift) + (idx & (Rp - 1));
+              id = (cfg.prefetch & 4) ? ldg_u32_hint(gp, l2_evict_last_policy()) : __ldg(gp);
+            }
           }
           bool keep = false;
           if (id != kSentinel) {
@@ -870,8 +929,9 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           phase ^= 8u;
           __syncthreads();
         } else {
+          ++gstamp;
           dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, 1, worst, s.newid, s.newk,
-                                                                      &C->nkeys[sp]);
+                                                                      &C->nkeys[sp], gcache, gstamp);
           __syncthreads();
         }
       }
@@ -957,6 +1017,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           select_parents(sp ^ 1);
           if (lane == 0) { C->cur = cur; C->cnt = lcnt; }
         }
+        if (gcache) asm volatile("cp.async.wait_all;" ::: "memory");  // cached rows landed (in warp 0's shadow)
         __syncthreads();
         cur = C->cur;
         lcnt = C->cnt;
@@ -1010,13 +1071,16 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
         lcnt = (cnt + nk) < L ? cnt + nk : L;
       }
       liters += np_step > 0 ? 1 : 0;
+      if (gcache) asm volatile("cp.async.wait_all;" ::: "memory");
       __syncthreads();
       lap(3);
     }
   }
 
   // ================= publish the first k =================
+  if (gcache) asm volatile("cp.async.wait_all;" ::: "memory");
   if (tid == 0) {
+    C->gc_stamp = gstamp + 1;
     if (st) st->t_loop1 = globaltimer();
     C->cnt = lcnt;
     C->iters = liters;
