@@ -15,7 +15,7 @@ seconds, so these tests check SAMPLED outputs the oracle computes one by one:
     and recall@k (truth from O1) is no lower than O2's recall at identical
     (itopk, width, offset_beam, T, seeds) minus 0.005 (BASELINE north_star)
 
-Inputs are synth's C2 / C4 recipes (SIFT1M- / GloVe-100-shaped).  Truth and
+Inputs are synth's C2 / C4 / C3 recipes (SIFT1M- / GloVe-100- / GIST1M-shaped).  Truth and
 expected values come only from oracle/ (O1, O2), computed here, never from
 the CUDA path.
 """
@@ -95,11 +95,11 @@ def _check_invariants(X, Q, ids, ds, metric):
         assert np.all(np.abs(ds[t] - ref) <= 1e-5 * scale + 1e-30), "distance tolerance"
 
 
-@pytest.mark.parametrize("name", ["C2", "C4"])
+@pytest.mark.parametrize("name", ["C2", "C4", "C3"])
 def test_fullsize_knn_graph_rows_match_oracle(name):
     """Sampled rows of the exact kNN graph (the input of the prune) == O1 with
     self exclusion, modulo equal-distance ties (BASELINE north_star)."""
-    w, X, Q, G, idx, rows, knn_rows, _, _ = workload(name, 500 if name == "C2" else 150)
+    w, X, Q, G, idx, rows, knn_rows, _, _ = workload(name, {"C2": 500, "C4": 150, "C3": 120}[name])
     for r, g in zip(rows, knn_rows):
         oi, od = oracle.brute_force(X, X[r:r + 1], w.knn_degree, w.metric, self_base=int(r))
         oi = oi[0]
@@ -133,6 +133,13 @@ def test_fullsize_C2_search_bench_launch(itopk, width, T, threads, shared):
 @pytest.mark.parametrize("itopk,width,T,threads,shared", [(128, 16, 1, 512, False), (128, 16, 4, 1024, True)])
 def test_fullsize_C4_search_ip_k100(itopk, width, T, threads, shared):
     _search_case("C4", 150, itopk, width, T, threads, shared)
+
+
+@pytest.mark.parametrize("itopk,width,T,threads,shared", [(64, 8, 4, 512, False), (64, 8, 4, 512, True)])
+def test_fullsize_C3_search_960d(itopk, width, T, threads, shared):
+    """GIST1M-shaped 1M x 960 (3.84 GB of vectors, 60 chunk groups per row)
+    at the C3 bench point."""
+    _search_case("C3", 120, itopk, width, T, threads, shared)
 
 
 def _search_case(name, n_sample, itopk, width, T, threads, shared):
