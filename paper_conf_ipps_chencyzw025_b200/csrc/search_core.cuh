@@ -640,30 +640,32 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
 // the list (the 32 smallest of the union, a bitonic sequence), 5-stage
 // bitonic merge.  Writes the first L (<= 32) keys to dst.  Warp-uniform.
 constexpr int kWarpMergeMax = 64;
-__device__ __forceinline__ void warp_bitonic_merge(const uint64_t* src, int cnt, const uint64_t* newk, int nk,
-                                                   uint64_t* dst, int L, int lane) {
-  uint64_t mine = lane < cnt ? src[lane] : kKeyMax;
-  for (int c0 = 0; c0 < nk; c0 += 32) {
-    uint64_t x = (c0 + lane < nk) ? newk[c0 + lane] : kKeyMax;
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a < b ? b : a; }
+// bitonic sort of one key per lane, ascending across the warp
+__device__ __forceinline__ uint64_t warp_bitonic_sort32(uint64_t x, int lane) {
 #pragma unroll
-    for (int kk = 2; kk <= 32; kk <<= 1) {
+  for (int kk = 2; kk <= 32; kk <<= 1) {
 #pragma unroll
-      for (int j = kk >> 1; j > 0; j >>= 1) {
-        const uint64_t y = __shfl_xor_sync(0xffffffffu, x, j);
-        const bool keep_min = ((lane & j) == 0) == ((lane & kk) == 0);
-        x = keep_min ? (x < y ? x : y) : (x < y ? y : x);
-      }
+    for (int j = kk >> 1; j > 0; j >>= 1) {
+      const uint64_t y = __shfl_xor_sync(0xffffffffu, x, j);
+      const bool keep_min = ((lane & j) == 0) == ((lane & kk) == 0);
+      x = keep_min ? umin64(x, y) : umax64(x, y);
     }
-    const uint64_t xr = __shfl_sync(0xffffffffu, x, 31 - lane);
-    uint64_t m = mine < xr ? mine : xr;
-#pragma unroll
-    for (int j = 16; j > 0; j >>= 1) {
-      const uint64_t y = __shfl_xor_sync(0xffffffffu, m, j);
-      m = ((lane & j) == 0) ? (m < y ? m : y) : (m < y ? y : m);
-    }
-    mine = m;
   }
-  if (lane < L) dst[lane] = mine;
+  return x;
+}
+// merge an ascending block (one key per lane) into the ascending list (one
+// key per lane): reverse the block, lane-wise min (the 32 smallest of the
+// union, bitonic), 5-stage bitonic merge -> the first 32 of the union
+__device__ __forceinline__ uint64_t warp_bitonic_merge32(uint64_t list, uint64_t sorted_block, int lane) {
+  uint64_t m = umin64(list, __shfl_sync(0xffffffffu, sorted_block, 31 - lane));
+#pragma unroll
+  for (int j = 16; j > 0; j >>= 1) {
+    const uint64_t y = __shfl_xor_sync(0xffffffffu, m, j);
+    m = ((lane & j) == 0) ? umin64(m, y) : umax64(m, y);
+  }
+  return m;
 }
 
 // Preconditions: s.q holds the query (d4 float4, zero tail); init_cta() ran.
@@ -1002,20 +1004,76 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     {
       const int nk = C->nkeys[sp];
       const int cnt = lcnt;
-      if (CS == 1 && L <= 32 && nk <= kWarpMergeMax && !(cfg.prefetch & 64)) {
-        // fused path (short lists): warp 0 merges with a warp-level bitonic
-        // merge and selects the next step's parents right away, so
-        // a step costs one CTA barrier here instead of three
+      if (CS == 1 && L <= 32 && nk <= kWarpMergeMax && !(cfg.prefetch & (64 | 2))) {
+        // fused path (short lists): warp 0 merges the new keys into the list
+        // with a warp-level bitonic merge -- warp 1 sorts the second
+        // block of 32 new keys meanwhile -- and selects the next step's
+        // parents from the merged list in its registers, so a step costs one
+        // CTA barrier here instead of three
+        uint64_t* sorted2 = reinterpret_cast<uint64_t*>(s.part);
+        if constexpr (NT >= 64) {
+          if (warp == 1 && nk > 32) {
+            const uint64_t x = (32 + lane < nk) ? s.newk[32 + lane] : kKeyMax;
+            sorted2[lane] = warp_bitonic_sort32(x, lane);
+            __threadfence_block();
+            asm volatile("bar.arrive 1, 64;" ::: "memory");
+          }
+        }
         if (warp == 0) {
+          const uint64_t* src = cur ? s.list[1] : s.list[0];
+          uint64_t* dst = cur ? s.list[0] : s.list[1];
+          uint64_t mine = lane < cnt ? src[lane] : kKeyMax;
           if (nk > 0) {
-            warp_bitonic_merge(cur ? s.list[1] : s.list[0], cnt, s.newk, nk, cur ? s.list[0] : s.list[1], L, lane);
+            mine = warp_bitonic_merge32(mine, warp_bitonic_sort32(lane < nk ? s.newk[lane] : kKeyMax, lane), lane);
+            if (nk > 32) {
+              uint64_t x2;
+              if constexpr (NT >= 64) {
+                asm volatile("bar.sync 1, 64;" ::: "memory");
+                x2 = sorted2[lane];
+              } else {
+                x2 = warp_bitonic_sort32(32 + lane < nk ? s.newk[32 + lane] : kKeyMax, lane);
+              }
+              mine = warp_bitonic_merge32(mine, x2, lane);
+            }
             cur ^= 1;
             lcnt = (cnt + nk) < L ? cnt + nk : L;
+          } else {
+            dst = const_cast<uint64_t*>(src);
           }
           liters += np_step > 0 ? 1 : 0;
-          __syncwarp();
-          select_parents(sp ^ 1);
-          if (lane == 0) { C->cur = cur; C->cnt = lcnt; }
+          // ---- select (P:L217 step 1) from the registers: the first w
+          // unchecked keys in list order (one under greedy search), R6/R7
+          const bool un = lane < lcnt && !(mine & 1ull);
+          const unsigned um = __ballot_sync(0xffffffffu, un);
+          const int found = __popc(um);
+          int done = 0, np = 0;
+          if (found == 0) {
+            done = 1;
+          } else if ((int)liters >= cfg.max_iter) {
+            done = 1;
+            if (lane == 0) C->cap_hit = 1;
+          } else {
+            int diff = C->diffusing;
+            if (__ffs(um) - 1 >= cfg.off) diff = 1;     // P:L249 (sticky, R6)
+            np = diff ? (found < cfg.w ? found : cfg.w) : 1;
+            const int rank = __popc(um & ((1u << lane) - 1u));
+            if (un && rank < np) {
+              s.sel[32 + rank] = (int)key_id(mine);
+              mine |= 1ull;                             // mark checked (Alg.1 l.7)
+            }
+            if (lane == 0) C->diffusing = diff;
+          }
+          if (lane < L) dst[lane] = mine;
+          if (lane == 0) {
+            C->done = done;
+            C->np = np;
+            C->nnew[sp ^ 1] = 0;
+            C->nkeys[sp ^ 1] = 0;
+            if (!done) C->parents += np;
+            if (!C->spilled && gtab != nullptr && C->vis_count + step_max_new > (hcap * 3) / 4) C->spilled = 1;
+            C->cur = cur;
+            C->cnt = lcnt;
+          }
         }
         if (gcache) asm volatile("cp.async.wait_all;" ::: "memory");  // cached rows landed (in warp 0's shadow)
         __syncthreads();
