@@ -639,7 +639,7 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
 // bitonic sort of the block in registers, reversed, lane-wise min against
 // the list (the 32 smallest of the union, a bitonic sequence), 5-stage
 // bitonic merge.  Writes the first L (<= 32) keys to dst.  Warp-uniform.
-constexpr int kWarpMergeMax = 64;
+constexpr int kWarpMergeMax = 128;  // new keys: one block per warp of warps 0..3
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a < b ? b : a; }
 // bitonic sort of one key per lane, ascending across the warp
@@ -1006,17 +1006,18 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       const int cnt = lcnt;
       if (CS == 1 && L <= 32 && nk <= kWarpMergeMax && !(cfg.prefetch & (64 | 2))) {
         // fused path (short lists): warp 0 merges the new keys into the list
-        // with a warp-level bitonic merge -- warp 1 sorts the second
-        // block of 32 new keys meanwhile -- and selects the next step's
+        // with a warp-level bitonic merge -- warps 1..3 sort the
+        // further blocks of 32 new keys meanwhile -- and selects the next step's
         // parents from the merged list in its registers, so a step costs one
         // CTA barrier here instead of three
-        uint64_t* sorted2 = reinterpret_cast<uint64_t*>(s.part);
-        if constexpr (NT >= 64) {
-          if (warp == 1 && nk > 32) {
-            const uint64_t x = (32 + lane < nk) ? s.newk[32 + lane] : kKeyMax;
-            sorted2[lane] = warp_bitonic_sort32(x, lane);
+        uint64_t* sorted2 = reinterpret_cast<uint64_t*>(s.part);  // blocks 1..3, sorted
+        const int nblk = (nk + 31) >> 5;
+        if constexpr (NT >= 128) {
+          if (warp >= 1 && warp < nblk) {
+            const uint64_t x = (32 * warp + lane < nk) ? s.newk[32 * warp + lane] : kKeyMax;
+            sorted2[32 * warp + lane] = warp_bitonic_sort32(x, lane);
             __threadfence_block();
-            asm volatile("bar.arrive 1, 64;" ::: "memory");
+            asm volatile("bar.arrive 1, %0;" ::"r"(32 * nblk) : "memory");
           }
         }
         if (warp == 0) {
@@ -1025,15 +1026,17 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           uint64_t mine = lane < cnt ? src[lane] : kKeyMax;
           if (nk > 0) {
             mine = warp_bitonic_merge32(mine, warp_bitonic_sort32(lane < nk ? s.newk[lane] : kKeyMax, lane), lane);
-            if (nk > 32) {
-              uint64_t x2;
-              if constexpr (NT >= 64) {
-                asm volatile("bar.sync 1, 64;" ::: "memory");
-                x2 = sorted2[lane];
-              } else {
-                x2 = warp_bitonic_sort32(32 + lane < nk ? s.newk[32 + lane] : kKeyMax, lane);
+            if (nblk > 1) {
+              if constexpr (NT >= 128) asm volatile("bar.sync 1, %0;" ::"r"(32 * nblk) : "memory");
+              for (int b = 1; b < nblk; ++b) {
+                uint64_t xb;
+                if constexpr (NT >= 128) {
+                  xb = sorted2[32 * b + lane];
+                } else {
+                  xb = warp_bitonic_sort32(32 * b + lane < nk ? s.newk[32 * b + lane] : kKeyMax, lane);
+                }
+                mine = warp_bitonic_merge32(mine, xb, lane);
               }
-              mine = warp_bitonic_merge32(mine, x2, lane);
             }
             cur ^= 1;
             lcnt = (cnt + nk) < L ? cnt + nk : L;
