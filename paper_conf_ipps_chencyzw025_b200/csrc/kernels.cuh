@@ -148,6 +148,10 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
   uint32_t* vbm2 = (A.cfg.shared && P.vbm) ? P.vbm + (uint64_t)slot * 2 * P.vbm_words : nullptr;
   uint32_t served = 0;  // queries this CTA has finished (= last epoch in devq mode)
   uint32_t last_epoch = 0;
+  // host ring: the slot's two ring entries (sub-slots) alternate, 1 first
+  // (runtime.cu); the epoch last seen in each tells a stale READY apart
+  int sub = 1;
+  uint32_t last_ep_sub[2] = {0u, 0u};
 
   for (;;) {
     // ---------------- acquire work (rank 0) and publish it to the slot's CTAs
@@ -159,10 +163,10 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
           uint32_t st;
           unsigned ns = 64;
           for (;;) {
-            st = ld_acquire_sys(&P.ring[slot].state);
+            st = ld_acquire_sys(&P.ring[2 * slot + sub].state);
             uint32_t kind = st & 0xFFu, ep = st >> 8;
             if (kind == kSlotQuit) break;
-            if (kind == kSlotReady && ep != last_epoch) break;
+            if (kind == kSlotReady && ep != last_ep_sub[sub]) break;
             __nanosleep(ns);
             if (ns < 256) ns <<= 1;
           }
@@ -193,7 +197,7 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         // at once (volatile: never a stale line; ordered after thread 0's
         // acquire of the state by the barrier), staged into the slot's HBM
         // buffer for the other CTAs and into this CTA's shared memory
-        const float4* src = P.ring_q + (uint64_t)slot * A.cfg.d4;
+        const float4* src = P.ring_q + (uint64_t)(2 * slot + sub) * A.cfg.d4;
         float4* dst = P.qbuf + (uint64_t)slot * A.cfg.d4;
         for (int i = tid; i < A.cfg.d4; i += NT) {
           const float4 v = ld_volatile_f4(src + i);
@@ -201,10 +205,10 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
           s.q[i] = v;
         }
         if (tid == NT - 1) {
-          const int4 sp4 = ld_volatile_i4(reinterpret_cast<const int4*>(&P.ring[slot]));
+          const int4 sp4 = ld_volatile_i4(reinterpret_cast<const int4*>(&P.ring[2 * slot + sub]));
           P.dparams[slot] = make_int4(sp4.y, sp4.z, sp4.w, 0);
         }
-        if (tid == NT - 2) P.dtag[slot] = *((const volatile unsigned long long*)&P.ring[slot].tag);
+        if (tid == NT - 2) P.dtag[slot] = *((const volatile unsigned long long*)&P.ring[2 * slot + sub].tag);
       }
       __syncthreads();
       if (tid == 0) {
@@ -285,8 +289,8 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     ResultEntry* out;
     CtaStats* stp;
     if (P.mode == 0) {
-      out = P.ring_res + ((uint64_t)slot * P.T + rank) * P.kmax;
-      stp = P.ring_stats + (uint64_t)slot * P.T + rank;
+      out = P.ring_res + ((uint64_t)(2 * slot + sub) * P.T + rank) * P.kmax;
+      stp = P.ring_stats + (uint64_t)(2 * slot + sub) * P.T + rank;
     } else {
       out = P.dq_res + ((uint64_t)item * P.T + rank) * P.kmax;
       stp = P.dq_stats + (uint64_t)item * P.T + rank;
@@ -307,11 +311,15 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     if (tid == 0) {
       if (P.mode == 0) {
         __threadfence_system();
-        st_release_sys(P.ring_done + (uint64_t)slot * P.T + rank, epoch);
+        st_release_sys(P.ring_done + (uint64_t)(2 * slot + sub) * P.T + rank, epoch);
       } else {
         __threadfence();
         atomicAdd(P.slot_fin + slot, 1u);
       }
+    }
+    if (P.mode == 0) {  // the slot's next query is in its other ring entry
+      last_ep_sub[sub] = epoch;
+      sub ^= 1;
     }
   }
 }

@@ -12,6 +12,7 @@
 #include <cstring>
 #include <deque>
 #include <limits>
+#include <memory>
 #include <queue>
 #include <thread>
 #include <vector>
@@ -87,9 +88,17 @@ struct algas_server {
   float4* qbuf = nullptr;
   unsigned long long* gtab = nullptr;  // the server's own HBM spill tables
   uint32_t* vbm = nullptr;             // SHARED visited bitmaps, two per slot
-  // host-side slot bookkeeping (host owns: EMPTY/claimed/in-flight)
+  // Every slot has TWO ring entries ("sub-slots", index u = 2*slot + b):
+  // the slot's queries alternate between them (b = 1, 0, 1, ...), so the
+  // host can stage a slot's next query while its current one runs, and the
+  // slot's CTAs start it without a host round trip (dynamic batching keeps
+  // B searches running; the staged ones wait in host memory like the FIFO).
+  // Host-side bookkeeping per sub-slot (host owns: EMPTY/claimed/in-flight):
   std::vector<std::atomic<int>>* hstate = nullptr;  // 0 free, 1 claimed, 2 in flight
-  std::vector<uint32_t> epoch;
+  std::vector<uint32_t> epoch;   // per sub-slot: epoch of its query
+  std::vector<uint32_t> next_ep; // per slot: epoch of its next query
+  std::vector<int> next_sub;     // per slot: sub-slot of its next query
+  std::unique_ptr<std::atomic<int>[]> slot_lock;  // per slot: claim lock
   std::vector<uint64_t> tags;
   std::vector<int> kq;
   std::vector<std::chrono::steady_clock::time_point> t_submit;
@@ -117,32 +126,47 @@ struct algas_server {
   std::mutex pq_mu;
   std::deque<Pending> pending;
   std::atomic<int64_t> n_pending{0};
-  std::vector<uint64_t> queue_ns;  // per slot: FIFO wait of its current query
+  std::vector<uint64_t> queue_ns;  // per sub-slot: FIFO wait of its query
 };
 
 namespace {
-// None -> Work of a claimed slot q: payload first, state word last (release)
-void write_slot(algas_server* s, int q, const float* query, uint64_t tag, int32_t k, int32_t itopk, int32_t width) {
-  memcpy(s->ringq_h + (size_t)q * s->dim, query, (size_t)s->dim * 4);
-  RingSlot* rs = &s->ring_h[q];
+// None -> Work of a claimed sub-slot u (epoch already assigned):
+// payload first, state word last (release)
+void write_slot(algas_server* s, int u, const float* query, uint64_t tag, int32_t k, int32_t itopk, int32_t width) {
+  memcpy(s->ringq_h + (size_t)u * s->dim, query, (size_t)s->dim * 4);
+  RingSlot* rs = &s->ring_h[u];
   rs->k = k;
   rs->L = itopk;
   rs->w = width;
   rs->tag = tag;
-  s->tags[q] = tag;
-  s->kq[q] = k;
-  const uint32_t ep = (s->epoch[q] + 1) & 0xFFFFFFu;
-  s->epoch[q] = ep == 0 ? 1 : ep;
-  s->t_submit[q] = std::chrono::steady_clock::now();
-  (*s->hstate)[q].store(2, std::memory_order_release);
-  __atomic_store_n(&rs->state, (s->epoch[q] << 8) | kSlotReady, __ATOMIC_RELEASE);
+  s->tags[u] = tag;
+  s->kq[u] = k;
+  s->t_submit[u] = std::chrono::steady_clock::now();
+  (*s->hstate)[u].store(2, std::memory_order_release);
+  __atomic_store_n(&rs->state, (s->epoch[u] << 8) | kSlotReady, __ATOMIC_RELEASE);
 }
-// claim a free slot (host state 0 -> 1), scanning from `start`; -1 if none
+// claim the next sub-slot of a slot whose next sub-slot is free (host state
+// 0 -> 1) and give it the slot's next epoch, scanning slots from `start`, a
+// slot with nothing in flight first; returns the sub-slot index or -1
 int claim_slot(algas_server* s, int start) {
-  for (int i = 0; i < s->slots; ++i) {
-    const int q = (start + i) % s->slots;
-    int expect = 0;
-    if ((*s->hstate)[q].compare_exchange_strong(expect, 1, std::memory_order_acq_rel)) return q;
+  for (int pass = 0; pass < 2; ++pass) {
+    for (int i = 0; i < s->slots; ++i) {
+      const int q = (start + i) % s->slots;
+      int unlocked = 0;
+      if (!s->slot_lock[q].compare_exchange_strong(unlocked, 1, std::memory_order_acquire)) continue;
+      const int u = 2 * q + s->next_sub[q];
+      const bool idle = (*s->hstate)[u ^ 1].load(std::memory_order_acquire) == 0;
+      int expect = 0;
+      if ((pass == 1 || idle) && (*s->hstate)[u].compare_exchange_strong(expect, 1, std::memory_order_acq_rel)) {
+        s->epoch[u] = s->next_ep[q];
+        const uint32_t ne = (s->next_ep[q] + 1) & 0xFFFFFFu;
+        s->next_ep[q] = ne == 0 ? 1 : ne;
+        s->next_sub[q] ^= 1;
+        s->slot_lock[q].store(0, std::memory_order_release);
+        return u;
+      }
+      s->slot_lock[q].store(0, std::memory_order_release);
+    }
   }
   return -1;
 }
@@ -159,7 +183,7 @@ void drain_pending(algas_server* s, int start) {
     write_slot(s, q, p.q.data(), p.tag, p.k, p.L, p.w);
     s->pending.pop_front();
     s->n_pending.fetch_sub(1, std::memory_order_acq_rel);
-    start = q + 1;
+    start = q / 2 + 1;
   }
 }
 }  // namespace
@@ -172,7 +196,8 @@ static void poller_main(algas_server* s, int me, int nth) {
   int idle = 0;
   while (!s->stop.load(std::memory_order_acquire)) {
     bool any = false;
-    for (int q = me; q < s->slots; q += nth) {
+    for (int q = 0; q < 2 * s->slots; ++q) {  // sub-slots of this poller's slots
+      if ((q >> 1) % nth != me) continue;
       if ((*s->hstate)[q].load(std::memory_order_acquire) != 2) continue;
       const uint32_t ep = s->epoch[q];
       bool all = true;
@@ -206,7 +231,7 @@ static void poller_main(algas_server* s, int me, int nth) {
       __atomic_store_n(&s->ring_h[q].state, (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
       s->queue_ns[q] = 0;
       (*s->hstate)[q].store(0, std::memory_order_release);
-      drain_pending(s, q);
+      drain_pending(s, q >> 1);
       {
         std::lock_guard<std::mutex> lk(s->cq_mu);
         s->cq.push_back(std::move(d));
@@ -256,19 +281,24 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   memset(hp, 0, (bytes));                                                              \
   if ((e = cudaHostGetDevicePointer((void**)&dp, hp, 0)) != cudaSuccess)               \
     return cleanup(set_error(ALGAS_ECUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(e)));
-  SRV_ALLOC(s->ring_h, s->ring_d, sizeof(RingSlot) * slots);
-  SRV_ALLOC(s->ringq_h, s->ringq_d, (size_t)slots * s->dim * 4);
-  SRV_ALLOC(s->res_h, s->res_d, sizeof(ResultEntry) * (size_t)slots * s->T * s->kmax);
-  SRV_ALLOC(s->st_h, s->st_d, sizeof(CtaStats) * (size_t)slots * s->T);
-  SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)slots * s->T);
+  const int nsub = 2 * slots;  // two ring entries per slot (sub-slots)
+  SRV_ALLOC(s->ring_h, s->ring_d, sizeof(RingSlot) * nsub);
+  SRV_ALLOC(s->ringq_h, s->ringq_d, (size_t)nsub * s->dim * 4);
+  SRV_ALLOC(s->res_h, s->res_d, sizeof(ResultEntry) * (size_t)nsub * s->T * s->kmax);
+  SRV_ALLOC(s->st_h, s->st_d, sizeof(CtaStats) * (size_t)nsub * s->T);
+  SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)nsub * s->T);
 #undef SRV_ALLOC
-  s->hstate = new std::vector<std::atomic<int>>(slots);
+  s->hstate = new std::vector<std::atomic<int>>(nsub);
   for (auto& a : *s->hstate) a.store(0);
-  s->epoch.assign(slots, 0);
-  s->tags.assign(slots, 0);
-  s->kq.assign(slots, s->kmax);
-  s->t_submit.resize(slots);
-  s->queue_ns.assign(slots, 0);
+  s->epoch.assign(nsub, 0);
+  s->tags.assign(nsub, 0);
+  s->kq.assign(nsub, s->kmax);
+  s->t_submit.resize(nsub);
+  s->queue_ns.assign(nsub, 0);
+  s->next_ep.assign(slots, 1);
+  s->next_sub.assign(slots, 1);  // the kernel serves sub-slot 1 first, then alternates
+  s->slot_lock.reset(new std::atomic<int>[slots]);
+  for (int q = 0; q < slots; ++q) s->slot_lock[q].store(0);
   const size_t ctl_bytes = control_bytes(slots);
   if ((e = cudaMalloc(&s->ctl, ctl_bytes)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc: %s", cudaGetErrorString(e)));
@@ -416,7 +446,7 @@ int algas_server_destroy(algas_server* s) {
   int rc = ALGAS_OK;
   if (s->ring_h && s->stream) {
     // Quit: every slot, then wait for the kernel to exit
-    for (int q = 0; q < s->slots; ++q) __atomic_store_n(&s->ring_h[q].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+    for (int u = 0; u < 2 * s->slots; ++u) __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
     auto t0 = std::chrono::steady_clock::now();
     for (;;) {
       cudaError_t e = cudaStreamQuery(s->stream);

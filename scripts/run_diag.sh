@@ -1,3 +1,5 @@
 # ad-hoc GPU diagnostics (one gpurun call)
-timeout 900 python -m pytest tests/test_search_gpu.py -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc=$?; tail -3 gpurun_out/pytest_gpu.log
-for PF in 8 8; do echo "== ALGAS_PREFETCH=$PF"; ALGAS_PREFETCH=$PF timeout 300 python scripts/probe_call.py C2 12,12,1,4,1024,1 32,8,1,2,1024,1 2>&1 | grep -E "^recall|^latency|^per query"; done > gpurun_out/fm.log 2>&1
+timeout 900 python bench.py --ctas 4 --threads 1024 --width 12 --visited 1 --no-cpu --no-sweep > gpurun_out/bench_e2e.json 2> gpurun_out/bench_e2e.err; echo bench rc=$?
+python -c "
+import json;l=json.load(open('gpurun_out/bench_e2e.json'))
+print(l['value'], json.dumps(l['latency_us']), json.dumps(l['e2e']))"
