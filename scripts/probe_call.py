@@ -1,6 +1,6 @@
 """Where does a search_dynamic call / a query spend its time? (GPU box)
 
-usage: [ALGAS_TRACE=1] python scripts/probe_call.py C2 L,w,off,T,threads,visited [L,w,off,T,threads,visited ...]
+usage: [ALGAS_TRACE=1] python scripts/probe_call.py C2 L,w,off,T,threads,visited[,seeds] [...]
 Prints per call: CUDA-event time, host call phases, kernel time; per config:
 per-query work counters, phase cycles, and the device-timestamp timeline of a
 query (pickup -> CTAs in loop -> loop end -> published)."""
@@ -29,10 +29,13 @@ idx = algas.Index(Xd, G, w.metric)
 st = torch.cuda.current_stream()
 
 for spec in sys.argv[2:]:
-    L, wd, off, T, nt, vis = (int(x) for x in spec.split(","))
+    f = [int(x) for x in spec.split(",")]
+    L, wd, off, T, nt, vis = f[:6]
+    S = f[6] if len(f) > 6 else 32
     p = algas.default_params(k=w.k, itopk=L, width=wd, offset_beam=off, ctas_per_query=T, threads_per_cta=nt,
-                             slots=32, seed=1, visited_mode=vis)
-    print(f"==== L={L} w={wd} off={off} T={T} threads={nt} visited={'shared' if vis else 'private'}", flush=True)
+                             slots=32, seed=1, visited_mode=vis, n_seeds=S)
+    print(f"==== L={L} w={wd} off={off} T={T} threads={nt} visited={'shared' if vis else 'private'} seeds={S}",
+          flush=True)
     for i in range(4):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()

@@ -1,5 +1,2 @@
-# ad-hoc GPU diagnostics (one gpurun call)
-timeout 900 python bench.py --ctas 4 --threads 1024 --width 12 --visited 1 --no-cpu --no-sweep > gpurun_out/bench_e2e.json 2> gpurun_out/bench_e2e.err; echo bench rc=$?
-python -c "
-import json;l=json.load(open('gpurun_out/bench_e2e.json'))
-print(l['value'], json.dumps(l['latency_us']), json.dumps(l['e2e']))"
+# ad-hoc GPU diagnostics (one gpurun call): fixed entry sample
+for EF in 0 1; do echo "== ENTRY_FIXED=$EF"; ALGAS_ENTRY_FIXED=$EF timeout 600 python scripts/probe_call.py C2 12,12,1,4,1024,1,32 12,12,1,4,1024,1,256 10,10,1,4,1024,1,256 12,12,1,2,1024,1,256 2>&1 | grep -E "^====|^recall|^latency|^per query"; done > gpurun_out/entry.log
