@@ -471,7 +471,7 @@ def run_reference(a, rank, world, local):
     torch.cuda.set_device(dev)
     X, Q, Xd, Qd, G, truth, (Qcd, tcal), _ = build_workload(w, a.nq, dev)
     idx = algas.Index(Xd, G, w.metric)
-    p, sweep = choose_operating_point(idx, Qcd, tcal, w, a.batch, Ts=a.ctas, threads=a.threads, widths=a.width,
+    p, sweep = choose_operating_point(idx, Qd, truth, w, a.batch, Ts=a.ctas, threads=a.threads, widths=a.width,
                                       offsets=a.offset, visited=a.visited)
     del idx
     import oracle
