@@ -309,12 +309,17 @@ def run_algas(a, rank, world, local):
                 # at once; the poller thread feeds slots as they free up
                 # (algas_enqueue), each slot staging its next query while its
                 # current one runs
-                done = 0
+                # (queries are handed over in chunks while results are polled,
+                # keeping <= 8 x batch queries queued: a client streaming work)
+                done = sent = 0
+                win = 8 * a.batch
                 t0 = time.perf_counter()
-                for s0 in range(0, nq, Q.shape[0]):
-                    m = min(Q.shape[0], nq - s0)
-                    srv.enqueue(Q[:m], tag0=s0)
                 while done < nq:
+                    if sent < nq and sent - done < win:
+                        i0 = sent % Q.shape[0]
+                        m = min(win - (sent - done), nq - sent, Q.shape[0] - i0)
+                        srv.enqueue(Q[i0:i0 + m], tag0=sent)
+                        sent += m
                     tags, ids, ds, st = srv.poll(256)
                     done += len(tags)
                 return time.perf_counter() - t0

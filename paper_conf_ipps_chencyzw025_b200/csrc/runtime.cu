@@ -39,12 +39,31 @@ int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t*
     if (kin > 0 && e.id != kSentinel) pq.push(H{e.dist, e.id, c, 0});
   }
   int n = 0;
+  // repeated ids (R11): a linear scan of the emitted ids for small k, an
+  // open-addressing set for large k (k = 100 would cost k^2/2 compares)
+  const bool use_set = k > 32;
+  uint32_t set_bits = 6;
+  while ((1u << set_bits) < 2u * (uint32_t)k) ++set_bits;
+  thread_local std::vector<uint32_t> set;
+  if (use_set) set.assign((size_t)1 << set_bits, kSentinel);
+  auto seen_insert = [&](uint32_t id) -> bool {  // true if id was already emitted
+    const uint32_t mask = (1u << set_bits) - 1u;
+    uint32_t h = (id * 0x9E3779B1u) >> (32 - set_bits);
+    for (;; h = (h + 1) & mask) {
+      if (set[h] == id) return true;
+      if (set[h] == kSentinel) { set[h] = id; return false; }
+    }
+  };
   while (!pq.empty() && n < k) {
     H h = pq.top();
     pq.pop();
     bool dup = false;
-    for (int i = 0; i < n; ++i)
-      if (out_ids[i] == h.id) { dup = true; break; }
+    if (use_set) {
+      dup = seen_insert(h.id);
+    } else {
+      for (int i = 0; i < n; ++i)
+        if (out_ids[i] == h.id) { dup = true; break; }
+    }
     if (!dup) {
       out_ids[n] = h.id;
       out_d[n] = h.d;
@@ -121,7 +140,8 @@ struct algas_server {
     uint64_t tag;
     int32_t k, L, w;
     std::chrono::steady_clock::time_point t_enq;
-    std::vector<float> q;
+    std::shared_ptr<const std::vector<float>> blk;  // the enqueue call's copy of its queries
+    int64_t off;                                    // this query's offset in blk
   };
   std::mutex pq_mu;
   std::deque<Pending> pending;
@@ -180,7 +200,7 @@ void drain_pending(algas_server* s, int start) {
     algas_server::Pending& p = s->pending.front();
     s->queue_ns[q] = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
                          std::chrono::steady_clock::now() - p.t_enq).count();
-    write_slot(s, q, p.q.data(), p.tag, p.k, p.L, p.w);
+    write_slot(s, q, p.blk->data() + p.off, p.tag, p.k, p.L, p.w);
     s->pending.pop_front();
     s->n_pending.fetch_sub(1, std::memory_order_acq_rel);
     start = q / 2 + 1;
@@ -391,6 +411,8 @@ int algas_enqueue(algas_server* s, const float* queries, int64_t n, uint64_t tag
                      s->kmax, s->plan.cfg.L, s->plan.cfg.w);
   if (n == 0) return ALGAS_OK;
   const auto now = std::chrono::steady_clock::now();
+  // one copy of the whole call (the caller keeps ownership of `queries`)
+  auto blk = std::make_shared<const std::vector<float>>(queries, queries + n * (int64_t)s->dim);
   {
     std::lock_guard<std::mutex> lk(s->pq_mu);
     for (int64_t i = 0; i < n; ++i) {
@@ -400,7 +422,8 @@ int algas_enqueue(algas_server* s, const float* queries, int64_t n, uint64_t tag
       p.L = itopk;
       p.w = width;
       p.t_enq = now;
-      p.q.assign(queries + i * (int64_t)s->dim, queries + (i + 1) * (int64_t)s->dim);
+      p.blk = blk;
+      p.off = i * (int64_t)s->dim;
       s->pending.push_back(std::move(p));
     }
     s->inflight.fetch_add(n);

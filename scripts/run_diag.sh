@@ -1,4 +1,7 @@
-# ad-hoc GPU diagnostics (one gpurun call): refresh C3 / C4 bench lines and the f1 ablation
-timeout 900 python scripts/ablation.py C2 > gpurun_out/ablation.log 2>&1; echo ablation rc=$?
-timeout 1500 python bench.py --config C3 --nq 2000 --ctas 1,2,4,8 --threads 512 --width 8,16 > gpurun_out/bench_C3.json 2> gpurun_out/bench_C3.err; echo C3 rc=$?
-timeout 1500 python bench.py --config C4 --ctas 1,2,4,8 --threads 512,1024 --width 8,16 > gpurun_out/bench_C4.json 2> gpurun_out/bench_C4.err; echo C4 rc=$?
+# ad-hoc GPU diagnostics (one gpurun call)
+timeout 900 python -m pytest tests/test_search_gpu.py -x -q -k "server or enqueue" > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc=$?; tail -2 gpurun_out/pytest_gpu.log
+timeout 900 python bench.py --ctas 4 --threads 1024 --width 12 --visited 1 --no-cpu --no-sweep > gpurun_out/bench_e2e.json 2> gpurun_out/bench_e2e.err; echo bench rc=$?
+timeout 900 python bench.py --config C4 --ctas 4 --threads 1024 --width 16 --visited 1 --no-cpu --no-sweep > gpurun_out/bench_e2e_C4.json 2> gpurun_out/bench_e2e_C4.err; echo bench rc=$?
+for f in bench_e2e bench_e2e_C4; do python -c "
+import json;l=json.load(open('gpurun_out/$f.json'))
+print('$f', l['value'], json.dumps(l['latency_us']), json.dumps(l['e2e']))"; done

@@ -52,6 +52,24 @@ def test_host_merge_matches_oracle_merge():
         assert a[2] == b[2]
 
 
+def test_host_merge_large_k_matches_oracle_merge():
+    """k > 32 takes the hashed duplicate filter (k = 100 at C4): same output
+    as the oracle's merge, including repeated ids across per-CTA lists."""
+    rng = np.random.default_rng(4)
+    for _ in range(100):
+        m = int(rng.integers(0, 600))
+        ids = rng.integers(0, 300, size=m).astype(np.uint32)
+        ids[rng.random(m) < 0.05] = algas.SENTINEL
+        table = rng.integers(0, 50, size=300).astype(np.float32)
+        ds = np.where(ids == algas.SENTINEL, np.float32(np.inf), table[np.minimum(ids, 299)]).astype(np.float32)
+        k = int(rng.integers(33, 160))
+        a = algas.merge_topk(ids, ds, k)
+        b = oracle.merge_topk(ids, ds, k)
+        np.testing.assert_array_equal(a[0], b[0])
+        np.testing.assert_array_equal(a[1], b[1])
+        assert a[2] == b[2]
+
+
 def test_tuner_equations_match_oracle_and_table2():
     L = algas.lib()
     g = json.load(open(os.path.join(ROOT, "tests", "golden", "table2_tuner.json")))
