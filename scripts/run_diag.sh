@@ -1,7 +1,3 @@
-# ad-hoc GPU diagnostics (one gpurun call)
-timeout 900 python -m pytest tests/test_search_gpu.py -x -q -k "server or enqueue" > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc=$?; tail -2 gpurun_out/pytest_gpu.log
-timeout 900 python bench.py --ctas 4 --threads 1024 --width 12 --visited 1 --no-cpu --no-sweep > gpurun_out/bench_e2e.json 2> gpurun_out/bench_e2e.err; echo bench rc=$?
-timeout 900 python bench.py --config C4 --ctas 4 --threads 1024 --width 16 --visited 1 --no-cpu --no-sweep > gpurun_out/bench_e2e_C4.json 2> gpurun_out/bench_e2e_C4.err; echo bench rc=$?
-for f in bench_e2e bench_e2e_C4; do python -c "
-import json;l=json.load(open('gpurun_out/$f.json'))
-print('$f', l['value'], json.dumps(l['latency_us']), json.dumps(l['e2e']))"; done
+# ad-hoc GPU diagnostics (one gpurun call): chunk config 7 (4 lanes x 8 chunks) A/B
+timeout 900 python -m pytest tests/test_search_gpu.py -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc=$?; tail -1 gpurun_out/pytest_gpu.log
+for CC in 0 7 0 7; do echo "== ALGAS_CC=$CC"; ALGAS_CC=$CC timeout 300 python scripts/probe_call.py C2 12,12,1,4,1024,1 32,8,1,2,1024,1 2>&1 | grep -E "^recall|^latency|^per query"; done > gpurun_out/cc.log 2>&1
