@@ -210,10 +210,16 @@ int algas_search_dynamic(const algas_index *idx, const float *queries_dev, int64
 /* ------------------------------------------------------------------ */
 /* Launches the persistent kernel (cooperative launch: all slots x T CTAs
  * co-resident).  params->k / itopk are the per-server maxima; a
- * submit may ask for smaller k/itopk/width.  *out is NULL on failure. */
+ * submit may ask for smaller k/itopk/width.  *out is NULL on failure.
+ * Each of the B slots has two ring entries in host-mapped memory: a slot
+ * runs one query at a time (B searches in flight) while its next query can
+ * already be staged in the other entry, so a slot's CTAs start the next
+ * query without waiting for the host (the host merges the finished one
+ * meanwhile).  Submitting fills idle slots first.  Host poller threads:
+ * params->host_threads. */
 int algas_server_create(const algas_index *idx, const algas_params *params, algas_server **out);
-/* Non-blocking.  query: dim fp32 in HOST memory.  Claims an EMPTY slot
- * (EMPTY -> READY); ALGAS_EAGAIN if every slot is busy.
+/* Non-blocking.  query: dim fp32 in HOST memory (copied).  Claims a free
+ * ring entry (EMPTY -> READY); ALGAS_EAGAIN if every entry is busy.
  * k <= server k, itopk <= server itopk, width <= 32 (0 -> server value). */
 int algas_submit(algas_server *s, const float *query, uint64_t tag, int32_t k, int32_t itopk,
                  int32_t width);
