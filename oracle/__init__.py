@@ -38,6 +38,7 @@ _lib = None
 SENTINEL = 0xFFFFFFFF
 L2 = 0
 IP = 1
+COSINE = 2  # -(q.x)/(|q||x|), R29
 
 
 def build(force: bool = False) -> str:
@@ -47,7 +48,7 @@ def build(force: bool = False) -> str:
         return _LIB_PATH
     tmp = _LIB_PATH + f".tmp{os.getpid()}"
     subprocess.check_call(["gcc", "-O2", "-std=c99", "-ffp-contract=off", "-fno-fast-math",
-                           "-fPIC", "-shared", "-Wall", "-o", tmp, _SRC])
+                           "-fPIC", "-shared", "-Wall", "-o", tmp, _SRC, "-lm"])
     os.replace(tmp, _LIB_PATH)
     return _LIB_PATH
 

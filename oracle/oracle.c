@@ -34,6 +34,7 @@
  *                                     the paper; pinned by hand-worked
  *                                     examples and invariants, R24)
  */
+#include <math.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -41,6 +42,7 @@
 #define ORC_SENTINEL 0xFFFFFFFFu
 #define ORC_L2 0
 #define ORC_IP 1
+#define ORC_COSINE 2
 
 /* ------------------------------------------------------------------ */
 /* Counter-based generator for entry points (R5).            */
@@ -77,6 +79,19 @@ float orc_distance(const float *q, const float *x, int32_t d, int32_t metric)
             acc = acc + t * t;
         }
         return acc;
+    }
+    if (metric == ORC_COSINE) {
+        /* COSINE (two of the paper's datasets are "cosine";
+         * DESIGN.md R29): -(q.x) / (|q| |x|), the negated cosine similarity,
+         * in double; a zero vector has distance 0 to everything. */
+        double qx = 0.0, qq = 0.0, xx = 0.0;
+        for (j = 0; j < d; j++) {
+            qx += (double)q[j] * (double)x[j];
+            qq += (double)q[j] * (double)q[j];
+            xx += (double)x[j] * (double)x[j];
+        }
+        if (qq == 0.0 || xx == 0.0) return 0.0f;
+        return (float)(-qx / (sqrt(qq) * sqrt(xx)));
     }
     for (j = 0; j < d; j++)
         acc = acc + q[j] * x[j];

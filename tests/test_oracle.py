@@ -380,3 +380,66 @@ def test_generator_acceptance_C1_small():
     assert len({find(u) for u in range(n)}) == 1
     ids, ds, st = oracle.search(X, G, Q, oracle.make_params(k=10, L=16, T=1, S=32, seed=0))
     assert st["iters"].max() / st["iters"].mean() >= 1.3
+
+
+# ---------------------------------------------------------------- COSINE (f3, R29)
+def test_cosine_hand_values():
+    """-(q.x)/(|q||x|): parallel -1, orthogonal 0, opposite +1, (3,4).(4,3) = 24/25."""
+    q = np.array([1, 0], np.float32)
+    assert oracle.distance(q, np.array([2, 0], np.float32), oracle.COSINE) == -1.0
+    assert oracle.distance(q, np.array([0, 3], np.float32), oracle.COSINE) == 0.0
+    assert oracle.distance(q, np.array([-5, 0], np.float32), oracle.COSINE) == 1.0
+    assert oracle.distance(np.array([3, 4], np.float32), np.array([4, 3], np.float32),
+                           oracle.COSINE) == np.float32(-0.96)
+    assert oracle.distance(q, np.zeros(2, np.float32), oracle.COSINE) == 0.0
+
+
+def test_cosine_angles_closed_form():
+    """q = (cos a, sin a), x = r (cos b, sin b), any r > 0: -cos(a - b)."""
+    rng = np.random.default_rng(3)
+    for _ in range(200):
+        a, b = rng.uniform(-np.pi, np.pi, 2)
+        r = rng.uniform(0.01, 100.0)
+        q = np.array([np.cos(a), np.sin(a)], np.float32)
+        x = (r * np.array([np.cos(b), np.sin(b)])).astype(np.float32)
+        assert abs(oracle.distance(q, x, oracle.COSINE) + np.cos(a - b)) <= 1e-6
+
+
+def test_cosine_bruteforce_circle_order():
+    """n points on the unit circle at angles 2 pi i / n, each scaled by its own
+    random radius (cosine ignores it); the k nearest of a query at angle
+    theta are the k smallest angular gaps, a closed-form order."""
+    n, k = 360, 9
+    rng = np.random.default_rng(4)
+    ang = 2 * np.pi * np.arange(n) / n
+    rad = rng.uniform(0.1, 10.0, n)
+    X = np.stack([rad * np.cos(ang), rad * np.sin(ang)], 1).astype(np.float32)
+    X = np.concatenate([X, np.zeros((n, 2), np.float32)], 1)  # d = 4 (row alignment)
+    thetas = 2 * np.pi * (np.arange(20) + 0.3) / 20   # never equidistant from two points
+    Q = np.stack([np.cos(thetas), np.sin(thetas), np.zeros(20), np.zeros(20)], 1).astype(np.float32)
+    ids, ds = oracle.brute_force(X, Q, k, oracle.COSINE)
+    for t, th in enumerate(thetas):
+        gap = np.abs((ang - th + np.pi) % (2 * np.pi) - np.pi)
+        assert set(ids[t].tolist()) == set(np.argsort(gap)[:k].tolist())
+        np.testing.assert_allclose(ds[t], -np.cos(np.sort(gap)[:k]), atol=1e-6)
+
+
+def test_cosine_search_exhaustive_equals_bruteforce():
+    """L >= n on a connected graph: O2 scores every point, O2 == O1 (COSINE)."""
+    n, d = 150, 8
+    rng = np.random.default_rng(24)
+    X = rng.standard_normal((n, d)).astype(np.float32) * rng.uniform(0.5, 3.0, (n, 1)).astype(np.float32)
+    Q = rng.standard_normal((6, d)).astype(np.float32)
+    G = synth.random_graph(n, 6, seed=23)
+    p = oracle.make_params(k=12, L=n, w=2, off=4, T=2, S=2, max_iter=10 * n, shared_visited=1, seed=5)
+    seeds = [oracle.entry_point(5, t, c, j, n) for t in range(6) for c in range(2) for j in range(2)]
+    assert _reachable(G, seeds).all()
+    ids, ds, st = oracle.search(X, G, Q, p, metric=oracle.COSINE)
+    ei, ed = oracle.brute_force(X, Q, 12, oracle.COSINE)
+    np.testing.assert_array_equal(ids, ei)
+    np.testing.assert_array_equal(ds, ed)
+    # and O1 COSINE ranks like -q.x on rows normalised in float64 (numpy)
+    Xn = X / np.linalg.norm(X.astype(np.float64), axis=1, keepdims=True)
+    for t in range(6):
+        ref = -(Xn @ Q[t].astype(np.float64)) / np.linalg.norm(Q[t].astype(np.float64))
+        np.testing.assert_allclose(ed[t], np.sort(ref)[:12], atol=1e-6)
