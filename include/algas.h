@@ -49,7 +49,12 @@ extern "C" {
 #define ALGAS_MAX_CTAS 64     /* max CTAs per query (N_parallel)        */
 #define ALGAS_MAX_SEEDS 256   /* max random entry points per CTA        */
 
-enum algas_metric { ALGAS_L2 = 0, ALGAS_IP = 1 };
+/* L2: squared Euclidean; IP: -q.x; COSINE: -(q.x)/(|q||x|), the negated
+ * cosine similarity (the paper's cosine datasets; DESIGN.md
+ * R29).  COSINE is served as IP on unit rows: algas_index_create normalises
+ * its HBM copy of the data, every search kernel normalises the query in
+ * shared memory when it is staged; a zero row / query scores 0. */
+enum algas_metric { ALGAS_L2 = 0, ALGAS_IP = 1, ALGAS_COSINE = 2 };
 
 enum algas_status {
     ALGAS_OK = 0,
@@ -162,7 +167,10 @@ const char *algas_version(void);
  * graph == NULL builds the graph: exact kNN with 2*degree neighbours
  * (algas_knn) followed by CAGRA-style pruning to `degree` (algas_prune).
  * EINVAL (returns NULL): n < 1 or n >= 2^31, dim < 4, dim % 4 != 0,
- * dim > ALGAS_MAX_DIM, degree < 1 or > ALGAS_MAX_DEGREE, bad metric. */
+ * dim > ALGAS_MAX_DIM, degree < 1 or > ALGAS_MAX_DEGREE, bad metric.
+ * metric COSINE: the HBM copy of data is normalised to unit rows (the
+ * caller's buffer is untouched) and the built graph is the IP graph of the
+ * unit rows (= the cosine kNN graph). */
 algas_index *algas_index_create(const float *data, int64_t n, int32_t dim, int32_t metric,
                                 const uint32_t *graph, int32_t degree);
 int algas_index_destroy(algas_index *idx);

@@ -21,13 +21,14 @@ from .build import LIB as _LIB_PATH, build as _build
 SENTINEL = 0xFFFFFFFF
 L2 = 0
 IP = 1
+COSINE = 2  # -(q.x)/(|q||x|): IP on unit rows (include/algas.h, R29)
 VISITED_PRIVATE = 0
 VISITED_SHARED = 1
 
 OK, EINVAL, ENOMEM, ECUDA, EAGAIN, ESTATE, ENCCL, EOVERFLOW = 0, -1, -2, -3, -4, -5, -6, -7
 
 __all__ = ["Index", "Server", "Params", "QueryStats", "RunInfo", "lib", "knn", "prune", "build_graph",
-           "merge_topk", "merge_topk_parts", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP"]
+           "merge_topk", "merge_topk_parts", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP", "COSINE"]
 
 
 class AlgasError(RuntimeError):

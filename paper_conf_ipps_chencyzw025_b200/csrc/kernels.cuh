@@ -92,6 +92,7 @@ __global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
     const int c = (int)(item - qi * a.T);
     const float4* qsrc = a.queries + qi * a.cfg.d4;
     for (int i = threadIdx.x; i < a.cfg.d4; i += NT) s.q[i] = qsrc[i];
+    if (a.cfg.cosine) normalize_query<NT>(s.q, a.cfg.d4);
     __syncthreads();
     CtaStats* st = a.stats ? a.stats + item : nullptr;
     search_cta<NT, TL, CPL, METRIC>(a.cfg, s, a.tag0 + (uint64_t)qi, (uint32_t)c, a.k, gt,
@@ -278,6 +279,7 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       const uint4 z = make_uint4(0u, 0u, 0u, 0u);
       for (int64_t i = lo + tid; i < hi; i += NT) o4[i] = z;
     }
+    if (A.cfg.cosine) normalize_query<NT>(s.q, A.cfg.d4);  // COSINE (R29), before the cluster push
     if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
     __syncthreads();
 

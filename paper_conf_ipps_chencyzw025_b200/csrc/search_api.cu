@@ -157,7 +157,7 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   pl.k = k;
   pl.smem = lay.total;
   pl.visited_mode = p->visited_mode;
-  pl.metric = idx->metric;
+  pl.metric = idx->metric == ALGAS_COSINE ? ALGAS_IP : idx->metric;  // COSINE = IP on unit rows (R29)
   pl.cluster = cs;
   // a persistent grid of more searches than SMs runs two 256/512-thread CTAs
   // per SM (the build with half the registers per thread)
@@ -183,6 +183,7 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   c.prefetch = prefetch;
   c.gc_bits = gcbits;
   c.seed = p->seed;
+  c.cosine = idx->metric == ALGAS_COSINE ? 1 : 0;
   c.shared = p->visited_mode == ALGAS_VISITED_SHARED ? 1 : 0;
   if (c.shared && cs > 1) return set_error(ALGAS_EINVAL, "SHARED visited mode needs cluster_size 1");
   int nb = 0;
@@ -390,12 +391,33 @@ void algas_params_default(algas_params* p) {
 }
 
 const char* algas_last_error(void) { return g_err.c_str(); }
+// COSINE index (R29): one warp per row, v <- v / |v| (fp32; a zero row stays 0)
+__global__ void normalize_rows_kernel(float4* x, int64_t n, int d4) {
+  const int64_t row = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= n) return;
+  float4* r = x + row * d4;
+  float ss = 0.f;
+  for (int i = lane; i < d4; i += 32) {
+    const float4 v = r[i];
+    ss = fmaf(v.x, v.x, fmaf(v.y, v.y, fmaf(v.z, v.z, fmaf(v.w, v.w, ss))));
+  }
+  for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+  if (ss <= 0.f) return;
+  const float inv = 1.0f / sqrtf(ss);
+  for (int i = lane; i < d4; i += 32) {
+    float4 v = r[i];
+    v.x *= inv; v.y *= inv; v.z *= inv; v.w *= inv;
+    r[i] = v;
+  }
+}
+
 const char* algas_version(void) { return "algas-b200 0.1 (sm_100a)"; }
 
 algas_index* algas_index_create(const float* data, int64_t n, int32_t dim, int32_t metric, const uint32_t* graph,
                                 int32_t degree) {
   if (!data || n < 1 || n >= (1LL << 31) || dim < 4 || dim % 4 != 0 || dim > ALGAS_MAX_DIM || degree < 1 ||
-      degree > ALGAS_MAX_DEGREE || (metric != ALGAS_L2 && metric != ALGAS_IP)) {
+      degree > ALGAS_MAX_DEGREE || (metric != ALGAS_L2 && metric != ALGAS_IP && metric != ALGAS_COSINE)) {
     set_error(ALGAS_EINVAL, "algas_index_create: bad arguments (n=%lld dim=%d degree=%d metric=%d)", (long long)n,
               dim, degree, metric);
     return nullptr;
@@ -420,13 +442,21 @@ algas_index* algas_index_create(const float* data, int64_t n, int32_t dim, int32
   cudaError_t e;
   if ((e = cudaMalloc(&idx->d_data, dbytes)) != cudaSuccess) return fail("cudaMalloc data", e);
   if ((e = cudaMemcpy(idx->d_data, data, dbytes, cudaMemcpyDefault)) != cudaSuccess) return fail("copy data", e);
+  if (metric == ALGAS_COSINE) {
+    // unit rows in HBM: the search (and the graph build) run as IP on them (R29)
+    const int64_t warps_per_block = 8;
+    normalize_rows_kernel<<<(unsigned)((n + warps_per_block - 1) / warps_per_block), 32 * warps_per_block>>>(
+        reinterpret_cast<float4*>(idx->d_data), n, dim / 4);
+    if ((e = cudaGetLastError()) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess)
+      return fail("normalize rows", e);
+  }
   if ((e = cudaMalloc(&idx->d_graph, (size_t)n * gpitch)) != cudaSuccess) return fail("cudaMalloc graph", e);
   if ((e = cudaMemset(idx->d_graph, 0xFF, (size_t)n * gpitch)) != cudaSuccess) return fail("memset graph", e);
   std::vector<uint32_t> built;
   const uint32_t* g = graph;
   if (!g) {
     built.resize((size_t)n * degree);
-    int rc = algas_build_graph(idx->d_data, n, dim, metric, std::min<int64_t>(2 * degree, std::max<int64_t>(1, n - 1)),
+    int rc = algas_build_graph(idx->d_data, n, dim, metric == ALGAS_COSINE ? ALGAS_IP : metric, std::min<int64_t>(2 * degree, std::max<int64_t>(1, n - 1)),
                                degree, 1, built.data());
     if (rc != ALGAS_OK) {
       algas_index_destroy(idx);

@@ -218,6 +218,8 @@ struct SearchCfg {
   int32_t shared;        // 1: SHARED visited mode -- the HBM table passed to search_cta is the
                          //    query's table, shared by its T CTAs; the shared-memory
                          //    hash is this CTA's cache of it
+  int32_t cosine;        // 1: COSINE index (unit data rows, METRIC = kIP): the staged query is
+                         //    normalised in shared memory (normalize_query) before the search
   uint64_t seed;
 };
 
@@ -666,6 +668,33 @@ __device__ __forceinline__ uint64_t warp_bitonic_merge32(uint64_t list, uint64_t
     m = ((lane & j) == 0) ? umin64(m, y) : umax64(m, y);
   }
   return m;
+}
+
+// COSINE (R29): q <- q / |q| in shared memory, by warp 0, between two CTA
+// barriers (the staging threads' stores are visible to warp 0 after the
+// first; everyone reads the unit query after the second).  Every CTA of a
+// query computes the same fp32 value in the same order.  Zero query: kept.
+template <int NT>
+__device__ __forceinline__ void normalize_query(float4* q, int d4) {
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    const int lane = threadIdx.x;
+    float ss = 0.f;
+    for (int i = lane; i < d4; i += 32) {
+      const float4 v = q[i];
+      ss = fmaf(v.x, v.x, fmaf(v.y, v.y, fmaf(v.z, v.z, fmaf(v.w, v.w, ss))));
+    }
+    for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+    if (ss > 0.f) {
+      const float inv = 1.0f / sqrtf(ss);
+      for (int i = lane; i < d4; i += 32) {
+        float4 v = q[i];
+        v.x *= inv; v.y *= inv; v.z *= inv; v.w *= inv;
+        q[i] = v;
+      }
+    }
+  }
+  __syncthreads();
 }
 
 // Preconditions: s.q holds the query (d4 float4, zero tail); init_cta() ran.
