@@ -147,6 +147,39 @@ def knn_graph(X, K: int, metric: int = L2):
     return brute_force(X, X, K, metric, self_base=0)
 
 
+def knn_partitioned(X, k: int, n_clusters: int, overlap: int, metric: int = L2):
+    """Partitioned approximate kNN graph (R30), step by
+    step: (1) centres = rows floor(j n / m); (2) each point's `overlap`
+    nearest centres (O1 over the centres); (3) cluster members in ascending
+    id; (4) O1 inside each cluster, self excluded, k_j = min(k, s_j - 1);
+    (5) per point: its cluster lists merged by (dist, id), repeated ids
+    dropped, first k (orc_merge_topk).  Parity unpinned by the paper (it
+    gives no build algorithm); pinned by m = 1 and overlap = m (== O1) and a
+    hand-worked example (tests/test_oracle.py)."""
+    X = _f32(X)
+    n = X.shape[0]
+    m, c = n_clusters, overlap
+    centres = X[[(j * n) // m for j in range(m)]]
+    asg, _ = brute_force(centres, X, c, metric)
+    cand_i = np.full((n, c, k), SENTINEL, np.uint32)
+    cand_d = np.full((n, c, k), np.inf, np.float32)
+    for j in range(m):
+        mem = np.array([i for i in range(n) if j in asg[i]], np.int64)
+        if mem.shape[0] < 2:
+            continue
+        kj = min(k, mem.shape[0] - 1)
+        li, ld = brute_force(X[mem], X[mem], kj, metric, self_base=0)
+        for t, i in enumerate(mem):
+            r = list(asg[i]).index(j)
+            cand_i[i, r, :kj] = mem[li[t]]
+            cand_d[i, r, :kj] = ld[t]
+    ids = np.empty((n, k), np.uint32)
+    ds = np.empty((n, k), np.float32)
+    for i in range(n):
+        ids[i], ds[i], _ = merge_topk(cand_i[i], cand_d[i], k)
+    return ids, ds
+
+
 def merge_topk(ids, dists, k: int):
     ids, dists = _u32(ids).ravel(), _f32(dists).ravel()
     oi = np.empty(k, np.uint32)

@@ -443,3 +443,52 @@ def test_cosine_search_exhaustive_equals_bruteforce():
     for t in range(6):
         ref = -(Xn @ Q[t].astype(np.float64)) / np.linalg.norm(Q[t].astype(np.float64))
         np.testing.assert_allclose(ed[t], np.sort(ref)[:12], atol=1e-6)
+
+
+# ---------------------------------------------------------------- partitioned kNN build (f4, R30)
+def test_knn_partitioned_hand_example():
+    """1-d points 0,1,2 | 10,11,12 (d padded to 4); m = 2 -> centres rows 0
+    and 3 (x = 0, x = 10); overlap 1 -> clusters {0,1,2}, {3,4,5}; k = 3:
+    each point sees only its own cluster (2 neighbours), the 3rd slot is
+    padding, unlike the exact kNN whose 3rd neighbour crosses the gap."""
+    x = np.array([0, 1, 2, 10, 11, 12], np.float32)
+    X = np.zeros((6, 4), np.float32)
+    X[:, 0] = x
+    ids, ds = oracle.knn_partitioned(X, 3, 2, 1)
+    assert ids[0].tolist() == [1, 2, oracle.SENTINEL] and ds[0].tolist()[:2] == [1.0, 4.0]
+    assert ids[1].tolist()[:2] == [0, 2] and ds[1].tolist()[:2] == [1.0, 1.0]   # tie by id
+    assert ids[5].tolist()[:2] == [4, 3] and ds[5].tolist()[:2] == [1.0, 4.0]
+    assert np.isinf(ds[:, 2]).all()
+    ei, ed = oracle.knn_graph(X, 3)
+    assert ei[2].tolist() == [1, 0, 3] and ed[2, 2] == 64.0
+
+
+@pytest.mark.parametrize("metric", [oracle.L2, oracle.IP])
+def test_knn_partitioned_reduces_to_exact(metric):
+    """m = 1 (one cluster = everything) and overlap = m (every point in
+    every cluster) both reduce to the exact kNN graph (O1, self excluded)."""
+    X = synth.lattice(120, 8, seed=31, metric=metric)
+    ei, ed = oracle.knn_graph(X, 7, metric)
+    for m, c in ((1, 1), (5, 5)):
+        ids, ds = oracle.knn_partitioned(X, 7, m, c, metric)
+        np.testing.assert_array_equal(ids, ei)
+        np.testing.assert_array_equal(ds, ed)
+
+
+def test_knn_partitioned_entries_are_true_neighbours():
+    """Any m: every entry is a real point != self with its exact distance,
+    rows sorted and duplicate-free; recall vs the exact graph rises with overlap."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 1500)
+    ei, _ = oracle.knn_graph(X, 10)
+    rec = []
+    for c in (1, 3):
+        ids, ds = oracle.knn_partitioned(X, 10, 12, c)
+        for i in range(0, 1500, 37):
+            real = ids[i][ids[i] != oracle.SENTINEL]
+            assert i not in real.tolist() and len(set(real.tolist())) == len(real)
+            ref = ((X[real].astype(np.float64) - X[i]) ** 2).sum(1)
+            np.testing.assert_allclose(ds[i, :len(real)], ref, rtol=1e-5)
+            assert np.all(np.diff(ds[i, :len(real)]) >= 0)
+        rec.append(oracle.recall(ids, ei, 10))
+    assert rec[1] > rec[0] and rec[1] > 0.8, rec
