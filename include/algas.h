@@ -345,6 +345,22 @@ int algas_prune(const uint32_t *knn, int64_t n, int32_t knn_degree, int32_t degr
  * (else the first `degree` kNN columns).  out_graph: n x degree. */
 int algas_build_graph(const float *data, int64_t n, int32_t dim, int32_t metric,
                       int32_t knn_degree, int32_t degree, int32_t prune, uint32_t *out_graph);
+/* Partitioned approximate kNN of the base set (DESIGN.md
+ * R30; the paper builds its graphs with CAGRA [25] P:L293 and gives no
+ * build algorithm): centres = rows floor(j*n/n_clusters), j < n_clusters;
+ * every point joins the clusters of its `overlap` nearest centres
+ * ((dist, centre) order); exact kNN (algas_knn, self excluded) inside each
+ * cluster; each point's cluster lists merged by (dist, id), duplicates
+ * dropped, first k kept, padded with (SENTINEL, +inf).  n_clusters = 1 is
+ * the exact kNN.  out_ids/out_dists: n x k, host or device.  EINVAL: n < 2,
+ * k outside [1, 1024], n_clusters outside [1, n], overlap outside
+ * [1, n_clusters], bad dim/metric. */
+int algas_knn_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric, int32_t k,
+                          int32_t n_clusters, int32_t overlap, uint32_t *out_ids, float *out_dists);
+/* algas_build_graph with algas_knn_partitioned as its kNN step. */
+int algas_build_graph_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric,
+                                  int32_t knn_degree, int32_t degree, int32_t prune,
+                                  int32_t n_clusters, int32_t overlap, uint32_t *out_graph);
 
 #if defined(__GNUC__)
 #pragma GCC visibility pop

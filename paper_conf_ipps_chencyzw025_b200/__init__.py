@@ -28,7 +28,7 @@ VISITED_SHARED = 1
 OK, EINVAL, ENOMEM, ECUDA, EAGAIN, ESTATE, ENCCL, EOVERFLOW = 0, -1, -2, -3, -4, -5, -6, -7
 
 __all__ = ["Index", "Server", "Params", "QueryStats", "RunInfo", "lib", "knn", "prune", "build_graph",
-           "merge_topk", "merge_topk_parts", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP", "COSINE"]
+           "merge_topk", "merge_topk_parts", "knn_partitioned", "build_graph_partitioned", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP", "COSINE"]
 
 
 class AlgasError(RuntimeError):
@@ -93,7 +93,7 @@ EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_i
            "algas_server_create", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
-           "algas_build_graph"]
+           "algas_build_graph", "algas_knn_partitioned", "algas_build_graph_partitioned"]
 
 _lock = threading.Lock()
 _lib = None
@@ -147,6 +147,8 @@ def lib(build_if_missing: bool = True):
         L.algas_knn_last_stats.restype = i64
         L.algas_prune.argtypes = [P, i64, i32, i32, P]
         L.algas_build_graph.argtypes = [P, i64, i32, i32, i32, i32, i32, P]
+        L.algas_knn_partitioned.argtypes = [P, i64, i32, i32, i32, i32, i32, P, P]
+        L.algas_build_graph_partitioned.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i32, P]
         _lib = L
         return L
 
@@ -366,6 +368,30 @@ def knn(base, queries, k: int, metric: int = L2, self_base: int = -1):
     dp, _d = _ptr(ds)
     _check(lib().algas_knn(bp, int(base.shape[0]), qp, nq, dim, metric, k, self_base, ip, dp))
     return ids, ds
+
+
+def knn_partitioned(data, k: int, n_clusters: int, overlap: int = 2, metric: int = L2):
+    """Partitioned approximate kNN of the base set (algas_knn_partitioned, R30)."""
+    n, dim = int(data.shape[0]), int(data.shape[1])
+    ids = _alloc_like(data, (n, k), np.uint32, "int32")
+    ds = _alloc_like(data, (n, k), np.float32, "float32")
+    dp, _a = _ptr(data)
+    ip, _c = _ptr(ids)
+    sp, _d = _ptr(ds)
+    _check(lib().algas_knn_partitioned(dp, n, dim, metric, k, n_clusters, overlap, ip, sp))
+    return ids, ds
+
+
+def build_graph_partitioned(data, degree: int, n_clusters: int, overlap: int = 2, knn_degree: int | None = None,
+                            metric: int = L2, prune: bool = True):
+    """algas_build_graph_partitioned: partitioned kNN + the same prune as build_graph."""
+    n, dim = int(data.shape[0]), int(data.shape[1])
+    kd = knn_degree if knn_degree is not None else 2 * degree
+    out = np.empty((n, degree), np.uint32)
+    dp, _a = _ptr(data)
+    _check(lib().algas_build_graph_partitioned(dp, n, dim, metric, kd, degree, 1 if prune else 0, n_clusters,
+                                               overlap, _ptr(out)[0]))
+    return out
 
 
 def knn_last_stats():

@@ -18,6 +18,7 @@
 #include <cmath>
 #include <cstdlib>
 #include <mutex>
+#include <thread>
 #include <cstring>
 #include <vector>
 
@@ -577,6 +578,49 @@ static int knn_screened(const float* X, int64_t n, const float* Q, int64_t nq, i
   return ALGAS_OK;
 }
 
+// rows idx[0..m) of X (d4 float4 per row) into out, one warp per row
+__global__ void gather_rows_kernel(const float4* __restrict__ X, const uint32_t* __restrict__ idx, int64_t m, int d4,
+                                   float4* __restrict__ out) {
+  const int64_t r = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (r >= m) return;
+  const float4* src = X + (int64_t)idx[r] * d4;
+  float4* dst = out + r * d4;
+  for (int i = threadIdx.x & 31; i < d4; i += 32) dst[i] = src[i];
+}
+
+static int gather_rows(const float* X, const uint32_t* d_idx, int64_t m, int dim, float* out) {
+  if (m == 0) return ALGAS_OK;
+  gather_rows_kernel<<<(unsigned)((m + 7) / 8), 256>>>(reinterpret_cast<const float4*>(X), d_idx, m, dim / 4,
+                                                       reinterpret_cast<float4*>(out));
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  return ALGAS_OK;
+}
+
+// kNN lists (device, n x K, sorted rows, no self) -> graph (R24)
+static int graph_from_knn(const uint32_t* dk, int64_t n, int K, int degree, int prune, uint32_t* out_graph) {
+  const int R = std::min(degree, K);
+  std::vector<uint32_t> tmp;
+  int rc;
+  if (prune) {
+    if (R == degree) return algas_prune(dk, n, K, R, out_graph);
+    tmp.resize((size_t)n * R);
+    if ((rc = algas_prune(dk, n, K, R, tmp.data()))) return rc;
+  } else {
+    tmp.resize((size_t)n * R);
+    ALGAS_CUDA_TRY(cudaMemcpy2D(tmp.data(), (size_t)R * 4, dk, (size_t)K * 4, (size_t)R * 4, (size_t)n,
+                                cudaMemcpyDeviceToHost));
+    if (R == degree) {
+      ALGAS_CUDA_TRY(cudaMemcpy(out_graph, tmp.data(), tmp.size() * 4, cudaMemcpyDefault));
+      return ALGAS_OK;
+    }
+  }
+  // fewer than `degree` neighbours exist: pad rows with sentinels
+  std::vector<uint32_t> full((size_t)n * degree, kSentinel);
+  for (int64_t i = 0; i < n; ++i) std::copy(tmp.begin() + i * R, tmp.begin() + (i + 1) * R, full.begin() + i * degree);
+  ALGAS_CUDA_TRY(cudaMemcpy(out_graph, full.data(), full.size() * 4, cudaMemcpyDefault));
+  return ALGAS_OK;
+}
+
 }  // namespace algas
 
 using namespace algas;
@@ -677,36 +721,119 @@ int algas_build_graph(const float* data, int64_t n, int32_t dim, int32_t metric,
   if (!data || !out_graph || n < 2 || knn_degree < degree || degree < 1)
     return set_error(ALGAS_EINVAL, "algas_build_graph: bad arguments");
   const int K = (int)std::min<int64_t>(knn_degree, n - 1);
-  const int R = std::min(degree, K);
-  uint32_t* dk = nullptr;
-  float* dd = nullptr;
-  ALGAS_CUDA_TRY(cudaMalloc(&dk, (size_t)n * K * 4));
-  Dev guard_k;
-  guard_k.p = dk;
-  ALGAS_CUDA_TRY(cudaMalloc(&dd, (size_t)n * K * 4));
-  Dev guard_d;
-  guard_d.p = dd;
-  int rc = algas_knn(data, n, data, n, dim, metric, K, 0, dk, dd);
+  Dev guard_k, guard_d;
+  ALGAS_CUDA_TRY(cudaMalloc(&guard_k.p, (size_t)n * K * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&guard_d.p, (size_t)n * K * 4));
+  int rc = algas_knn(data, n, data, n, dim, metric, K, 0, (uint32_t*)guard_k.p, (float*)guard_d.p);
   if (rc) return rc;
-  std::vector<uint32_t> tmp;
-  if (prune) {
-    if (R == degree) return algas_prune(dk, n, K, R, out_graph);
-    tmp.resize((size_t)n * R);
-    if ((rc = algas_prune(dk, n, K, R, tmp.data()))) return rc;
-  } else {
-    tmp.resize((size_t)n * R);
-    ALGAS_CUDA_TRY(cudaMemcpy2D(tmp.data(), (size_t)R * 4, dk, (size_t)K * 4, (size_t)R * 4, (size_t)n,
-                                cudaMemcpyDeviceToHost));
-    if (R == degree) {
-      ALGAS_CUDA_TRY(cudaMemcpy(out_graph, tmp.data(), tmp.size() * 4, cudaMemcpyDefault));
-      return ALGAS_OK;
+  return graph_from_knn((const uint32_t*)guard_k.p, n, K, degree, prune, out_graph);
+}
+
+// Partitioned approximate kNN (R30): sampled
+// centres, each point assigned to its `overlap` nearest centres, exact kNN
+// inside every cluster (algas_knn, self excluded), per-point merge of its
+// cluster lists by (dist, id) with duplicates removed.
+int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t k, int32_t n_clusters,
+                          int32_t overlap, uint32_t* out_ids, float* out_dists) {
+  if (!data || !out_ids || !out_dists || n < 2 || n >= (1LL << 31) || dim < 4 || dim % 4 != 0 || k < 1 ||
+      k > 1024 || n_clusters < 1 || n_clusters > n || overlap < 1 || overlap > n_clusters ||
+      (metric != ALGAS_L2 && metric != ALGAS_IP))
+    return set_error(ALGAS_EINVAL, "algas_knn_partitioned: bad arguments");
+  Dev hx;
+  const float* X = nullptr;
+  int rc;
+  if ((rc = to_device(data, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
+  const int64_t m = n_clusters;
+  const int c = overlap;
+  // 1. centres: rows floor(j n / m), j < m
+  std::vector<uint32_t> cid(m);
+  for (int64_t j = 0; j < m; ++j) cid[j] = (uint32_t)((j * n) / m);
+  Dev hcid, hC, hmem, hB;
+  ALGAS_CUDA_TRY(cudaMalloc(&hcid.p, (size_t)m * 4));
+  ALGAS_CUDA_TRY(cudaMemcpy(hcid.p, cid.data(), (size_t)m * 4, cudaMemcpyHostToDevice));
+  ALGAS_CUDA_TRY(cudaMalloc(&hC.p, (size_t)m * dim * 4));
+  if ((rc = gather_rows(X, (const uint32_t*)hcid.p, m, dim, (float*)hC.p))) return rc;
+  // 2. assignment: the c nearest centres of every point, (dist, centre) order
+  std::vector<uint32_t> asg((size_t)n * c);
+  std::vector<float> asgd((size_t)n * c);
+  if ((rc = algas_knn((const float*)hC.p, m, X, n, dim, metric, c, -1, asg.data(), asgd.data()))) return rc;
+  // 3. members of each cluster, ascending global id
+  std::vector<int64_t> start(m + 1, 0);
+  for (size_t e = 0; e < asg.size(); ++e) ++start[asg[e] + 1];
+  for (int64_t j = 0; j < m; ++j) start[j + 1] += start[j];
+  std::vector<uint32_t> mem(asg.size());
+  {
+    std::vector<int64_t> fill(start.begin(), start.end() - 1);
+    for (int64_t i = 0; i < n; ++i)
+      for (int r = 0; r < c; ++r) {
+        const uint32_t j = asg[(size_t)i * c + r];
+        mem[fill[j]++] = (uint32_t)i;
+      }
+  }
+  int64_t smax = 0;
+  for (int64_t j = 0; j < m; ++j) smax = std::max(smax, start[j + 1] - start[j]);
+  // 4. exact kNN inside each cluster (rows gathered contiguously; local id
+  //    order == global id order, so (dist, id) ties resolve as globally)
+  ALGAS_CUDA_TRY(cudaMalloc(&hmem.p, std::max<size_t>(mem.size() * 4, 16)));
+  ALGAS_CUDA_TRY(cudaMemcpy(hmem.p, mem.data(), mem.size() * 4, cudaMemcpyHostToDevice));
+  ALGAS_CUDA_TRY(cudaMalloc(&hB.p, (size_t)smax * dim * 4));
+  std::vector<uint32_t> cand((size_t)n * c * k, kSentinel);
+  std::vector<float> candd((size_t)n * c * k, INFINITY);
+  std::vector<uint32_t> li;
+  std::vector<float> ld;
+  for (int64_t j = 0; j < m; ++j) {
+    const int64_t sj = start[j + 1] - start[j];
+    if (sj < 2) continue;
+    const int kj = (int)std::min<int64_t>(k, sj - 1);
+    if ((rc = gather_rows(X, (const uint32_t*)hmem.p + start[j], sj, dim, (float*)hB.p))) return rc;
+    li.resize((size_t)sj * kj);
+    ld.resize((size_t)sj * kj);
+    if ((rc = algas_knn((const float*)hB.p, sj, (const float*)hB.p, sj, dim, metric, kj, 0, li.data(), ld.data())))
+      return rc;
+    // scatter into each member's candidate block for this cluster
+    for (int64_t t = 0; t < sj; ++t) {
+      const uint32_t i = mem[start[j] + t];
+      int r = 0;
+      while (asg[(size_t)i * c + r] != (uint32_t)j) ++r;
+      uint32_t* ci = cand.data() + ((size_t)i * c + r) * k;
+      float* cd = candd.data() + ((size_t)i * c + r) * k;
+      for (int e = 0; e < kj; ++e) {
+        const uint32_t l = li[(size_t)t * kj + e];
+        ci[e] = l == kSentinel ? kSentinel : mem[start[j] + l];
+        cd[e] = ld[(size_t)t * kj + e];
+      }
     }
   }
-  // n - 1 < degree: pad rows with sentinels
-  std::vector<uint32_t> full((size_t)n * degree, kSentinel);
-  for (int64_t i = 0; i < n; ++i) std::copy(tmp.begin() + i * R, tmp.begin() + (i + 1) * R, full.begin() + i * degree);
-  ALGAS_CUDA_TRY(cudaMemcpy(out_graph, full.data(), full.size() * 4, cudaMemcpyDefault));
+  // 5. per-point merge (dist, id), duplicates dropped, padded to k
+  std::vector<uint32_t> oi((size_t)n * k);
+  std::vector<float> od((size_t)n * k);
+  const int nth = (int)std::max<unsigned>(1, std::min<unsigned>(16, std::thread::hardware_concurrency()));
+  std::vector<std::thread> th;
+  for (int w = 0; w < nth; ++w)
+    th.emplace_back([&, w] {
+      for (int64_t i = w; i < n; i += nth)
+        algas_merge_topk(cand.data() + (size_t)i * c * k, candd.data() + (size_t)i * c * k, c * k, k,
+                         oi.data() + (size_t)i * k, od.data() + (size_t)i * k);
+    });
+  for (auto& t : th) t.join();
+  ALGAS_CUDA_TRY(cudaMemcpy(out_ids, oi.data(), oi.size() * 4, cudaMemcpyDefault));
+  ALGAS_CUDA_TRY(cudaMemcpy(out_dists, od.data(), od.size() * 4, cudaMemcpyDefault));
   return ALGAS_OK;
+}
+
+int algas_build_graph_partitioned(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t knn_degree,
+                                  int32_t degree, int32_t prune, int32_t n_clusters, int32_t overlap,
+                                  uint32_t* out_graph) {
+  if (!data || !out_graph || n < 2 || knn_degree < degree || degree < 1)
+    return set_error(ALGAS_EINVAL, "algas_build_graph_partitioned: bad arguments");
+  const int K = (int)std::min<int64_t>(knn_degree, n - 1);
+  Dev guard_k, guard_d;
+  ALGAS_CUDA_TRY(cudaMalloc(&guard_k.p, (size_t)n * K * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&guard_d.p, (size_t)n * K * 4));
+  int rc = algas_knn_partitioned(data, n, dim, metric, K, n_clusters, overlap, (uint32_t*)guard_k.p,
+                                 (float*)guard_d.p);
+  if (rc) return rc;
+  return graph_from_knn((const uint32_t*)guard_k.p, n, K, degree, prune, out_graph);
 }
 
 }  // extern "C"
