@@ -357,7 +357,9 @@ int algas_build_graph(const float *data, int64_t n, int32_t dim, int32_t metric,
  * [1, n_clusters], bad dim/metric. */
 int algas_knn_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric, int32_t k,
                           int32_t n_clusters, int32_t overlap, uint32_t *out_ids, float *out_dists);
-/* algas_build_graph with algas_knn_partitioned as its kNN step. */
+/* algas_build_graph with algas_knn_partitioned as its kNN step; rows the
+ * partition left short (clusters of <= knn_degree points) are completed
+ * with the exact kNN of those rows over the whole set before the prune. */
 int algas_build_graph_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric,
                                   int32_t knn_degree, int32_t degree, int32_t prune,
                                   int32_t n_clusters, int32_t overlap, uint32_t *out_graph);

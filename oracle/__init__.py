@@ -150,7 +150,8 @@ def knn_graph(X, K: int, metric: int = L2):
 def knn_partitioned(X, k: int, n_clusters: int, overlap: int, metric: int = L2):
     """Partitioned approximate kNN graph (R30), step by
     step: (1) centres = rows floor(j n / m); (2) each point's `overlap`
-    nearest centres (O1 over the centres); (3) cluster members in ascending
+    nearest centres with room (capacity ceil(2 c n / m), n if 4c >= m), after
+    8 Lloyd iterations on a row sample; (3) cluster members in ascending
     id; (4) O1 inside each cluster, self excluded, k_j = min(k, s_j - 1);
     (5) per point: its cluster lists merged by (dist, id), repeated ids
     dropped, first k (orc_merge_topk).  Parity unpinned by the paper (it
@@ -159,8 +160,38 @@ def knn_partitioned(X, k: int, n_clusters: int, overlap: int, metric: int = L2):
     X = _f32(X)
     n = X.shape[0]
     m, c = n_clusters, overlap
-    centres = X[[(j * n) // m for j in range(m)]]
-    asg, _ = brute_force(centres, X, c, metric)
+    centres = X[[(j * n) // m for j in range(m)]].copy()
+    # (1b) 8 Lloyd iterations on the sample rows floor(i n / ns), ns = min(n, 32 m):
+    # nearest centre (O1), centre = mean of its rows (double, row order), empty stays
+    if m > 1:
+        ns = min(n, 32 * m)
+        S = X[[(i * n) // ns for i in range(ns)]]
+        for _ in range(8):
+            a1, _d = brute_force(centres, S, 1, metric)
+            for j in range(m):
+                rows = [i for i in range(ns) if a1[i, 0] == j]
+                if rows:
+                    acc = np.zeros(X.shape[1], np.float64)
+                    for i in rows:
+                        acc += S[i].astype(np.float64)
+                    centres[j] = (acc / len(rows)).astype(np.float32)
+    # (2) capacity-constrained: P nearest centres per point; points in id
+    # order take the first c with room, else the lowest-index ones with room
+    P = min(m, 4 * c + 4)
+    pref, _ = brute_force(centres, X, P, metric)
+    cap = n if 4 * c >= m else -(-2 * c * n // m)
+    load = [0] * m
+    asg = np.zeros((n, c), np.int64)
+    for i in range(n):
+        got = []
+        for j in list(pref[i]) + list(range(m)):
+            if len(got) == c:
+                break
+            if load[j] < cap and j not in got:
+                got.append(int(j))
+                load[j] += 1
+        assert len(got) == c
+        asg[i] = got
     cand_i = np.full((n, c, k), SENTINEL, np.uint32)
     cand_d = np.full((n, c, k), np.inf, np.float32)
     for j in range(m):

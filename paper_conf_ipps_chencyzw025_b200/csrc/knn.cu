@@ -15,7 +15,9 @@
 #include <cublas_v2.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 #include <mutex>
 #include <thread>
@@ -729,6 +731,8 @@ int algas_build_graph(const float* data, int64_t n, int32_t dim, int32_t metric,
   return graph_from_knn((const uint32_t*)guard_k.p, n, K, degree, prune, out_graph);
 }
 
+constexpr int kLloyd = 8;
+
 // Partitioned approximate kNN (R30): sampled
 // centres, each point assigned to its `overlap` nearest centres, exact kNN
 // inside every cluster (algas_knn, self excluded), per-point merge of its
@@ -739,6 +743,15 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
       k > 1024 || n_clusters < 1 || n_clusters > n || overlap < 1 || overlap > n_clusters ||
       (metric != ALGAS_L2 && metric != ALGAS_IP))
     return set_error(ALGAS_EINVAL, "algas_knn_partitioned: bad arguments");
+  static const bool trace = getenv("ALGAS_TRACE") != nullptr;
+  auto t_last = std::chrono::steady_clock::now();
+  auto phase = [&](const char* name) {
+    if (!trace) return;
+    cudaDeviceSynchronize();
+    const auto t = std::chrono::steady_clock::now();
+    fprintf(stderr, "[algas_knn_partitioned] %s %.3f s\n", name, std::chrono::duration<double>(t - t_last).count());
+    t_last = t;
+  };
   Dev hx;
   const float* X = nullptr;
   int rc;
@@ -753,10 +766,74 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
   ALGAS_CUDA_TRY(cudaMemcpy(hcid.p, cid.data(), (size_t)m * 4, cudaMemcpyHostToDevice));
   ALGAS_CUDA_TRY(cudaMalloc(&hC.p, (size_t)m * dim * 4));
   if ((rc = gather_rows(X, (const uint32_t*)hcid.p, m, dim, (float*)hC.p))) return rc;
-  // 2. assignment: the c nearest centres of every point, (dist, centre) order
+  // 1b. kLloyd Lloyd iterations on the sample rows floor(i n / ns), ns =
+  //     min(n, 32 m): each sample row to its nearest centre, centre = mean of
+  //     its rows (double sums in row order, rounded to fp32; an empty
+  //     centre stays).  Moves centres off the high-dimensional hubs.
+  if (m > 1) {
+    const int64_t ns = std::min<int64_t>(n, 32 * m);
+    std::vector<uint32_t> sid(ns);
+    for (int64_t i = 0; i < ns; ++i) sid[i] = (uint32_t)((i * n) / ns);
+    Dev hsid, hS;
+    ALGAS_CUDA_TRY(cudaMalloc(&hsid.p, (size_t)ns * 4));
+    ALGAS_CUDA_TRY(cudaMemcpy(hsid.p, sid.data(), (size_t)ns * 4, cudaMemcpyHostToDevice));
+    ALGAS_CUDA_TRY(cudaMalloc(&hS.p, (size_t)ns * dim * 4));
+    if ((rc = gather_rows(X, (const uint32_t*)hsid.p, ns, dim, (float*)hS.p))) return rc;
+    std::vector<float> S((size_t)ns * dim), C((size_t)m * dim);
+    ALGAS_CUDA_TRY(cudaMemcpy(S.data(), hS.p, S.size() * 4, cudaMemcpyDeviceToHost));
+    ALGAS_CUDA_TRY(cudaMemcpy(C.data(), hC.p, C.size() * 4, cudaMemcpyDeviceToHost));
+    std::vector<uint32_t> a1(ns);
+    std::vector<float> a1d(ns);
+    std::vector<double> acc((size_t)m * dim);
+    std::vector<int64_t> cnt(m);
+    for (int it = 0; it < kLloyd; ++it) {
+      if ((rc = algas_knn((const float*)hC.p, m, (const float*)hS.p, ns, dim, metric, 1, -1, a1.data(), a1d.data())))
+        return rc;
+      std::fill(acc.begin(), acc.end(), 0.0);
+      std::fill(cnt.begin(), cnt.end(), 0);
+      for (int64_t i = 0; i < ns; ++i) {
+        const uint32_t j = a1[i];
+        ++cnt[j];
+        for (int t = 0; t < dim; ++t) acc[(size_t)j * dim + t] += (double)S[(size_t)i * dim + t];
+      }
+      for (int64_t j = 0; j < m; ++j)
+        if (cnt[j] > 0)
+          for (int t = 0; t < dim; ++t) C[(size_t)j * dim + t] = (float)(acc[(size_t)j * dim + t] / (double)cnt[j]);
+      ALGAS_CUDA_TRY(cudaMemcpy(hC.p, C.data(), C.size() * 4, cudaMemcpyHostToDevice));
+    }
+  }
+  // 2. assignment under a capacity (hub centres of high-dimensional data
+  //    would otherwise take half the points): every point's P nearest
+  //    centres in (dist, centre) order; points in id order take the first c
+  //    of them that still have room (cap = ceil(2 c n / m), or n when
+  //    4 c >= m), else the
+  //    lowest-index centres with room (R30)
+  const int P = (int)std::min<int64_t>(m, 4 * c + 4);
+  std::vector<uint32_t> pref((size_t)n * P);
+  std::vector<float> prefd((size_t)n * P);
+  if ((rc = algas_knn((const float*)hC.p, m, X, n, dim, metric, P, -1, pref.data(), prefd.data()))) return rc;
   std::vector<uint32_t> asg((size_t)n * c);
-  std::vector<float> asgd((size_t)n * c);
-  if ((rc = algas_knn((const float*)hC.p, m, X, n, dim, metric, c, -1, asg.data(), asgd.data()))) return rc;
+  {
+    const int64_t cap = 4 * (int64_t)c >= m ? n : (2 * (int64_t)c * n + m - 1) / m;
+    std::vector<int64_t> load(m, 0);
+    int64_t low = 0;  // every centre below `low` is full
+    for (int64_t i = 0; i < n; ++i) {
+      uint32_t* a = asg.data() + (size_t)i * c;
+      int got = 0;
+      for (int e = 0; e < P && got < c; ++e) {
+        const uint32_t j = pref[(size_t)i * P + e];
+        if (load[j] < cap) { a[got++] = j; ++load[j]; }
+      }
+      for (int64_t j = low; got < c && j < m; ++j) {
+        if (load[j] >= cap) { if (j == low) ++low; continue; }
+        bool dup = false;
+        for (int r = 0; r < got; ++r) dup |= a[r] == (uint32_t)j;
+        if (!dup) { a[got++] = (uint32_t)j; ++load[j]; }
+      }
+      if (got < c) return set_error(ALGAS_ESTATE, "algas_knn_partitioned: assignment ran out of room");
+    }
+  }
+  phase("assign");
   // 3. members of each cluster, ascending global id
   std::vector<int64_t> start(m + 1, 0);
   for (size_t e = 0; e < asg.size(); ++e) ++start[asg[e] + 1];
@@ -777,6 +854,7 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
   ALGAS_CUDA_TRY(cudaMalloc(&hmem.p, std::max<size_t>(mem.size() * 4, 16)));
   ALGAS_CUDA_TRY(cudaMemcpy(hmem.p, mem.data(), mem.size() * 4, cudaMemcpyHostToDevice));
   ALGAS_CUDA_TRY(cudaMalloc(&hB.p, (size_t)smax * dim * 4));
+  phase("members");
   std::vector<uint32_t> cand((size_t)n * c * k, kSentinel);
   std::vector<float> candd((size_t)n * c * k, INFINITY);
   std::vector<uint32_t> li;
@@ -788,8 +866,12 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
     if ((rc = gather_rows(X, (const uint32_t*)hmem.p + start[j], sj, dim, (float*)hB.p))) return rc;
     li.resize((size_t)sj * kj);
     ld.resize((size_t)sj * kj);
+    const auto tc0 = std::chrono::steady_clock::now();
     if ((rc = algas_knn((const float*)hB.p, sj, (const float*)hB.p, sj, dim, metric, kj, 0, li.data(), ld.data())))
       return rc;
+    if (trace && j < 4)
+      fprintf(stderr, "[algas_knn_partitioned] cluster %lld size %lld knn %.4f s\n", (long long)j, (long long)sj,
+              std::chrono::duration<double>(std::chrono::steady_clock::now() - tc0).count());
     // scatter into each member's candidate block for this cluster
     for (int64_t t = 0; t < sj; ++t) {
       const uint32_t i = mem[start[j] + t];
@@ -804,6 +886,13 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
       }
     }
   }
+  if (trace) {
+    int64_t fb = 0;
+    const int64_t sc = algas_knn_last_stats(&fb);
+    fprintf(stderr, "[algas_knn_partitioned] m=%lld largest cluster %lld, rows screened %lld, fallback %lld\n",
+            (long long)m, (long long)smax, (long long)sc, (long long)fb);
+  }
+  phase("clusters");
   // 5. per-point merge (dist, id), duplicates dropped, padded to k
   std::vector<uint32_t> oi((size_t)n * k);
   std::vector<float> od((size_t)n * k);
@@ -816,6 +905,7 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
                          oi.data() + (size_t)i * k, od.data() + (size_t)i * k);
     });
   for (auto& t : th) t.join();
+  phase("merge");
   ALGAS_CUDA_TRY(cudaMemcpy(out_ids, oi.data(), oi.size() * 4, cudaMemcpyDefault));
   ALGAS_CUDA_TRY(cudaMemcpy(out_dists, od.data(), od.size() * 4, cudaMemcpyDefault));
   return ALGAS_OK;
@@ -833,6 +923,34 @@ int algas_build_graph_partitioned(const float* data, int64_t n, int32_t dim, int
   int rc = algas_knn_partitioned(data, n, dim, metric, K, n_clusters, overlap, (uint32_t*)guard_k.p,
                                  (float*)guard_d.p);
   if (rc) return rc;
+  // rows the partition left short (clusters of <= K points) are completed by
+  // the exact kNN of those rows over the whole set (the prune needs full rows)
+  std::vector<uint32_t> hk((size_t)n * K);
+  ALGAS_CUDA_TRY(cudaMemcpy(hk.data(), guard_k.p, hk.size() * 4, cudaMemcpyDeviceToHost));
+  std::vector<uint32_t> shortr;
+  for (int64_t i = 0; i < n; ++i)
+    if (hk[(size_t)i * K + K - 1] == kSentinel) shortr.push_back((uint32_t)i);
+  if (!shortr.empty()) {
+    Dev hx, hs, hq;
+    const float* X = nullptr;
+    if ((rc = to_device(data, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
+    const int64_t ns = (int64_t)shortr.size();
+    const int K1 = (int)std::min<int64_t>(K + 1, n);
+    ALGAS_CUDA_TRY(cudaMalloc(&hs.p, (size_t)ns * 4));
+    ALGAS_CUDA_TRY(cudaMemcpy(hs.p, shortr.data(), (size_t)ns * 4, cudaMemcpyHostToDevice));
+    ALGAS_CUDA_TRY(cudaMalloc(&hq.p, (size_t)ns * dim * 4));
+    if ((rc = gather_rows(X, (const uint32_t*)hs.p, ns, dim, (float*)hq.p))) return rc;
+    std::vector<uint32_t> ei((size_t)ns * K1);
+    std::vector<float> ed((size_t)ns * K1);
+    if ((rc = algas_knn(X, n, (const float*)hq.p, ns, dim, metric, K1, -1, ei.data(), ed.data()))) return rc;
+    for (int64_t t = 0; t < ns; ++t) {
+      uint32_t* row = hk.data() + (size_t)shortr[t] * K;
+      int o = 0;
+      for (int e = 0; e < K1 && o < K; ++e)
+        if (ei[(size_t)t * K1 + e] != shortr[t]) row[o++] = ei[(size_t)t * K1 + e];
+    }
+    ALGAS_CUDA_TRY(cudaMemcpy(guard_k.p, hk.data(), hk.size() * 4, cudaMemcpyHostToDevice));
+  }
   return graph_from_knn((const uint32_t*)guard_k.p, n, K, degree, prune, out_graph);
 }
 

@@ -1,0 +1,74 @@
+"""Graph-build timing: exact kNN + prune vs the partitioned
+build (algas_build_graph_partitioned, R30) on a workload's
+synthetic base set; kNN-graph recall of the partitioned lists on a sample of
+rows and search recall@k of both graphs at one fixed search point.
+
+    python scripts/build_timing.py C2 --clusters 64 128 --overlap 2
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+
+def main():
+    import torch
+
+    import paper_conf_ipps_chencyzw025_b200 as algas
+    import synth
+    ap = argparse.ArgumentParser()
+    ap.add_argument("workload", default="C2")
+    ap.add_argument("--clusters", type=int, nargs="+", default=[64, 128])
+    ap.add_argument("--overlap", type=int, nargs="+", default=[2])
+    ap.add_argument("--nq", type=int, default=2000)
+    a = ap.parse_args()
+    w = synth.WORKLOADS[a.workload]
+    X = synth.base_vectors(w)
+    Q = synth.query_vectors(w, a.nq)
+    Xd = torch.from_numpy(X).cuda()
+    Qd = torch.from_numpy(Q).cuda()
+    ti, _ = algas.knn(Xd, Qd, w.k, w.metric)
+    ti = ti.cpu().numpy().view(np.uint32)
+    sample = np.arange(0, w.n, max(1, w.n // 2000))
+    se, _ = algas.knn(Xd, Xd[torch.from_numpy(sample).cuda()], w.knn_degree, w.metric)
+    se = se.cpu().numpy().view(np.uint32)  # includes self at column 0 (self_base not applied)
+    p = algas.default_params(k=w.k, itopk=64, width=8, offset_beam=1, n_seeds=32, ctas_per_query=1,
+                             threads_per_cta=512, seed=3)
+    out = {"workload": w.name, "n": w.n, "dim": w.dim, "knn_degree": w.knn_degree, "degree": w.degree}
+    torch.cuda.synchronize()
+    t0 = time.time()
+    ge = algas.build_graph(Xd, w.degree, knn_degree=w.knn_degree, metric=w.metric)
+    torch.cuda.synchronize()
+    out["exact_build_s"] = time.time() - t0
+    r = algas.Index(Xd, ge, w.metric).search(Q, params=p)
+    out["exact_search_recall"] = float((r["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
+    out["partitioned"] = []
+    for m in a.clusters:
+        for c in a.overlap:
+            torch.cuda.synchronize()
+            t0 = time.time()
+            ids, _ = algas.knn_partitioned(Xd, w.knn_degree, m, c, w.metric)
+            torch.cuda.synchronize()
+            t_knn = time.time() - t0
+            ids = ids.cpu().numpy().view(np.uint32)
+            hit = np.mean([len(set(ids[i].tolist()) & set(se[j, 1:].tolist())) / (w.knn_degree - 1)
+                           for j, i in enumerate(sample)])
+            t0 = time.time()
+            gp = algas.build_graph_partitioned(Xd, w.degree, m, c, knn_degree=w.knn_degree, metric=w.metric)
+            torch.cuda.synchronize()
+            t_build = time.time() - t0
+            rp = algas.Index(Xd, gp, w.metric).search(Q, params=p)
+            rec = float((rp["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
+            out["partitioned"].append({"clusters": m, "overlap": c, "knn_s": t_knn, "build_s": t_build,
+                                       "knn_graph_recall_sample": float(hit), "search_recall": rec})
+            print(json.dumps(out["partitioned"][-1]), flush=True)
+    print(json.dumps(out))
+
+
+if __name__ == "__main__":
+    main()

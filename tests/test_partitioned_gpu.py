@@ -57,3 +57,16 @@ def test_knn_partitioned_rejects():
     for m, c in ((0, 1), (11, 1), (4, 5)):
         with pytest.raises(algas.AlgasError):
             algas.knn_partitioned(X, 3, m, c)
+
+
+def test_build_graph_partitioned_short_clusters_completed():
+    """Many clusters with overlap 1: some hold <= knn_degree points, their
+    rows come back short from algas_knn_partitioned; the graph builder
+    completes them (no sentinel reaches the prune, every row is full)."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 3000)
+    ki, _ = algas.knn_partitioned(X, 48, 200, 1)
+    assert (ki == algas.SENTINEL).any()
+    g = algas.build_graph_partitioned(X, 24, n_clusters=200, overlap=1, knn_degree=48)
+    assert (g < X.shape[0]).mean() > 0.999
+    assert not (g == np.arange(X.shape[0])[:, None]).any()
