@@ -16,6 +16,11 @@ Parity status per function:
     (== O1), hand-worked path / star / disconnected graphs, w=1 == off>=L.
   * orc_merge_topk (A9)                    pinned: brute-force sort + dedupe.
   * orc_tuner_*                            pinned: Table II closed form.
+  * COSINE metric (R29)                     pinned: hand values, angle closed
+    form, unit-circle ordering with random radii.
+  * knn_partitioned (f4, R30)              parity unpinned by the paper (no
+    build algorithm in it); pinned by m = 1 / overlap = m == O1 and a
+    hand-worked 1-d example.
   * orc_prune (K10)                        parity unpinned by the paper (the
     CAGRA algorithm is only cited); pinned by a hand-worked
     example and invariants.
