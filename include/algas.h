@@ -328,7 +328,8 @@ int algas_tune(const algas_device_props *props, int32_t slots, int32_t dim, int3
  * screen candidates with tensor-core 3xTF32 GEMMs (cuBLAS), re-rank them
  * with the exact fp32 direct-form distance and certify each query (bound on
  * the screening error), redoing uncertified queries on the direct CUDA-core
- * path; ALGAS_KNN_MODE=direct|screened forces one.  Errors: EINVAL on bad
+ * path; ALGAS_KNN_MODE=direct|screened forces one.  metric COSINE: IP on
+ * unit-row copies of base and queries (R29).  Errors: EINVAL on bad
  * arguments, ENOMEM/ECUDA from the device. */
 int algas_knn(const float *base, int64_t n, const float *queries, int64_t nq, int32_t dim,
               int32_t metric, int32_t k, int64_t self_base, uint32_t *out_ids, float *out_dists);

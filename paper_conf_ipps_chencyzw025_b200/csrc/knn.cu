@@ -580,6 +580,27 @@ static int knn_screened(const float* X, int64_t n, const float* Q, int64_t nq, i
   return ALGAS_OK;
 }
 
+// COSINE (R29): dst row = src row / |src row| (fp32; a zero row stays 0), one warp per row
+__global__ void normalize_copy_kernel(const float4* __restrict__ src, int64_t n, int d4, float4* __restrict__ dst) {
+  const int64_t r = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (r >= n) return;
+  const int lane = threadIdx.x & 31;
+  const float4* a = src + r * d4;
+  float4* b = dst + r * d4;
+  float ss = 0.f;
+  for (int i = lane; i < d4; i += 32) {
+    const float4 v = a[i];
+    ss = fmaf(v.x, v.x, fmaf(v.y, v.y, fmaf(v.z, v.z, fmaf(v.w, v.w, ss))));
+  }
+  for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+  const float inv = ss > 0.f ? 1.0f / sqrtf(ss) : 1.0f;
+  for (int i = lane; i < d4; i += 32) {
+    float4 v = a[i];
+    v.x *= inv; v.y *= inv; v.z *= inv; v.w *= inv;
+    b[i] = v;
+  }
+}
+
 // rows idx[0..m) of X (d4 float4 per row) into out, one warp per row
 __global__ void gather_rows_kernel(const float4* __restrict__ X, const uint32_t* __restrict__ idx, int64_t m, int d4,
                                    float4* __restrict__ out) {
@@ -632,14 +653,30 @@ extern "C" {
 int algas_knn(const float* base, int64_t n, const float* queries, int64_t nq, int32_t dim, int32_t metric, int32_t k,
               int64_t self_base, uint32_t* out_ids, float* out_dists) {
   if (!base || !queries || !out_ids || !out_dists || n < 1 || n >= (1LL << 31) || nq < 0 || dim < 4 ||
-      dim % 4 != 0 || k < 1 || k > 1024 || (metric != ALGAS_L2 && metric != ALGAS_IP))
+      dim % 4 != 0 || k < 1 || k > 1024 || (metric != ALGAS_L2 && metric != ALGAS_IP && metric != ALGAS_COSINE))
     return set_error(ALGAS_EINVAL, "algas_knn: bad arguments");
   if (nq == 0) return ALGAS_OK;
-  Dev hx, hq;
+  Dev hx, hq, hxn, hqn;
   const float *X = nullptr, *Q = nullptr;
   int rc;
   if ((rc = to_device(base, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
   if ((rc = to_device(queries, (size_t)nq * dim * 4, hq, (const void**)&Q))) return rc;
+  if (metric == ALGAS_COSINE) {
+    // IP on unit copies of both sides (R29)
+    const bool same = X == Q && n == nq;
+    ALGAS_CUDA_TRY(cudaMalloc(&hxn.p, (size_t)n * dim * 4));
+    normalize_copy_kernel<<<(unsigned)((n + 7) / 8), 256>>>(reinterpret_cast<const float4*>(X), n, dim / 4,
+                                                            reinterpret_cast<float4*>(hxn.p));
+    if (!same) {
+      ALGAS_CUDA_TRY(cudaMalloc(&hqn.p, (size_t)nq * dim * 4));
+      normalize_copy_kernel<<<(unsigned)((nq + 7) / 8), 256>>>(reinterpret_cast<const float4*>(Q), nq, dim / 4,
+                                                               reinterpret_cast<float4*>(hqn.p));
+    }
+    ALGAS_CUDA_TRY(cudaGetLastError());
+    X = (const float*)hxn.p;
+    Q = same ? X : (const float*)hqn.p;
+    metric = ALGAS_IP;
+  }
   // path: tensor-core screen + exact rerank + certificate (default for large
   // problems), or the direct CUDA-core path; ALGAS_KNN_MODE=direct|screened
   const char* env = getenv("ALGAS_KNN_MODE");
@@ -741,7 +778,7 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
                           int32_t overlap, uint32_t* out_ids, float* out_dists) {
   if (!data || !out_ids || !out_dists || n < 2 || n >= (1LL << 31) || dim < 4 || dim % 4 != 0 || k < 1 ||
       k > 1024 || n_clusters < 1 || n_clusters > n || overlap < 1 || overlap > n_clusters ||
-      (metric != ALGAS_L2 && metric != ALGAS_IP))
+      (metric != ALGAS_L2 && metric != ALGAS_IP && metric != ALGAS_COSINE))
     return set_error(ALGAS_EINVAL, "algas_knn_partitioned: bad arguments");
   static const bool trace = getenv("ALGAS_TRACE") != nullptr;
   auto t_last = std::chrono::steady_clock::now();

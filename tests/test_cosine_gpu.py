@@ -119,3 +119,17 @@ def test_cosine_built_graph_and_zero_query():
     _check(X, Q, r["ids"], r["dists"])
     z = idx.search(np.zeros((2, X.shape[1]), np.float32), params=p)
     assert np.all(z["ids"] != SENT) and np.all(z["dists"] == 0.0)
+
+
+def test_cosine_knn_matches_oracle():
+    """algas_knn(COSINE) (IP on unit copies) against the oracle's fp64 cosine
+    brute force: ids equal except near-ties, distances within 2e-5."""
+    X, Q, G, ti = cosine_case()
+    gi, gd = algas.knn(X, Q, 10, algas.COSINE)
+    oi, od = oracle.brute_force(X, Q, 10, oracle.COSINE)
+    assert (gi == oi).mean() > 0.99
+    np.testing.assert_allclose(gd, od, atol=2e-5)
+    si, sd = algas.knn(X, X, 8, algas.COSINE, self_base=0)
+    oi, od = oracle.knn_graph(X, 8, oracle.COSINE)
+    assert (si == oi).mean() > 0.99
+    np.testing.assert_allclose(sd, od, atol=2e-5)
