@@ -129,6 +129,12 @@ typedef struct algas_query_stats {
     uint64_t t_loop_end_ns;
     uint64_t t_entry_last_ns;  /* the last CTA to start its search (query staged) */
     uint64_t queue_ns;    /* host: algas_enqueue -> into a slot (0 for algas_submit) */
+    /* candidate updates (P:L219 step 4) by path: the warp-register bitonic
+     * merge fused with the next selection, and the CTA-wide rank merge
+     * (steps with more than 128 surviving new keys, e.g. while the list
+     * fills, or lists longer than the register budget) */
+    uint32_t merges_bitonic;
+    uint32_t merges_rank;
 } algas_query_stats;
 
 /* Optional per-call timing filled by the search entry points. */
@@ -226,6 +232,20 @@ int algas_search_dynamic(const algas_index *idx, const float *queries_dev, int64
  * meanwhile).  Submitting fills idle slots first.  Host poller threads:
  * params->host_threads. */
 int algas_server_create(const algas_index *idx, const algas_params *params, algas_server **out);
+/* As algas_server_create, but the persistent kernel is NOT launched: the
+ * ring, poller threads and device state exist, and algas_submit may stage
+ * up to two queries per slot into the ring (None -> Work) before
+ * algas_server_start launches the kernel.  For bounded sessions under tools
+ * that serialise kernel launches (profilers, compute-sanitizer), where the
+ * host cannot submit while the launch call blocks. */
+int algas_server_create_deferred(const algas_index *idx, const algas_params *params,
+                                 algas_server **out);
+/* Launch a deferred server's kernel.  quit_when_idle != 0 makes it a bounded
+ * session: every free ring entry becomes QUIT -- now and whenever a
+ * finished query's entry is recycled -- so the kernel exits after the staged
+ * queries; submit/enqueue then fail with ALGAS_ESTATE.  Results are still
+ * collected with algas_poll.  ALGAS_ESTATE if already started. */
+int algas_server_start(algas_server *s, int32_t quit_when_idle);
 /* Non-blocking.  query: dim fp32 in HOST memory (copied).  Claims a free
  * ring entry (EMPTY -> READY); ALGAS_EAGAIN if every entry is busy.
  * k <= server k, itopk <= server itopk, width <= 32 (0 -> server value). */

@@ -6,8 +6,12 @@ product path (``paper_conf_ipps_chencyzw025_b200``) never imports it and shares
 no code with it; see ``oracle/oracle.c`` for the function-by-function citation
 of /root/reference/PAPER.md (P:L<line>).
 
-This module is argument marshalling only (numpy <-> ``liboracle.so``); every
-step of the oracle's arithmetic lives in ``oracle.c``.
+This module is argument marshalling (numpy <-> ``liboracle.so``) for every
+function whose arithmetic lives in ``oracle.c`` -- with ONE documented
+exception: ``knn_partitioned`` (f4, R30) writes its clustering
+steps (Lloyd means in float64, the capacity-constrained assignment) in plain
+numpy/Python here, calling O1 (``orc_brute_force``) and the merge
+(``orc_merge_topk``) for its distance and top-k steps.
 
 Parity status per function:
   * orc_distance / orc_brute_force (O1)   pinned: numpy float64 argsort,
@@ -19,8 +23,9 @@ Parity status per function:
   * COSINE metric (R29)                     pinned: hand values, angle closed
     form, unit-circle ordering with random radii.
   * knn_partitioned (f4, R30)              parity unpinned by the paper (no
-    build algorithm in it); pinned by m = 1 / overlap = m == O1 and a
-    hand-worked 1-d example.
+    build algorithm in it); pinned by m = 1 / overlap = m == O1 and two
+    hand-worked 1-d examples, one where a Lloyd move and the capacity bound
+    (4c < m) each change a cluster.
   * orc_prune (K10)                        parity unpinned by the paper (the
     CAGRA algorithm is only cited); pinned by a hand-worked
     example and invariants.

@@ -16,7 +16,7 @@ import threading
 
 import numpy as np
 
-from .build import LIB as _LIB_PATH, build as _build
+from .build import LIB as _LIB_PATH, build as _build, built_hash as _built_hash, source_hash as _source_hash
 
 SENTINEL = 0xFFFFFFFF
 L2 = 0
@@ -54,7 +54,8 @@ class QueryStats(ctypes.Structure):
                 ("cyc_gather", ctypes.c_uint64), ("cyc_dist", ctypes.c_uint64), ("cyc_sort", ctypes.c_uint64),
                 ("t_loop_first_ns", ctypes.c_uint64), ("t_loop_last_ns", ctypes.c_uint64),
                 ("t_loop_end_ns", ctypes.c_uint64), ("t_entry_last_ns", ctypes.c_uint64),
-                ("queue_ns", ctypes.c_uint64)]
+                ("queue_ns", ctypes.c_uint64), ("merges_bitonic", ctypes.c_uint32),
+                ("merges_rank", ctypes.c_uint32)]
 
 
 STATS_DTYPE = np.dtype([("iters", np.uint32), ("max_iters", np.uint32), ("parents", np.uint32),
@@ -63,7 +64,8 @@ STATS_DTYPE = np.dtype([("iters", np.uint32), ("max_iters", np.uint32), ("parent
                         ("t_end_ns", np.uint64), ("latency_ns", np.uint64), ("cyc_select", np.uint64),
                         ("cyc_gather", np.uint64), ("cyc_dist", np.uint64), ("cyc_sort", np.uint64),
                         ("t_loop_first_ns", np.uint64), ("t_loop_last_ns", np.uint64), ("t_loop_end_ns", np.uint64),
-                        ("t_entry_last_ns", np.uint64), ("queue_ns", np.uint64)])
+                        ("t_entry_last_ns", np.uint64), ("queue_ns", np.uint64), ("merges_bitonic", np.uint32),
+                        ("merges_rank", np.uint32)])
 assert STATS_DTYPE.itemsize == ctypes.sizeof(QueryStats)
 
 
@@ -90,7 +92,7 @@ class Tuning(ctypes.Structure):
 # every symbol include/algas.h declares (checked by tests/test_abi.py)
 EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_index_create",
            "algas_index_destroy", "algas_index_info", "algas_search", "algas_search_ex", "algas_search_dynamic",
-           "algas_server_create", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
+           "algas_server_create", "algas_server_create_deferred", "algas_server_start", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
            "algas_build_graph", "algas_knn_partitioned", "algas_build_graph_partitioned"]
@@ -100,15 +102,21 @@ _lib = None
 
 
 def lib(build_if_missing: bool = True):
-    """Load libalgas.so (building it first if it is missing or stale)."""
+    """Load libalgas.so, (re)building it first if it is missing or stale --
+    stale = its recorded source hash differs from the current sources' (a
+    stale library never loads silently: without build_if_missing it raises)."""
     global _lib
     with _lock:
         if _lib is not None:
             return _lib
-        if build_if_missing and not os.path.exists(_LIB_PATH):
+        stale = not os.path.exists(_LIB_PATH) or _built_hash() != _source_hash()
+        if stale and build_if_missing:
             _build()
+            stale = not os.path.exists(_LIB_PATH) or _built_hash() != _source_hash()
         if not os.path.exists(_LIB_PATH):
             raise AlgasError(ECUDA, f"CUDA extension {_LIB_PATH} is missing (run build.py)")
+        if stale:
+            raise AlgasError(ECUDA, f"CUDA extension {_LIB_PATH} is stale (sources changed; run build.py)")
         L = ctypes.CDLL(_LIB_PATH)
         P, i32, i64, u32, u64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_uint64
         L.algas_params_default.argtypes = [ctypes.POINTER(Params)]
@@ -125,6 +133,8 @@ def lib(build_if_missing: bool = True):
         L.algas_search_dynamic.argtypes = [P, P, i64, ctypes.POINTER(Params), u64, P, P, P, P,
                                            ctypes.POINTER(RunInfo)]
         L.algas_server_create.argtypes = [P, ctypes.POINTER(Params), ctypes.POINTER(P)]
+        L.algas_server_create_deferred.argtypes = [P, ctypes.POINTER(Params), ctypes.POINTER(P)]
+        L.algas_server_start.argtypes = [P, i32]
         L.algas_submit.argtypes = [P, P, u64, i32, i32, i32]
         L.algas_submit_many.argtypes = [P, P, i64, u64, i32, i32, i32, ctypes.POINTER(i64)]
         L.algas_enqueue.argtypes = [P, P, i64, u64, i32, i32, i32]
@@ -293,13 +303,21 @@ class Index:
 class Server:
     """Persistent kernel + host-mapped slot ring (algas_server_*)."""
 
-    def __init__(self, index: Index, params: Params):
+    def __init__(self, index: Index, params: Params, deferred: bool = False):
+        """deferred=True: algas_server_create_deferred -- stage queries with
+        submit(), then start() launches the kernel."""
         self.index = index
         self.params = params
         h = ctypes.c_void_p()
-        _check(lib().algas_server_create(index.handle, ctypes.byref(params), ctypes.byref(h)))
+        create = lib().algas_server_create_deferred if deferred else lib().algas_server_create
+        _check(create(index.handle, ctypes.byref(params), ctypes.byref(h)))
         self._h = h
         self.kmax = params.k
+
+    def start(self, quit_when_idle: bool = False) -> None:
+        """Launch a deferred server's kernel (algas_server_start); with
+        quit_when_idle the kernel exits after the staged queries."""
+        _check(lib().algas_server_start(self._h, 1 if quit_when_idle else 0))
 
     def submit(self, query: np.ndarray, tag: int, k: int = 0, itopk: int = 0, width: int = 0) -> bool:
         """True if accepted, False if every slot is busy (EAGAIN)."""

@@ -23,14 +23,33 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", 
          "--expt-relaxed-constexpr", "-Xptxas", "-v"]
 
 
-def _stale() -> bool:
-    if not os.path.exists(LIB):
-        return True
-    t = os.path.getmtime(LIB)
+def source_hash() -> str:
+    """sha256 over the library's sources, headers, kernel unit and this file
+    (content, not mtimes: a repo snapshot copied to another machine keeps
+    its hash but not necessarily its mtimes)."""
+    import hashlib
+    h = hashlib.sha256()
     for f in SOURCES + HEADERS + ["../build.py"]:
-        if os.path.getmtime(os.path.join(CSRC, f)) > t:
-            return True
-    return False
+        with open(os.path.join(CSRC, f), "rb") as fh:
+            h.update(f.encode() + b"\0" + fh.read())
+    h.update(" ".join(EXTRA_DEFS).encode())
+    return h.hexdigest()
+
+
+def _hash_path() -> str:
+    return LIB + ".srchash"
+
+
+def built_hash() -> str | None:
+    try:
+        with open(_hash_path()) as f:
+            return f.read().strip()
+    except OSError:
+        return None
+
+
+def _stale() -> bool:
+    return not os.path.exists(LIB) or built_hash() != source_hash()
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
@@ -66,6 +85,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-L" + cuda_lib, "-lcublas",
                            "-Xlinker", "-rpath=" + cuda_lib, "-lrt", "-lpthread", "-ldl"])
     os.replace(tmp, LIB)
+    with open(_hash_path(), "w") as f:
+        f.write(source_hash() + "\n")
     for o in objs:
         os.remove(o)
     if verbose:

@@ -210,6 +210,8 @@ inline void aggregate_cta_stats(const CtaStats* cs, int T, algas_query_stats* q)
     if (cs[c].t_loop0 > q->t_loop_last_ns) q->t_loop_last_ns = cs[c].t_loop0;
     if (cs[c].t_loop1 > q->t_loop_end_ns) q->t_loop_end_ns = cs[c].t_loop1;
     if (cs[c].t_entry > q->t_entry_last_ns) q->t_entry_last_ns = cs[c].t_entry;
+    q->merges_bitonic += cs[c].mg_bitonic;
+    q->merges_rank += cs[c].mg_rank;
   }
   q->t_start_ns = t0 == ~0ull ? 0 : t0;
   q->t_end_ns = t1;

@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
     if (a.cfg.cosine) normalize_query<NT>(s.q, a.cfg.d4);
     __syncthreads();
     CtaStats* st = a.stats ? a.stats + item : nullptr;
-    search_cta<NT, TL, CPL, METRIC>(a.cfg, s, a.tag0 + (uint64_t)qi, (uint32_t)c, a.k, gt,
+    search_cta<NT, TL, CPL, METRIC>(a.cfg, qpar_of(a.cfg), s, a.tag0 + (uint64_t)qi, (uint32_t)c, a.k, gt,
                                     a.epoch_base + (uint32_t)item, a.res + item * a.k, st);
     __syncthreads();
   }
@@ -152,13 +152,20 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
   // host ring: the slot's two ring entries (sub-slots) alternate, 1 first
   // (runtime.cu); the epoch last seen in each tells a stale READY apart
   int sub = 1;
-  uint32_t last_ep_sub[2] = {0u, 0u};
+  uint32_t last_ep0 = 0u, last_ep1 = 0u;  // (two scalars: a 2-array indexed by `sub` would live in local memory)
 
   for (;;) {
     // ---------------- acquire work (rank 0) and publish it to the slot's CTAs
     if (rank == 0) {
       if (tid == 0) {
         unsigned long long mb;
+        // every CTA of the slot finished the previous query (per-slot HBM
+        // finish counter) before the next one is staged: the slot's HBM
+        // query buffer, params and mailbox are rewritten only after all T
+        // CTAs consumed them, and in SHARED mode the bitmap share a CTA
+        // clears at its next pickup is no longer in use by a slower CTA
+        // (R26).  Wrap-safe difference of u32 counters.
+        while ((int)(ld_acquire_gpu32(P.slot_fin + slot) - served * (uint32_t)P.T) < 0) __nanosleep(32);
         if (P.mode == 0) {
           // host ring: poll the slot state in host memory
           uint32_t st;
@@ -167,7 +174,7 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
             st = ld_acquire_sys(&P.ring[2 * slot + sub].state);
             uint32_t kind = st & 0xFFu, ep = st >> 8;
             if (kind == kSlotQuit) break;
-            if (kind == kSlotReady && ep != last_ep_sub[sub]) break;
+            if (kind == kSlotReady && ep != (sub ? last_ep1 : last_ep0)) break;
             __nanosleep(ns);
             if (ns < 256) ns <<= 1;
           }
@@ -178,8 +185,6 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
             mb = ((unsigned long long)ep << 32) | (unsigned long long)slot;
           }
         } else {
-          // device queue: wait until every CTA of the slot finished the previous query
-          while (ld_acquire_gpu32(P.slot_fin + slot) < (unsigned)(served * P.T)) __nanosleep(32);
           int item = atomicAdd(P.queue_head, 1);
           if (item >= P.nq) {
             mb = kMboxQuit;
@@ -269,10 +274,12 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       // SHARED visited bitmap ("each CTA initializes a part of the
       // visited table"): this query uses buffer served & 1, and
       // every CTA clears its 1/T share of the OTHER buffer now, for the
-      // slot's next query, off the critical path of this one.  That buffer's last user (the previous query)
-      // is complete in every CTA (pickup waits for all T Finish signals),
-      // and these stores are ordered before the next query's first claim by
-      // this CTA's Finish release -> rank 0's acquire -> mailbox release.
+      // slot's next query, off the critical path of this one.  That buffer's
+      // last user (the previous query) is complete in every CTA: rank 0
+      // publishes a query only after the slot's finish counter shows all T
+      // CTAs done with the previous one (both feeds), and these stores are
+      // ordered before the next query's first claim by this CTA's finish
+      // (fence + counter increment) -> rank 0's acquire -> mailbox release.
       vbm = vbm2 + (uint64_t)(served & 1u) * P.vbm_words;
       uint4* o4 = reinterpret_cast<uint4*>(vbm2 + (uint64_t)((served & 1u) ^ 1u) * P.vbm_words);
       const int64_t n4 = P.vbm_words / 4, lo = n4 * rank / P.T, hi = n4 * (rank + 1) / P.T;
@@ -283,10 +290,7 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
     __syncthreads();
 
-    SearchCfg cfg = A.cfg;
-    cfg.L = par.y;
-    cfg.w = par.z;
-    if (cfg.off > cfg.L) cfg.off = cfg.L;
+    const QPar qp{par.y, par.z, A.cfg.off < par.y ? A.cfg.off : par.y};
     const int k = par.x;
     ResultEntry* out;
     CtaStats* stp;
@@ -298,7 +302,7 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       stp = P.dq_stats + (uint64_t)item * P.T + rank;
     }
     CtaStats local;
-    search_cta<NT, TL, CPL, METRIC, CS, MINB>(cfg, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
+    search_cta<NT, TL, CPL, METRIC, CS, MINB>(A.cfg, qp, s, tag, (uint32_t)rank, k, gt, P.epoch_base + served, out,
                                               &local, vbm);
     __syncthreads();
     if (tid == 0) {
@@ -316,11 +320,11 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         st_release_sys(P.ring_done + (uint64_t)(2 * slot + sub) * P.T + rank, epoch);
       } else {
         __threadfence();
-        atomicAdd(P.slot_fin + slot, 1u);
       }
+      atomicAdd(P.slot_fin + slot, 1u);  // the slot's rank 0 gates its next pickup on this
     }
     if (P.mode == 0) {  // the slot's next query is in its other ring entry
-      last_ep_sub[sub] = epoch;
+      if (sub) last_ep1 = epoch; else last_ep0 = epoch;
       sub ^= 1;
     }
   }

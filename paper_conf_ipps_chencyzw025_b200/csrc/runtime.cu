@@ -125,6 +125,12 @@ struct algas_server {
   std::vector<std::thread> pollers;
   std::atomic<bool> stop{false};
   std::atomic<bool> kernel_ok{true};
+  // bounded session (algas_server_start with quit_when_idle): no new work is
+  // accepted, and every ring entry that becomes free is set to QUIT, so the
+  // persistent kernel exits once the staged queries are done
+  std::atomic<bool> quit_when_idle{false};
+  bool launched = false;
+  PersistArgs pa;  // launch arguments (kept for a deferred launch)
   std::mutex cq_mu;
   struct Done {
     uint64_t tag;
@@ -248,7 +254,9 @@ static void poller_main(algas_server* s, int me, int nth) {
       // enqueued query (if any) goes straight into it -- before the result
       // is handed to the caller's completion queue (whose lock a polling
       // caller may hold)
-      __atomic_store_n(&s->ring_h[q].state, (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
+      const bool quit = s->quit_when_idle.load(std::memory_order_acquire) &&
+                        s->n_pending.load(std::memory_order_acquire) == 0;
+      __atomic_store_n(&s->ring_h[q].state, quit ? (uint32_t)kSlotQuit : (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
       s->queue_ns[q] = 0;
       (*s->hstate)[q].store(0, std::memory_order_release);
       drain_pending(s, q >> 1);
@@ -270,7 +278,33 @@ static void poller_main(algas_server* s, int me, int nth) {
 
 extern "C" {
 
+static int server_create(const algas_index* cidx, const algas_params* params, algas_server** out, bool launch);
+
 int algas_server_create(const algas_index* cidx, const algas_params* params, algas_server** out) {
+  return server_create(cidx, params, out, true);
+}
+
+int algas_server_create_deferred(const algas_index* cidx, const algas_params* params, algas_server** out) {
+  return server_create(cidx, params, out, false);
+}
+
+int algas_server_start(algas_server* s, int32_t quit_when_idle) {
+  if (!s) return set_error(ALGAS_EINVAL, "null server");
+  if (s->launched) return set_error(ALGAS_ESTATE, "server already started");
+  if (quit_when_idle) {
+    // every free ring entry becomes QUIT: a slot stops after its staged queries
+    s->quit_when_idle.store(true, std::memory_order_release);
+    for (int u = 0; u < 2 * s->slots; ++u)
+      if ((*s->hstate)[u].load(std::memory_order_acquire) == 0)
+        __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+  }
+  const int rc = launch_persistent(s->plan, s->pa, s->stream);
+  if (rc) return rc;
+  s->launched = true;
+  return ALGAS_OK;
+}
+
+static int server_create(const algas_index* cidx, const algas_params* params, algas_server** out, bool launch) {
   if (!out) return set_error(ALGAS_EINVAL, "null out");
   *out = nullptr;
   algas_index* idx = const_cast<algas_index*>(cidx);
@@ -355,8 +389,12 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
   pa.vbm = s->vbm;
   pa.vbm_words = vw;
   cudaDeviceSynchronize();
-  rc = launch_persistent(s->plan, pa, s->stream);
-  if (rc) return cleanup(rc);
+  s->pa = pa;
+  if (launch) {
+    rc = launch_persistent(s->plan, pa, s->stream);
+    if (rc) return cleanup(rc);
+    s->launched = true;
+  }
   const int nth = std::max(1, std::min(params->host_threads > 0 ? params->host_threads : 1, slots));
   for (int t = 0; t < nth; ++t) s->pollers.emplace_back(poller_main, s, t, nth);
   *out = s;
@@ -366,6 +404,7 @@ int algas_server_create(const algas_index* cidx, const algas_params* params, alg
 int algas_submit(algas_server* s, const float* query, uint64_t tag, int32_t k, int32_t itopk, int32_t width) {
   if (!s || !query) return set_error(ALGAS_EINVAL, "null argument");
   if (s->stop.load()) return set_error(ALGAS_ESTATE, "server is shutting down");
+  if (s->quit_when_idle.load()) return set_error(ALGAS_ESTATE, "bounded session: no new work after start");
   if (k <= 0) k = s->kmax;
   if (itopk <= 0) itopk = s->plan.cfg.L;
   if (width <= 0) width = s->plan.cfg.w;
@@ -403,6 +442,7 @@ int algas_enqueue(algas_server* s, const float* queries, int64_t n, uint64_t tag
                   int32_t width) {
   if (!s || (!queries && n > 0) || n < 0) return set_error(ALGAS_EINVAL, "null argument");
   if (s->stop.load()) return set_error(ALGAS_ESTATE, "server is shutting down");
+  if (s->quit_when_idle.load()) return set_error(ALGAS_ESTATE, "bounded session: no new work after start");
   if (k <= 0) k = s->kmax;
   if (itopk <= 0) itopk = s->plan.cfg.L;
   if (width <= 0) width = s->plan.cfg.w;
@@ -467,7 +507,7 @@ int algas_server_inflight(const algas_server* s, int64_t* n) {
 int algas_server_destroy(algas_server* s) {
   if (!s) return ALGAS_OK;
   int rc = ALGAS_OK;
-  if (s->ring_h && s->stream) {
+  if (s->ring_h && s->stream && s->launched) {
     // Quit: every slot, then wait for the kernel to exit
     for (int u = 0; u < 2 * s->slots; ++u) __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
     auto t0 = std::chrono::steady_clock::now();

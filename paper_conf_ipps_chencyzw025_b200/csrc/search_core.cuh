@@ -229,6 +229,7 @@ struct CtaStats {
   unsigned long long cyc_select, cyc_gather, cyc_dist, cyc_sort;  // SM cycles per phase
   unsigned long long t_loop0, t_loop1;  // globaltimer: search loop entered / left
   unsigned long long t_entry;           // globaltimer: search_cta entered (query staged)
+  uint32_t mg_bitonic, mg_rank;         // candidate updates: warp bitonic merge / rank merge
 };
 
 struct ResultEntry {
@@ -244,8 +245,11 @@ struct Ctrl {
   int nnew[2], nkeys[2];
   uint32_t gc_stamp;  // step stamp of the graph-row cache (claims one copy per slot and step)
   uint32_t iters, parents, dist_evals, cap_hit;
+  uint32_t mg_bitonic, mg_rank;  // candidate updates by the warp bitonic merge / by the rank merge
   uint32_t phase;  // bit b: parity of staging barrier b (b=2: step-ready, b=3: keys)
   uint64_t worst;  // prefilter key of the current step
+  unsigned long long cyc[4];  // per-phase SM cycles (thread 0)
+  long long tp;               // clock64 at the last phase boundary
   // cluster worker mailbox (written remotely by the leader before it arrives
   // on the worker's step-ready barrier)
   int w_cmd;       // kCmdStep / kCmdQuit
@@ -670,6 +674,117 @@ __device__ __forceinline__ uint64_t warp_bitonic_merge32(uint64_t list, uint64_t
   return m;
 }
 
+// Candidate update of the fused path ("parallel-friendly bitonic
+// sort ... merges the candidate list and expand list"), for lists of up to
+// Lp = 32*E keys: warp 0 holds the sorted list in registers, STRIPED (lane l,
+// register e = list position 32*e + l), and absorbs the step's new keys one
+// sorted block of 32 at a time (block 0 sorted here, blocks 1.. by warps
+// 1.. meanwhile).  Inserting block B: C[i] = min(A[i], B'[Lp-1-i]) with B'
+// = B padded by +inf -- only the last register row changes, and C holds the
+// Lp smallest keys of A u B as a bitonic sequence -- then a bitonic merge
+// network sorts C: strides 32m (m = E/2 .. 1) compare registers e, e|m of a
+// lane, strides 16 .. 1 compare lanes (shuffle xor).  A block whose
+// smallest key is >= the list's Lp-th key cannot enter and is skipped.
+// Then the next step's parents are selected from the registers (P:L217 step
+// 1, R6/R7) and the first L keys are written to dst.  Warp-uniform; only
+// lane 0 reads/writes the Ctrl fields it owns.
+template <int E, int NT>
+__device__ __forceinline__ void warp_merge_select(const SearchCfg& cfg, const Smem& s, Ctrl* C, int lane, int cnt,
+                                                  int nk, int nblk, const uint64_t* sorted2, int L, int W, int OFF,
+                                                  int sp, uint32_t& liters, int np_step, int& cur, int& lcnt) {
+  const uint64_t* src = cur ? s.list[1] : s.list[0];
+  uint64_t* dst = cur ? s.list[0] : s.list[1];
+  uint64_t x[E];
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const int i = 32 * e + lane;
+    x[e] = i < cnt ? src[i] : kKeyMax;
+  }
+  if (nk > 0) {
+    for (int b = 0; b < nblk; ++b) {
+      uint64_t blk;
+      if (b == 0 || NT < 128) {
+        blk = warp_bitonic_sort32(32 * b + lane < nk ? s.newk[32 * b + lane] : kKeyMax, lane);
+      } else {
+        if (b == 1) asm volatile("bar.sync 1, %0;" ::"r"(32 * nblk) : "memory");
+        blk = sorted2[32 * b + lane];
+      }
+      const uint64_t last = __shfl_sync(0xffffffffu, x[E - 1], 31);
+      if (__shfl_sync(0xffffffffu, blk, 0) >= last) continue;  // nothing of it can enter
+      x[E - 1] = umin64(x[E - 1], __shfl_sync(0xffffffffu, blk, 31 - lane));
+#pragma unroll
+      for (int m = E >> 1; m > 0; m >>= 1) {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          if (!(e & m)) {
+            const uint64_t a = x[e], c = x[e | m];
+            x[e] = umin64(a, c);
+            x[e | m] = umax64(a, c);
+          }
+        }
+      }
+#pragma unroll
+      for (int j = 16; j > 0; j >>= 1) {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          const uint64_t y = __shfl_xor_sync(0xffffffffu, x[e], j);
+          x[e] = (lane & j) ? umax64(x[e], y) : umin64(x[e], y);
+        }
+      }
+    }
+    cur ^= 1;
+    lcnt = (cnt + nk) < L ? cnt + nk : L;
+  } else {
+    dst = const_cast<uint64_t*>(src);
+  }
+  liters += np_step > 0 ? 1 : 0;
+  // ---- select (P:L217 step 1) from the registers: the first w unchecked
+  // keys in list order (one under greedy search), R6/R7
+  int tot = 0, first_un = -1;
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const unsigned um = __ballot_sync(0xffffffffu, 32 * e + lane < lcnt && !(x[e] & 1ull));
+    if (first_un < 0 && um) first_un = 32 * e + __ffs(um) - 1;
+    tot += __popc(um);
+  }
+  const int diff0 = __shfl_sync(0xffffffffu, lane == 0 ? C->diffusing : 0, 0);
+  int done = 0, np = 0, diff = diff0;
+  if (tot == 0) {
+    done = 1;
+  } else if ((int)liters >= cfg.max_iter) {
+    done = 1;
+    if (lane == 0) C->cap_hit = 1;
+  } else {
+    if (first_un >= OFF) diff = 1;        // P:L249 (sticky, R6)
+    np = diff ? (tot < W ? tot : W) : 1;
+    int base = 0;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const bool un = 32 * e + lane < lcnt && !(x[e] & 1ull);
+      const unsigned um = __ballot_sync(0xffffffffu, un);
+      const int rank = base + __popc(um & ((1u << lane) - 1u));
+      if (un && rank < np) {
+        s.sel[32 + rank] = (int)key_id(x[e]);
+        x[e] |= 1ull;                           // mark checked (Alg.1 l.7)
+      }
+      base += __popc(um);
+    }
+  }
+#pragma unroll
+  for (int e = 0; e < E; ++e)
+    if (32 * e + lane < L) dst[32 * e + lane] = x[e];
+  if (lane == 0) {
+    C->diffusing = diff;
+    C->done = done;
+    C->np = np;
+    C->nnew[sp ^ 1] = 0;
+    C->nkeys[sp ^ 1] = 0;
+    if (!done) C->parents += np;
+    C->cur = cur;
+    C->cnt = lcnt;
+  }
+}
+
 // COSINE (R29): q <- q / |q| in shared memory, by warp 0, between two CTA
 // barriers (the staging threads' stores are visible to warp 0 after the
 // first; everyone reads the unit query after the second).  Every CTA of a
@@ -697,13 +812,22 @@ __device__ __forceinline__ void normalize_query(float4* q, int d4) {
   __syncthreads();
 }
 
+// Per-query search parameters that may differ from the launch's SearchCfg
+// (a server query can ask for a smaller L / w): passed by value so the
+// SearchCfg itself stays in the kernel's parameter space (a local copy of the
+// whole struct would occupy registers for the life of the kernel).
+struct QPar {
+  int L, w, off;
+};
+__host__ __device__ inline QPar qpar_of(const SearchCfg& c) { return QPar{c.L, c.w, c.off}; }
+
 // Preconditions: s.q holds the query (d4 float4, zero tail); init_cta() ran.
 // Writes min(k, |list|) results to out[0..k) (rest padded) and the CTA's
 // counters to *st.  CS > 1: this CTA is the leader of a cluster whose
 // other CTAs run search_worker() in lock step (two cluster barriers per step).
 template <int NT, int TL, int CPL, int METRIC, int CS = 1, int MINB = 1>
-__device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, uint32_t cta_rank, int k,
-                           unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st,
+__device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, uint64_t tag, uint32_t cta_rank,
+                           int k, unsigned long long* gtab, uint32_t epoch, ResultEntry* out, CtaStats* st,
                            uint32_t* vbm = nullptr) {
   const int tid = threadIdx.x;
   const int lane = tid & 31;
@@ -712,11 +836,11 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   const int team = tid / TL;
   const int tl = tid % TL;
   Ctrl* C = s.ctrl;
-  const int L = cfg.L;
+  const int L = qp.L, W = qp.w, OFF = qp.off;
   const int hbits = cfg.hash_bits;
   const int hcap = 1 << hbits;
   const int Rp = 1 << cfg.rp_shift;
-  const int step_max_new = cfg.w * Rp;
+  const int step_max_new = W * Rp;
 
   if (tid == 0 && st) st->t_entry = globaltimer();
   // ---- reset per-query state (16-B stores)
@@ -729,7 +853,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     C->cnt = 0; C->nnew[0] = C->nnew[1] = 0; C->nkeys[0] = C->nkeys[1] = 0; C->np = 0; C->done = 0;
     C->diffusing = 0;
     C->vis_count = 0; C->spilled = 0; C->overflow = 0; C->cur = 0;
-    C->iters = 0; C->parents = 0; C->dist_evals = 0; C->cap_hit = 0;
+    C->iters = 0; C->parents = 0; C->dist_evals = 0; C->cap_hit = 0; C->mg_bitonic = 0; C->mg_rank = 0;
   }
   uint32_t phase = C->phase;  // staging-barrier parities carried across queries
   __syncthreads();
@@ -762,14 +886,18 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   if (tid == 0) C->vis_count = C->nnew[0];
 
   if (tid == 0 && st) st->t_loop0 = globaltimer();
-  // per-phase SM cycles (thread 0; the paper's calc/sort split, Fig. 3/17)
-  long long tp = clock64();
-  unsigned long long cyc[4] = {0, 0, 0, 0};  // select, gather+filter, distance, merge
+  // per-phase SM cycles (thread 0; the paper's calc/sort split, Fig. 3/17),
+  // kept in shared memory: registers held across the whole search loop
+  // would spill under the 64-register budget of a 1024-thread CTA
+  if (tid == 0) {
+    C->cyc[0] = C->cyc[1] = C->cyc[2] = C->cyc[3] = 0;  // select, gather+filter, distance, merge
+    C->tp = clock64();
+  }
   auto lap = [&](int ph) {
     if (tid == 0) {
-      long long t = clock64();
-      cyc[ph] += (unsigned long long)(t - tp);
-      tp = t;
+      const long long t = clock64();
+      C->cyc[ph] += (unsigned long long)(t - C->tp);
+      C->tp = t;
     }
   };
 
@@ -793,8 +921,8 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     // also look past the parents: the next few unchecked candidates are
     // the likely parents of the next step, whose graph rows are
     // prefetched into L2 now (prefetch bit 1; results are unaffected)
-    const int pf = (cfg.prefetch & 2) ? (cfg.w < 16 ? cfg.w : 32 - cfg.w) : 0;
-    const int want = cfg.w + pf;
+    const int pf = (cfg.prefetch & 2) ? (W < 16 ? W : 32 - W) : 0;
+    const int want = W + pf;
     int found = 0;
     for (int base = 0; base < cnt && found < want; base += 32) {
       int i = base + lane;
@@ -805,7 +933,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       found += __popc(m);
     }
     const int found_all = found < want ? found : want;
-    if (found > cfg.w) found = cfg.w;
+    if (found > W) found = W;
     __syncwarp();
     int done = 0, np = 0;
     if (found == 0) {
@@ -814,8 +942,8 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       done = 1;
       if (lane == 0) C->cap_hit = 1;
     } else {
-      int diff = C->diffusing;
-      if (s.sel[0] >= cfg.off) diff = 1;          // P:L249 (sticky, R6)
+      int diff = __shfl_sync(0xffffffffu, lane == 0 ? C->diffusing : 0, 0);  // lane 0 owns the word
+      if (s.sel[0] >= OFF) diff = 1;              // P:L249 (sticky, R6)
       np = diff ? found : 1;
       if (lane < np) {
         int pos = s.sel[lane];
@@ -1033,12 +1161,12 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
     {
       const int nk = C->nkeys[sp];
       const int cnt = lcnt;
-      if (CS == 1 && L <= 32 && nk <= kWarpMergeMax && !(cfg.prefetch & (64 | 2))) {
-        // fused path (short lists): warp 0 merges the new keys into the list
-        // with a warp-level bitonic merge -- warps 1..3 sort the
-        // further blocks of 32 new keys meanwhile -- and selects the next step's
-        // parents from the merged list in its registers, so a step costs one
-        // CTA barrier here instead of three
+      // fused path: register bitonic merge + next select by warp 0 (lists of
+      // up to 32*kMaxE keys, <= kWarpMergeMax new keys: the common step --
+      // the bulk first steps of a query, when the list is still filling,
+      // take the rank merge below)
+      constexpr int kMaxE = (NT * MINB >= 1024) ? 4 : 16;  // list registers within the thread budget
+      if (CS == 1 && L <= 32 * kMaxE && nk <= kWarpMergeMax && !(cfg.prefetch & (64 | 2))) {
         uint64_t* sorted2 = reinterpret_cast<uint64_t*>(s.part);  // blocks 1..3, sorted
         const int nblk = (nk + 31) >> 5;
         if constexpr (NT >= 128) {
@@ -1050,62 +1178,19 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
           }
         }
         if (warp == 0) {
-          const uint64_t* src = cur ? s.list[1] : s.list[0];
-          uint64_t* dst = cur ? s.list[0] : s.list[1];
-          uint64_t mine = lane < cnt ? src[lane] : kKeyMax;
-          if (nk > 0) {
-            mine = warp_bitonic_merge32(mine, warp_bitonic_sort32(lane < nk ? s.newk[lane] : kKeyMax, lane), lane);
-            if (nblk > 1) {
-              if constexpr (NT >= 128) asm volatile("bar.sync 1, %0;" ::"r"(32 * nblk) : "memory");
-              for (int b = 1; b < nblk; ++b) {
-                uint64_t xb;
-                if constexpr (NT >= 128) {
-                  xb = sorted2[32 * b + lane];
-                } else {
-                  xb = warp_bitonic_sort32(32 * b + lane < nk ? s.newk[32 * b + lane] : kKeyMax, lane);
-                }
-                mine = warp_bitonic_merge32(mine, xb, lane);
-              }
-            }
-            cur ^= 1;
-            lcnt = (cnt + nk) < L ? cnt + nk : L;
-          } else {
-            dst = const_cast<uint64_t*>(src);
-          }
-          liters += np_step > 0 ? 1 : 0;
-          // ---- select (P:L217 step 1) from the registers: the first w
-          // unchecked keys in list order (one under greedy search), R6/R7
-          const bool un = lane < lcnt && !(mine & 1ull);
-          const unsigned um = __ballot_sync(0xffffffffu, un);
-          const int found = __popc(um);
-          int done = 0, np = 0;
-          if (found == 0) {
-            done = 1;
-          } else if ((int)liters >= cfg.max_iter) {
-            done = 1;
-            if (lane == 0) C->cap_hit = 1;
-          } else {
-            int diff = C->diffusing;
-            if (__ffs(um) - 1 >= cfg.off) diff = 1;     // P:L249 (sticky, R6)
-            np = diff ? (found < cfg.w ? found : cfg.w) : 1;
-            const int rank = __popc(um & ((1u << lane) - 1u));
-            if (un && rank < np) {
-              s.sel[32 + rank] = (int)key_id(mine);
-              mine |= 1ull;                             // mark checked (Alg.1 l.7)
-            }
-            if (lane == 0) C->diffusing = diff;
-          }
-          if (lane < L) dst[lane] = mine;
-          if (lane == 0) {
-            C->done = done;
-            C->np = np;
-            C->nnew[sp ^ 1] = 0;
-            C->nkeys[sp ^ 1] = 0;
-            if (!done) C->parents += np;
-            if (!C->spilled && gtab != nullptr && C->vis_count + step_max_new > (hcap * 3) / 4) C->spilled = 1;
-            C->cur = cur;
-            C->cnt = lcnt;
-          }
+          if (tid == 0) C->mg_bitonic++;
+          if (L <= 32)
+            warp_merge_select<1, NT>(cfg, s, C, lane, cnt, nk, nblk, sorted2, L, W, OFF, sp, liters, np_step, cur, lcnt);
+          else if (L <= 64)
+            warp_merge_select<2, NT>(cfg, s, C, lane, cnt, nk, nblk, sorted2, L, W, OFF, sp, liters, np_step, cur, lcnt);
+          else if (L <= 128)
+            warp_merge_select<4, NT>(cfg, s, C, lane, cnt, nk, nblk, sorted2, L, W, OFF, sp, liters, np_step, cur, lcnt);
+          else if (L <= 256)
+            warp_merge_select<8, NT>(cfg, s, C, lane, cnt, nk, nblk, sorted2, L, W, OFF, sp, liters, np_step, cur, lcnt);
+          else if constexpr (kMaxE >= 16)
+            warp_merge_select<16, NT>(cfg, s, C, lane, cnt, nk, nblk, sorted2, L, W, OFF, sp, liters, np_step, cur, lcnt);
+          if (tid == 0 && !C->spilled && gtab != nullptr && C->vis_count + step_max_new > (hcap * 3) / 4)
+            C->spilled = 1;
         }
         if (gcache) asm volatile("cp.async.wait_all;" ::: "memory");  // cached rows landed (in warp 0's shadow)
         __syncthreads();
@@ -1115,6 +1200,7 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
         lap(3);
         continue;
       }
+      if (tid == 0 && nk > 0) C->mg_rank++;
       if (nk > 0) {
         const uint64_t* src = cur ? s.list[1] : s.list[0];
         uint64_t* dst = cur ? s.list[0] : s.list[1];
@@ -1172,7 +1258,6 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
   if (tid == 0) {
     C->gc_stamp = gstamp + 1;
     if (st) st->t_loop1 = globaltimer();
-    C->cnt = lcnt;
     C->iters = liters;
   }
   const int cnt = lcnt;
@@ -1198,10 +1283,12 @@ __device__ void search_cta(const SearchCfg& cfg, const Smem& s, uint64_t tag, ui
       st->cap_hit = C->cap_hit;
       st->spilled = C->spilled;
       st->overflow = C->overflow;
-      st->cyc_select = cyc[0];
-      st->cyc_gather = cyc[1];
-      st->cyc_dist = cyc[2];
-      st->cyc_sort = cyc[3];
+      st->cyc_select = C->cyc[0];
+      st->cyc_gather = C->cyc[1];
+      st->cyc_dist = C->cyc[2];
+      st->cyc_sort = C->cyc[3];
+      st->mg_bitonic = C->mg_bitonic;
+      st->mg_rank = C->mg_rank;
     }
   }
 }

@@ -31,6 +31,10 @@ import synth
 pytestmark = pytest.mark.gpu
 SENT = algas.SENTINEL
 N_STREAM = 2000
+# sampled queries the oracle checks one by one: the whole 2000-query stream
+# at the C2 headline point (paired SE of the recall difference ~0.001, so the
+# north-star 0.005 bound is meaningful), fewer at C4 (k = 100) / C3 (960-d)
+N_SAMPLE = {"C2": 2000, "C4": 150, "C3": 120}
 _cache = {}
 
 
@@ -99,7 +103,7 @@ def _check_invariants(X, Q, ids, ds, metric):
 def test_fullsize_knn_graph_rows_match_oracle(name):
     """Sampled rows of the exact kNN graph (the input of the prune) == O1 with
     self exclusion, modulo equal-distance ties (BASELINE north_star)."""
-    w, X, Q, G, idx, rows, knn_rows, _, _ = workload(name, {"C2": 500, "C4": 150, "C3": 120}[name])
+    w, X, Q, G, idx, rows, knn_rows, _, _ = workload(name, N_SAMPLE[name])
     for r, g in zip(rows, knn_rows):
         oi, od = oracle.brute_force(X, X[r:r + 1], w.knn_degree, w.metric, self_base=int(r))
         oi = oi[0]
@@ -127,19 +131,19 @@ C2_POINTS = [(12, 8, 4, 1024, True), (12, 8, 4, 1024, False), (32, 8, 1, 512, Fa
 
 @pytest.mark.parametrize("itopk,width,T,threads,shared", C2_POINTS)
 def test_fullsize_C2_search_bench_launch(itopk, width, T, threads, shared):
-    _search_case("C2", 500, itopk, width, T, threads, shared)
+    _search_case("C2", N_SAMPLE["C2"], itopk, width, T, threads, shared)
 
 
 @pytest.mark.parametrize("itopk,width,T,threads,shared", [(128, 16, 1, 512, False), (128, 16, 4, 1024, True)])
 def test_fullsize_C4_search_ip_k100(itopk, width, T, threads, shared):
-    _search_case("C4", 150, itopk, width, T, threads, shared)
+    _search_case("C4", N_SAMPLE["C4"], itopk, width, T, threads, shared)
 
 
 @pytest.mark.parametrize("itopk,width,T,threads,shared", [(64, 8, 4, 512, False), (64, 8, 4, 512, True)])
 def test_fullsize_C3_search_960d(itopk, width, T, threads, shared):
     """GIST1M-shaped 1M x 960 (3.84 GB of vectors, 60 chunk groups per row)
     at the C3 bench point."""
-    _search_case("C3", 120, itopk, width, T, threads, shared)
+    _search_case("C3", N_SAMPLE["C3"], itopk, width, T, threads, shared)
 
 
 def _search_case(name, n_sample, itopk, width, T, threads, shared):
@@ -164,9 +168,12 @@ def _search_case(name, n_sample, itopk, width, T, threads, shared):
             # summation order -> nearly every query is identical
             same = np.mean([np.array_equal(a, b) for a, b in zip(ids, oi)])
             assert same >= 0.9, same
-    if not shared:
+    print(f"{name} L={itopk} w={width} T={T} nt={threads} shared={shared}: gpu {rg} oracle {ro}")
+    if not shared or name == "C2":
+        # north_star bound; at C2 over the whole 2000-query stream also for
+        # SHARED (3 seeds: 6000 query runs)
         assert np.mean(rg) >= np.mean(ro) - 0.005, (rg, ro)
-    else:
+    if shared:
         # SHARED: which CTA claims a point first is timing-dependent
         # on the GPU; the oracle's step-by-step round robin is one admissible
         # interleaving (R25).  Bound: within 0.015 of it (~3 sigma
@@ -177,3 +184,41 @@ def _search_case(name, n_sample, itopk, width, T, threads, shared):
                                 shared_visited=0, seed=1)
         oi, od = _oracle_search(X, G, Q[sample], op, w.metric, tag0=0)
         assert np.mean(rg) >= oracle.recall(oi, ti, w.k), (rg, oracle.recall(oi, ti, w.k))
+
+
+def test_fullsize_C2_server_shared_recall_matches_device_queue():
+    """The public e2e path at the C2 bench point in SHARED mode:
+    algas_enqueue -> host FIFO -> host-mapped ring (two entries per slot, so a
+    slot's next query is staged while the current one runs) -> persistent
+    kernel -> per-CTA lists in host memory -> host merge.  6000 queries (the
+    2000-query stream cycled with distinct tags, so distinct entry points).
+    Regression test of the ring-mode race where a fast CTA cleared its share
+    of a bitmap a slower CTA of the previous query still used: the server's
+    recall must be within 0.005 of the device-queue path's on the same tags,
+    and every tag completes exactly once."""
+    import torch
+    w, X, Q, G, idx, _, _, sample, ti = workload("C2", N_SAMPLE["C2"])
+    nq = 6000
+    tags_all = np.arange(nq)
+    Qs = np.ascontiguousarray(Q[tags_all % Q.shape[0]])
+    truth = ti[tags_all % Q.shape[0]]
+    p = _params(w, 12, 12, 4, 1024, True, 1)
+    r = idx.search_dynamic(torch.from_numpy(Qs).cuda(), p, tag0=0)
+    rec_dq = oracle.recall(r["ids"], truth, w.k)
+    got = np.full((nq, w.k), SENT, np.uint32)
+    seen = np.zeros(nq, np.int64)
+    with algas.Server(idx, p) as srv:
+        srv.enqueue(Qs, tag0=0)
+        done = 0
+        import time
+        t0 = time.time()
+        while done < nq and time.time() - t0 < 120:
+            tags, ids, ds, st = srv.poll(512)
+            t = tags.astype(np.int64)
+            got[t] = ids[:, :w.k]
+            np.add.at(seen, t, 1)
+            done += len(tags)
+    assert np.all(seen == 1), "every tag completes exactly once"
+    rec_srv = oracle.recall(got, truth, w.k)
+    print(f"server {rec_srv:.4f} device queue {rec_dq:.4f}")
+    assert rec_srv >= rec_dq - 0.005, (rec_srv, rec_dq)

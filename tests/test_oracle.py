@@ -35,7 +35,32 @@ def test_entry_points_in_range_and_spread():
     assert min(e) >= 0 and max(e) < n
     assert len(set(e)) > 0.7 * len(e)  # not degenerate
     assert oracle.entry_point(7, 3, 1, 2, n) == oracle.entry_point(7, 3, 1, 2, n)
-    assert oracle.entry_point(7, 3, 1, 2, n) != oracle.entry_point(8, 3, 1, 2, n) or True
+    # the seed enters the composition: another seed moves (almost) every entry point
+    moved = sum(oracle.entry_point(7, t, c, j, n) != oracle.entry_point(8, t, c, j, n)
+                for t in range(20) for c in range(4) for j in range(8))
+    assert moved > 0.95 * 640, moved
+
+
+def test_entry_point_hand_derived_from_published_vectors():
+    """R5: e = splitmix64(seed ^ splitmix64(tag ^ splitmix64(cta << 32 | j))) mod n,
+    evaluated by hand from the published state-0 outputs o0, o1, o2 of SplitMix64
+    (o_i = splitmix64(i * gamma)):  cta = j = 0 gives splitmix64(0) = o0; with
+    tag = o0 ^ gamma the middle call is splitmix64(gamma) = o1; with
+    seed = o1 ^ (2 gamma mod 2^64) the outer call is splitmix64(2 gamma) = o2.
+    So e = o2 mod n -- any other composition (e.g. tag + a) breaks it."""
+    g = _gold("splitmix64.json")
+    gamma = int(g["gamma_hex"], 16)
+    o0, o1, o2 = (int(h, 16) for h in g["state0_outputs_hex"])
+    M = 2**64 - 1
+    tag = o0 ^ gamma
+    seed = o1 ^ ((2 * gamma) & M)
+    for n in (7, 1000, 1_000_000, 100_000_000, 2**31 - 1):
+        assert oracle.entry_point(seed, tag, 0, 0, n) == o2 % n
+    # the cta / j word: (cta << 32) | j = gamma (cta = gamma >> 32, j = low 32
+    # bits) makes the inner call o1; tag = o1 ^ 2 gamma -> o2; seed = o2 ^ 0 -> o0
+    cta, j = gamma >> 32, gamma & 0xFFFFFFFF
+    assert oracle.entry_point(o2, o1 ^ ((2 * gamma) & M), cta, j, 1_000_003) == \
+        oracle.splitmix64(0) % 1_000_003 == o0 % 1_000_003
 
 
 # ---------------------------------------------------------------- distance
@@ -228,6 +253,49 @@ def test_search_path_graph_hand_trace():
     assert st["iters"][0] == 9 - e
     assert st["dist_evals"][0] == 11 - e
     assert st["parents"][0] == 9 - e
+
+
+# The beam-extend hand trace (R6/R7).  1-d points (d padded
+# to 4 with zeros) on a small directed graph, query at 0; squared distances
+# A=100 B=144 C=169 D=25 E=400 F=16 G=900.
+BEAM_X = [10, 12, 13, 5, 20, 4, 30]           # ids 0..6 = A B C D E F G
+BEAM_G = [[1, 2], [3, SENT], [4, SENT], [5, 0], [6, SENT], [3, SENT], [4, SENT]]
+BEAM_SEED = 3                                  # entry_point(3, tag 0, cta 0, j 0, n 7) = 0 = A
+
+
+def beam_case():
+    X = np.zeros((7, 4), np.float32)
+    X[:, 0] = BEAM_X
+    return X, np.array(BEAM_G, np.uint32), np.zeros((1, 4), np.float32)
+
+
+# (off, iters, parents, dist_evals), worked by hand in test_beam_extend_trigger_hand_trace
+BEAM_TRACES = [(1, 4, 6, 7), (2, 5, 5, 6), (5, 5, 5, 6)]
+
+
+@pytest.mark.parametrize("off,iters,parents,evals", BEAM_TRACES)
+def test_beam_extend_trigger_hand_trace(off, iters, parents, evals):
+    """L = 5, w = 2, one seed (A), T = 1.  Diffusing latches when the FIRST
+    unchecked position U[0] >= off and stays on (R6, sticky).
+
+    off = 1:  s1 list [A] U=[0], 0<1 greedy: expand A -> B, C; list [A* B C].
+              s2 U=[1,2], 1>=1 -> diffusing: expand B, C -> D, E; [D A* B* C* E].
+              s3 U=[0,4]: sticky, so 2 parents D, E -> F, G; [F D* A* B* C*] (E, G cut).
+              s4 U=[0] -> F (D visited).  s5 U=[] Finish.
+              iters 4, parents 1+2+2+1 = 6, evals 1+2+2+2 = 7.
+              (with '>' instead of '>=': s2 is greedy -> iters 5, parents 5;
+               non-sticky: s3 has U[0]=0 < 1 -> one parent -> parents 5, evals 6)
+    off = 2:  s2 U[0]=1 <2 greedy: B -> D; [D A* B* C].  s3 U=[0,3] greedy D -> F;
+              [F D* A* B* C].  s4 U=[0,4] greedy F.  s5 U=[4], 4>=2 diffusing: C -> E;
+              [F D* A* B* C*] (E cut).  s6 U=[] Finish: iters 5, parents 5, evals 6.
+    off = 5 (= L, beam extend off, Alg. 1): the same walk as off = 2.
+    In every case the result (k = 3) is F, D, A at 16, 25, 100."""
+    X, G, q = beam_case()
+    assert oracle.entry_point(BEAM_SEED, 0, 0, 0, 7) == 0
+    p = oracle.make_params(k=3, L=5, w=2, off=off, T=1, S=1, seed=BEAM_SEED)
+    ids, ds, st = oracle.search(X, G, q, p)
+    assert ids[0].tolist() == [5, 3, 0] and ds[0].tolist() == [16.0, 25.0, 100.0]
+    assert (st["iters"][0], st["parents"][0], st["dist_evals"][0]) == (iters, parents, evals)
 
 
 def test_search_star_graph():
@@ -461,6 +529,33 @@ def test_knn_partitioned_hand_example():
     assert np.isinf(ds[:, 2]).all()
     ei, ed = oracle.knn_graph(X, 3)
     assert ei[2].tolist() == [1, 0, 3] and ed[2, 2] == 64.0
+
+
+def test_knn_partitioned_capacity_and_lloyd_hand_example():
+    """m = 5 clusters, overlap c = 1 (4c < m: capacity ceil(2cn/m) = 4), n = 10,
+    1-d points by id x = 7 16 3 10 4 11 29 9 22 13 (d padded to 4), k = 3.
+    Initial centres = rows 0,2,4,6,8 = 7 3 4 29 22.
+    Lloyd 1 (sample = all rows; nearest centre, ties to the lower index):
+      7,10,11,9,13 -> c0; 16,22 -> c4; 3 -> c1; 4 -> c2; 29 -> c3
+      => centres 10 3 4 29 19.  Lloyd 2: same assignment (7 ties c0/c2 at 9
+      -> c0) => converged.
+    Capacity pass in id order, P = min(m, 4c+4) = 5 preferences:
+      c0 takes ids 0 (7), 3 (10), 5 (11), 7 (9) -> full; id 9 (13) prefers c0
+      (36) but it is full -> c4 (19, 36 < c2's 81).  Clusters: c0 {0,3,5,7},
+      c1 {2}, c2 {4}, c3 {6}, c4 {1,8,9}.
+    Without Lloyd, id 9 would go to c2 (tie 81 with c4 at 22, lower index);
+    without the capacity, to c0 -- both change row 9 below."""
+    x = np.array([7, 16, 3, 10, 4, 11, 29, 9, 22, 13], np.float32)
+    X = np.zeros((10, 4), np.float32)
+    X[:, 0] = x
+    ids, ds = oracle.knn_partitioned(X, 3, 5, 1)
+    S = oracle.SENTINEL
+    assert ids[9].tolist() == [1, 8, S] and ds[9].tolist()[:2] == [9.0, 81.0]     # c4: 16, 22
+    assert ids[1].tolist() == [9, 8, S] and ds[1].tolist()[:2] == [9.0, 36.0]
+    assert ids[0].tolist() == [7, 3, 5] and ds[0].tolist() == [4.0, 9.0, 16.0]    # c0: 9, 10, 11
+    assert ids[7].tolist() == [3, 0, 5] and ds[7].tolist() == [1.0, 4.0, 4.0]     # tie 4: id order
+    for i in (2, 4, 6):                                                           # singletons
+        assert ids[i].tolist() == [S, S, S] and np.isinf(ds[i]).all()
 
 
 @pytest.mark.parametrize("metric", [oracle.L2, oracle.IP])

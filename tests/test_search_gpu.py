@@ -197,6 +197,14 @@ LATTICE_CASES = [
     (2000, 100, algas.IP, 32, dict(k=10, itopk=48, width=2, offset_beam=12, n_seeds=32, ctas_per_query=1)),
     (2000, 960, algas.L2, 20, dict(k=10, itopk=32, width=2, offset_beam=8, n_seeds=8, ctas_per_query=1)),
     (1500, 256, algas.IP, 24, dict(k=5, itopk=5, width=1, n_seeds=1, ctas_per_query=4)),
+    # the C2 bench operating-point shape: L = 12, w = 12, R = 64 (Rp = 64), T = 4,
+    # beam from the first step -- up to 768 new ids and 3-4 key blocks per step
+    (4000, 128, algas.L2, 64, dict(k=10, itopk=12, width=12, offset_beam=1, n_seeds=32, ctas_per_query=4)),
+    # long lists (L = 64 ... 512): the multi-key-per-lane bitonic merge
+    (3000, 64, algas.L2, 32, dict(k=10, itopk=64, width=8, offset_beam=1, n_seeds=32, ctas_per_query=2)),
+    (3000, 100, algas.IP, 64, dict(k=100, itopk=128, width=16, offset_beam=1, n_seeds=32, ctas_per_query=2)),
+    (3000, 48, algas.L2, 40, dict(k=20, itopk=256, width=8, offset_beam=4, n_seeds=64, ctas_per_query=1)),
+    (5000, 32, algas.L2, 32, dict(k=64, itopk=512, width=16, offset_beam=1, n_seeds=128, ctas_per_query=1)),
 ]
 
 
@@ -222,6 +230,29 @@ def test_search_lattice_exact_trajectory(case, threads):
     np.testing.assert_array_equal(st["max_iters"].astype(np.int64), ost["max_iters"])
     assert (st["cap_hits"] == 0).all() and (st["overflows"] == 0).all()
     _check_invariants(X, Q, r["ids"], r["dists"], metric, p.k)
+    # the candidate update ran on the warp-register bitonic merge
+    # wherever the list fits the register budget (32 x 4 keys per lane at
+    # 1024 threads, 32 x 16 below); steps with > 128 new keys take the rank merge
+    if p.itopk <= (128 if threads == 1024 else 512):
+        assert st["merges_bitonic"].sum() > 0
+    assert (st["merges_bitonic"] + st["merges_rank"] <= st["iters"]).all()
+
+
+@pytest.mark.parametrize("threads", [32, 128, 1024])
+def test_search_beam_extend_hand_trace(threads):
+    """The hand-worked beam-extend trace of tests/test_oracle.py (R6: the
+    trigger is U[0] >= off and sticky): the GPU reproduces its step, parent
+    and evaluation counts for off = 1 / 2 / 5 and the result F, D, A."""
+    from test_oracle import BEAM_SEED, BEAM_TRACES, beam_case
+    X, G, q = beam_case()
+    idx = algas.Index(X, G)
+    for off, iters, parents, evals in BEAM_TRACES:
+        p = algas.default_params(k=3, itopk=5, width=2, offset_beam=off, n_seeds=1, ctas_per_query=1,
+                                 threads_per_cta=threads, seed=BEAM_SEED)
+        r = idx.search(q, params=p)
+        st = r["stats"][0]
+        assert r["ids"][0].tolist() == [5, 3, 0] and r["dists"][0].tolist() == [16.0, 25.0, 100.0]
+        assert (int(st["iters"]), int(st["parents"]), int(st["dist_evals"])) == (iters, parents, evals), off
 
 
 def test_search_spill_to_hbm_is_exact():
