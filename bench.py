@@ -351,17 +351,17 @@ def cpu_baseline(W, w, p, gpu_ids, budget_s=8.0):
                              max_iter=4 * p.itopk + 256, seed=p.seed)
     _, st1 = _oracle_parallel(X, G, Q[:npar], op1, w.metric, 0, cores)
     lat_us = s["lats"] * 1e6
-    return {"value": s["n"] / s["el"], "unit": "queries/s", "cores": 1, "kind": "oracle",
-            "sample": f"O2 T=1 L={L_cpu} w={op.w} off={op.off} S={CPU_S} (its smallest L with calibration "
-                      f"recall>={0.95 + MARGIN}), first {s['n']} measured queries one at a time on core "
-                      f"{cores[0]}, {s['el']:.1f}s",
+    return {"value": round(s["n"] / s["el"], 1), "unit": "queries/s", "cores": 1, "kind": "oracle",
+            "sample": f"O2 T=1 L={L_cpu} w={op.w} (own op point), {s['n']} queries 1-by-1 on core {cores[0]}, "
+                      f"{s['el']:.1f}s",
             "p50_us": round(float(np.percentile(lat_us, 50)), 1), "p99_us": round(float(np.percentile(lat_us, 99)), 1),
             "recall": round(recall_at(s["ids"], truth[:s["n"]], w.k), 4),
             "all_cores": {"value": round(qps_all, 1), "cores": len(cores)},
             "cpu_model": _cpu_model(),
             "parity": {"n": npar, "recall_oracle_gpu_params": round(recall_at(pid, truth[:npar], w.k), 4),
                        "recall_gpu": round(recall_at(gpu_ids[:npar], truth[:npar], w.k), 4)},
-            "unique_evals_T1": float(st1["dist_evals"].mean()), "unique_parents_T1": float(st1["parents"].mean())}
+            "unique_evals_T1": round(float(st1["dist_evals"].mean()), 1),
+            "unique_parents_T1": round(float(st1["parents"].mean()), 1)}
 
 
 def run_algas(a, rank, world, local):
@@ -498,6 +498,9 @@ def run_algas(a, rank, world, local):
     if rank != 0:
         return
     detail_path = write_detail(a, world, detail)
+    unique_b = None
+    if cpu:  # bytes ONE CTA needs (O2 T = 1 at the GPU's L, w): multi-CTA redundancy is not efficiency
+        unique_b = round(cpu["unique_parents_T1"] * Rp * 4 + cpu["unique_evals_T1"] * w.dim * 4 + w.dim * 4 + w.k * 8)
     line = {
         "metric": METRIC_NAME,
         "value": round(value, 1),
@@ -510,22 +513,23 @@ def run_algas(a, rank, world, local):
         "scaling": "weak",
         "vs_baseline": None,
         "dtype": "f32",
-        "data": "synthetic (seeded clustered Gaussian mixture; synth/)",
+        "data": "synthetic (seeded Gaussian mixture, synth/)",
         "config": {"workload": w.name, "n": w.n, "dim": w.dim, "metric": "L2" if w.metric == 0 else "IP",
                    "degree": w.degree, "k": w.k, "batch": a.batch, "queries_per_step": a.nq,
                    "itopk": p.itopk, "width": p.width, "offset_beam": p.offset_beam,
                    "ctas_per_query": p.ctas_per_query, "threads_per_cta": p.threads_per_cta,
                    "visited": "shared" if p.visited_mode else "private",
-                   "recall": round(float(np.mean(recs)), 4), "op_chosen_on": "calibration set (synth stream 1)",
-                   "parallelism": f"replicas x{world}", "l2": "flushed (256 MB write) between timed steps"},
+                   "recall": round(float(np.mean(recs)), 4), "op_from": "calibration set",
+                   "parallelism": f"replicas x{world}", "l2": "256MB flush between steps"},
         "latency_us": {"p50": round(float(np.percentile(lat, 50)), 1), "p99": round(float(np.percentile(lat, 99)), 1),
-                       "def": "device: slot pickup -> last CTA published"},
+                       "def": "device: pickup->published"},
         "clocks": clk.summary(),
         "e2e": e2e,
         "gpu_launches": a.steps,
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
                      "kernel": "persistent_kernel", "algo_bytes_per_query": round(float(bytes_q.mean())),
+                     "unique_bytes_per_query": unique_b,
                      "kernel_ms": round(float(np.mean(kern_ms)), 3)},
         "cpu_baseline": cpu,
         "work": {"evals_per_query": round(float(evals.mean()), 1), "parents_per_query": round(float(parents.mean()), 1),
@@ -556,6 +560,7 @@ def run_e2e(a, idx, p, Q, truth, w, world, dev, detail):
     import paper_conf_ipps_chencyzw025_b200 as algas
     ps = algas.default_params(**{f: getattr(p, f) for f, _ in p._fields_ if not f.startswith("reserved")})
     ps.host_threads = a.host_threads
+    ps.state_mirror = a.state_mirror
     srv = algas.Server(idx, ps)
     nQ = Q.shape[0]
     try:
@@ -619,9 +624,8 @@ def run_e2e(a, idx, p, Q, truth, w, world, dev, detail):
             "h2d_bytes_per_step": int(a.nq * (w.dim * 4 + 32)),
             "d2h_bytes_per_step": int(a.nq * (p.ctas_per_query * (w.k * 8 + 32) + 4)),
             "recall": round(rec, 4), "p50_us": lat_b[0], "p99_us": lat_b[1],
-            "batch": per_b,
-            "def": "algas_enqueue/algas_poll, host query -> merged host result; latency: closed loop, "
-                   "batch = queries outstanding"}
+            "batch": per_b, "state_mirror": a.state_mirror,
+            "def": "enqueue->poll host in/out; lat: closed loop [p50,p99,qps]"}
 
 
 def tuner_point(idx, W, w, slots, p_best, stream):
@@ -631,7 +635,7 @@ def tuner_point(idx, W, w, slots, p_best, stream):
     import paper_conf_ipps_chencyzw025_b200 as algas
     tu = algas.tune(slots, w.dim, w.degree, p_best.itopk, w.k)
     T, nt, wd, off = tu.ctas_per_query, tu.threads_per_cta, tu.width, tu.offset_beam
-    vis = 1 if (T > 1 and getattr(tu, "visited_mode", 1)) else 0
+    vis = tu.visited_mode if T > 1 else 0
     pts, pc = sweep_L(idx, W["Qcd"], W["tc"], w, slots, T, nt, wd, off, vis, 0.95 + MARGIN)
     if pc is None:
         return {"T": T, "threads": nt, "width": wd, "itopk": None, "qps": None, "ratio_to_swept": None}
@@ -735,6 +739,8 @@ def main():
     ap.add_argument("--visited", type=ints, default=(0, 1), help="visited modes: 0 private, 1 shared (P:L211)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--host-threads", type=int, default=0, help="server poller threads (0: library default)")
+    ap.add_argument("--state-mirror", type=int, default=0,
+                    help="e2e server: 1 = host mirrors slot state/params/query into HBM (P:L255-272)")
     ap.add_argument("--cpu-budget", type=float, default=8.0)
     ap.add_argument("--ref-queries-per-step", type=int, default=50)
     ap.add_argument("--detail", default=None, help="side file for the sweeps (default gpurun_out/bench_detail_*.json)")

@@ -99,6 +99,12 @@ typedef struct algas_params {
                                 slots q with q % host_threads == its index, merging
                                 and refilling them (Fig. 18); 0 -> 1 (measured best on
                                 the B200 box: more threads contend for the FIFO/queue locks) */
+    int32_t state_mirror;    /* persistent server: 1 = the host mirrors each staged query's
+                                state word, params and query into DEVICE memory (stream-
+                                ordered async copies from the host thread's private IO
+                                stream, P:L255-272's GDRCopy state copy without GDRCopy), so
+                                the slots' CTAs poll HBM instead of host memory over PCIe;
+                                0 (default) = CTAs poll the host-mapped ring */
     uint64_t seed;           /* entry-point generator seed (R5)                      */
 } algas_params;
 
@@ -317,7 +323,7 @@ typedef struct algas_tuning {
     int32_t offset_beam;
     int32_t hash_bits;
     int32_t stage_rows;
-    int32_t reserved;
+    int32_t visited_mode;     /* enum algas_visited: SHARED when T > 1 */
 } algas_tuning;
 
 /* Properties of the current device (props of P:L280-291 Table II). */
@@ -327,8 +333,8 @@ int32_t algas_tuner_max_parallel(int32_t slots, int32_t n_sm, int32_t max_blocks
 int32_t algas_tuner_blocks_per_sm(int32_t n_parallel, int32_t slots, int32_t n_sm);
 int64_t algas_tuner_smem_per_block(int64_t smem_per_sm, int32_t blocks_per_sm,
                                    int64_t smem_reserved_per_block);
-/* Full tuner: picks T, threads/CTA, width, offset_beam and the visited hash
- * size for `slots` concurrent queries of this shape so that every slot's
+/* Full tuner: picks T, threads/CTA, width, offset_beam, the visited mode and
+ * the visited hash size for `slots` concurrent queries of this shape so that every slot's
  * CTAs are co-resident and the per-block shared memory respects
  * P:L245 with M_reserved sized for the dimension.
  * props NULL -> algas_device_query().  Returns EINVAL if no configuration fits. */

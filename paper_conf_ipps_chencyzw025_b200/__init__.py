@@ -43,7 +43,8 @@ class Params(ctypes.Structure):
                 ("threads_per_cta", ctypes.c_int32), ("n_seeds", ctypes.c_int32),
                 ("max_iter", ctypes.c_int32), ("visited_mode", ctypes.c_int32), ("slots", ctypes.c_int32),
                 ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32),
-                ("cluster_size", ctypes.c_int32), ("host_threads", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("cluster_size", ctypes.c_int32), ("host_threads", ctypes.c_int32),
+                ("state_mirror", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class QueryStats(ctypes.Structure):
@@ -86,7 +87,7 @@ class Tuning(ctypes.Structure):
     _fields_ = [("ctas_per_query", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
                 ("smem_avail_per_block", ctypes.c_int64), ("smem_per_block", ctypes.c_int64),
                 ("threads_per_cta", ctypes.c_int32), ("width", ctypes.c_int32), ("offset_beam", ctypes.c_int32),
-                ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32), ("visited_mode", ctypes.c_int32)]
 
 
 # every symbol include/algas.h declares (checked by tests/test_abi.py)

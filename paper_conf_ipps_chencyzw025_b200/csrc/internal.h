@@ -145,6 +145,12 @@ struct PersistArgs {
   ResultEntry* ring_res;    // slots x T x kmax
   CtaStats* ring_stats;     // slots x T
   uint32_t* ring_done;      // slots x T
+  // state mirror (algas_params.state_mirror): per ring entry a device copy
+  // of the RingSlot line (state word first) followed by the query, written by
+  // the host with stream-ordered copies (payload, then state); null = poll
+  // the host-mapped ring
+  const uint8_t* mir;
+  int64_t mir_stride;       // bytes per mirrored entry (64 + dim*4, 16-B multiple)
   // device mailbox
   unsigned long long* mbox; // slots
   float4* qbuf;             // slots x d4

@@ -167,11 +167,14 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         // (R26).  Wrap-safe difference of u32 counters.
         while ((int)(ld_acquire_gpu32(P.slot_fin + slot) - served * (uint32_t)P.T) < 0) __nanosleep(32);
         if (P.mode == 0) {
-          // host ring: poll the slot state in host memory
+          // host ring: poll the slot state in host memory, or its
+          // device mirror in HBM (state_mirror: no PCIe read while polling)
           uint32_t st;
           unsigned ns = 64;
+          const uint32_t* mstate =
+              P.mir ? reinterpret_cast<const uint32_t*>(P.mir + (size_t)(2 * slot + sub) * P.mir_stride) : nullptr;
           for (;;) {
-            st = ld_acquire_sys(&P.ring[2 * slot + sub].state);
+            st = mstate ? ld_acquire_gpu32(mstate) : ld_acquire_sys(&P.ring[2 * slot + sub].state);
             uint32_t kind = st & 0xFFu, ep = st >> 8;
             if (kind == kSlotQuit) break;
             if (kind == kSlotReady && ep != (sub ? last_ep1 : last_ep0)) break;
@@ -203,7 +206,10 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         // at once (volatile: never a stale line; ordered after thread 0's
         // acquire of the state by the barrier), staged into the slot's HBM
         // buffer for the other CTAs and into this CTA's shared memory
-        const float4* src = P.ring_q + (uint64_t)(2 * slot + sub) * A.cfg.d4;
+        const uint8_t* ment = P.mir ? P.mir + (size_t)(2 * slot + sub) * P.mir_stride : nullptr;
+        const RingSlot* rs = ment ? reinterpret_cast<const RingSlot*>(ment) : &P.ring[2 * slot + sub];
+        const float4* src = ment ? reinterpret_cast<const float4*>(ment + sizeof(RingSlot))
+                                 : P.ring_q + (uint64_t)(2 * slot + sub) * A.cfg.d4;
         float4* dst = P.qbuf + (uint64_t)slot * A.cfg.d4;
         for (int i = tid; i < A.cfg.d4; i += NT) {
           const float4 v = ld_volatile_f4(src + i);
@@ -211,10 +217,10 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
           s.q[i] = v;
         }
         if (tid == NT - 1) {
-          const int4 sp4 = ld_volatile_i4(reinterpret_cast<const int4*>(&P.ring[2 * slot + sub]));
+          const int4 sp4 = ld_volatile_i4(reinterpret_cast<const int4*>(rs));
           P.dparams[slot] = make_int4(sp4.y, sp4.z, sp4.w, 0);
         }
-        if (tid == NT - 2) P.dtag[slot] = *((const volatile unsigned long long*)&P.ring[2 * slot + sub].tag);
+        if (tid == NT - 2) P.dtag[slot] = *((const volatile unsigned long long*)&rs->tag);
       }
       __syncthreads();
       if (tid == 0) {

@@ -131,6 +131,16 @@ struct algas_server {
   std::atomic<bool> quit_when_idle{false};
   bool launched = false;
   PersistArgs pa;  // launch arguments (kept for a deferred launch)
+  // state mirror: host staging of every ring entry (RingSlot line
+  // + query) in pinned memory and its device copy the CTAs poll; each host
+  // thread writes through its own IO stream ("private IO streams")
+  bool mirror = false;
+  uint8_t* mir_h = nullptr;
+  uint8_t* mir_d = nullptr;
+  int64_t mir_stride = 0;
+  uint64_t uid = 0;  // server identity for the per-thread stream cache
+  std::mutex io_mu;
+  std::vector<cudaStream_t> io_streams;
   std::mutex cq_mu;
   struct Done {
     uint64_t tag;
@@ -156,20 +166,64 @@ struct algas_server {
 };
 
 namespace {
+std::atomic<uint64_t> g_server_uid{1};
+
+// the calling thread's private IO stream for server s (created on first use,
+// destroyed with the server)
+cudaStream_t io_stream(algas_server* s) {
+  thread_local std::vector<std::pair<uint64_t, cudaStream_t>> cache;
+  for (auto& e : cache)
+    if (e.first == s->uid) return e.second;
+  cudaStream_t st = nullptr;
+  cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+  {
+    std::lock_guard<std::mutex> lk(s->io_mu);
+    s->io_streams.push_back(st);
+  }
+  if (cache.size() > 64) cache.erase(cache.begin());
+  cache.emplace_back(s->uid, st);
+  return st;
+}
+
+// state mirror: publish host staging entry u's state word `state` to the
+// device copy -- the payload (params + query) first, the state word last,
+// both stream-ordered on the calling thread's IO stream (with_payload = 0:
+// state only, e.g. QUIT)
+void mirror_publish(algas_server* s, int u, uint32_t state, bool with_payload) {
+  uint8_t* h = s->mir_h + (size_t)u * s->mir_stride;
+  uint8_t* d = s->mir_d + (size_t)u * s->mir_stride;
+  __atomic_store_n(reinterpret_cast<uint32_t*>(h), state, __ATOMIC_RELEASE);
+  cudaStream_t st = io_stream(s);
+  if (with_payload) cudaMemcpyAsync(d + 4, h + 4, (size_t)s->mir_stride - 4, cudaMemcpyHostToDevice, st);
+  cudaMemcpyAsync(d, h, 4, cudaMemcpyHostToDevice, st);
+}
+
 // None -> Work of a claimed sub-slot u (epoch already assigned):
 // payload first, state word last (release)
 void write_slot(algas_server* s, int u, const float* query, uint64_t tag, int32_t k, int32_t itopk, int32_t width) {
+  s->tags[u] = tag;
+  s->kq[u] = k;
+  s->t_submit[u] = std::chrono::steady_clock::now();
+  (*s->hstate)[u].store(2, std::memory_order_release);
+  const uint32_t state = (s->epoch[u] << 8) | kSlotReady;
+  if (s->mirror) {
+    uint8_t* h = s->mir_h + (size_t)u * s->mir_stride;
+    RingSlot* rs = reinterpret_cast<RingSlot*>(h);
+    rs->k = k;
+    rs->L = itopk;
+    rs->w = width;
+    rs->tag = tag;
+    memcpy(h + sizeof(RingSlot), query, (size_t)s->dim * 4);
+    mirror_publish(s, u, state, true);
+    return;
+  }
   memcpy(s->ringq_h + (size_t)u * s->dim, query, (size_t)s->dim * 4);
   RingSlot* rs = &s->ring_h[u];
   rs->k = k;
   rs->L = itopk;
   rs->w = width;
   rs->tag = tag;
-  s->tags[u] = tag;
-  s->kq[u] = k;
-  s->t_submit[u] = std::chrono::steady_clock::now();
-  (*s->hstate)[u].store(2, std::memory_order_release);
-  __atomic_store_n(&rs->state, (s->epoch[u] << 8) | kSlotReady, __ATOMIC_RELEASE);
+  __atomic_store_n(&rs->state, state, __ATOMIC_RELEASE);
 }
 // claim the next sub-slot of a slot whose next sub-slot is free (host state
 // 0 -> 1) and give it the slot's next epoch, scanning slots from `start`, a
@@ -257,6 +311,7 @@ static void poller_main(algas_server* s, int me, int nth) {
       const bool quit = s->quit_when_idle.load(std::memory_order_acquire) &&
                         s->n_pending.load(std::memory_order_acquire) == 0;
       __atomic_store_n(&s->ring_h[q].state, quit ? (uint32_t)kSlotQuit : (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
+      if (quit && s->mirror) mirror_publish(s, q, kSlotQuit, false);
       s->queue_ns[q] = 0;
       (*s->hstate)[q].store(0, std::memory_order_release);
       drain_pending(s, q >> 1);
@@ -295,8 +350,11 @@ int algas_server_start(algas_server* s, int32_t quit_when_idle) {
     // every free ring entry becomes QUIT: a slot stops after its staged queries
     s->quit_when_idle.store(true, std::memory_order_release);
     for (int u = 0; u < 2 * s->slots; ++u)
-      if ((*s->hstate)[u].load(std::memory_order_acquire) == 0)
+      if ((*s->hstate)[u].load(std::memory_order_acquire) == 0) {
         __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+        if (s->mirror) mirror_publish(s, u, kSlotQuit, false);
+      }
+    if (s->mirror) cudaStreamSynchronize(io_stream(s));
   }
   const int rc = launch_persistent(s->plan, s->pa, s->stream);
   if (rc) return rc;
@@ -342,6 +400,17 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   SRV_ALLOC(s->st_h, s->st_d, sizeof(CtaStats) * (size_t)nsub * s->T);
   SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)nsub * s->T);
 #undef SRV_ALLOC
+  s->uid = g_server_uid.fetch_add(1);
+  s->mirror = params->state_mirror != 0;
+  if (s->mirror) {
+    s->mir_stride = (int64_t)sizeof(RingSlot) + (int64_t)s->dim * 4;  // 16-B multiple (dim % 4 == 0)
+    if ((e = cudaHostAlloc((void**)&s->mir_h, (size_t)nsub * s->mir_stride, cudaHostAllocPortable)) != cudaSuccess)
+      return cleanup(set_error(ALGAS_ENOMEM, "cudaHostAlloc mirror staging: %s", cudaGetErrorString(e)));
+    memset(s->mir_h, 0, (size_t)nsub * s->mir_stride);
+    if ((e = cudaMalloc(&s->mir_d, (size_t)nsub * s->mir_stride)) != cudaSuccess)
+      return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc state mirror: %s", cudaGetErrorString(e)));
+    cudaMemset(s->mir_d, 0, (size_t)nsub * s->mir_stride);
+  }
   s->hstate = new std::vector<std::atomic<int>>(nsub);
   for (auto& a : *s->hstate) a.store(0);
   s->epoch.assign(nsub, 0);
@@ -388,6 +457,8 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   pa.epoch_base = 1;
   pa.vbm = s->vbm;
   pa.vbm_words = vw;
+  pa.mir = s->mir_d;
+  pa.mir_stride = s->mir_stride;
   cudaDeviceSynchronize();
   s->pa = pa;
   if (launch) {
@@ -509,7 +580,10 @@ int algas_server_destroy(algas_server* s) {
   int rc = ALGAS_OK;
   if (s->ring_h && s->stream && s->launched) {
     // Quit: every slot, then wait for the kernel to exit
-    for (int u = 0; u < 2 * s->slots; ++u) __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+    for (int u = 0; u < 2 * s->slots; ++u) {
+      __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+      if (s->mirror) mirror_publish(s, u, kSlotQuit, false);
+    }
     auto t0 = std::chrono::steady_clock::now();
     for (;;) {
       cudaError_t e = cudaStreamQuery(s->stream);
@@ -538,6 +612,9 @@ int algas_server_destroy(algas_server* s) {
     if (s->res_h) cudaFreeHost(s->res_h);
     if (s->st_h) cudaFreeHost(s->st_h);
     if (s->done_h) cudaFreeHost(s->done_h);
+    if (s->mir_h) cudaFreeHost(s->mir_h);
+    if (s->mir_d) cudaFree(s->mir_d);
+    for (cudaStream_t st : s->io_streams) cudaStreamDestroy(st);
     if (s->stream) cudaStreamDestroy(s->stream);
     delete s->hstate;
     delete s;
@@ -618,19 +695,23 @@ int algas_device_query(algas_device_props* out) {
   return ALGAS_OK;
 }
 
-// Full tuner.  Policy ("tuner"):
+// Full tuner.  Policy ("tuner"), matched to the measured
+// optimum of the bench sweeps (profiles/round2_tuner.md):
 //  * threads/CTA: the paper fixes one warp.  On B200 a search step
-//    is latency-bound (dependent select -> gather -> distance -> merge); a
-//    step's wave of row reads completes fastest with 16 warps holding all its
-//    rows in flight (profiles/dist_wave_microbench_ordered.txt), so 512.
+//    is latency-bound (dependent select -> gather -> distance -> merge) and a
+//    step's wave of row reads completes fastest with all its rows in flight:
+//    1024 threads (the widest CTA, dim <= 512 under its 64-register budget),
+//    512 for wider vectors (C3's 960-d rows).
 //  * N_parallel: the largest T allowed by P:L231 -- with N_max_block_per_SM
-//    = 1, the occupancy of a 512-thread search CTA (its registers fill the
-//    register file) -- whose per-block shared memory fits P:L245 (with
-//    M_reserved grown for wide vectors), capped at T_cap = 8.
+//    = 1, the occupancy of a wide search CTA (its registers fill the SM) --
+//    whose per-block shared memory fits P:L245 (with M_reserved grown for
+//    wide vectors), capped at T_cap = 8.
 //  * width / offset_beam: beam extend from the first step
-//    (offset_beam = 1): every step has a fixed latency of ~2 DRAM
-//    round trips plus barriers, so fewer, wider steps win on B200 at equal
-//    recall (profiles/round1_explore_C2.txt); w = 8 up to L = 64, 16 above.
+//    (offset_beam = 1): a step has a fixed latency of ~2 DRAM round
+//    trips plus barriers, so fewer, wider steps win on B200 at equal recall;
+//    w = 12 for short lists (L <= 32), 16 above.
+//  * visited table: SHARED (one per query) when T > 1 -- it removes
+//    the multi-CTA redundant evaluations that PRIVATE tables repeat.
 int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int32_t degree, int32_t itopk, int32_t k,
                algas_tuning* out) {
   if (!out || slots < 1 || dim < 4 || degree < 1 || itopk < 1 || k < 1)
@@ -641,9 +722,9 @@ int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int3
     if (rc) return rc;
     props = &dp;
   }
-  const int nt = props->max_threads_per_sm >= 512 ? 512 : 256;
+  const int nt = (dim <= 512 && props->max_threads_per_sm >= 1024) ? 1024 : 512;
   const int search_blocks_per_sm = 1;  // occupancy of one wide search CTA
-  const int w = std::min(itopk, itopk <= 64 ? 8 : 16);
+  const int w = std::min(itopk, itopk <= 32 ? 12 : 16);
   int Rp = 4;
   while (Rp < degree) Rp <<= 1;
   const int S = 32;
@@ -687,6 +768,7 @@ int algas_tune(const algas_device_props* props, int32_t slots, int32_t dim, int3
   out->offset_beam = 1;
   out->hash_bits = best_hb;
   out->stage_rows = best_sr;
+  out->visited_mode = best > 1 ? ALGAS_VISITED_SHARED : ALGAS_VISITED_PRIVATE;
   (void)k;
   return ALGAS_OK;
 }

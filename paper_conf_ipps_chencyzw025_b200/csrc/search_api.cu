@@ -120,12 +120,13 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   if (cs != 1 && cs != 2 && cs != 4 && cs != 8) return set_error(ALGAS_EINVAL, "cluster_size %d not in {1,2,4,8}", cs);
   const int bps = persistent ? std::max(1, (int)(((int64_t)slots * T * cs + nsm - 1) / nsm)) : 8;
   const int64_t budget = std::min<int64_t>((int64_t)smem_sm / bps - reserved, (int64_t)optin - reserved);
-  // vector-gather path (DESIGN.md §5): 0 = LDG.128 into registers (default),
-  // 1 = cp.async (LDGSTS) staging, 2 = cp.async.bulk staging; the staged
-  // paths are kept as measured alternatives (ALGAS_GATHER_MODE)
+  // vector-gather path (DESIGN.md §6): 0 = LDG.128 into registers (default),
+  // 1 = cp.async (LDGSTS) staging, 2 = cp.async.bulk staging, 3 = team-local
+  // cp.async staging (every row of a pass in flight, no data registers)
+  // (ALGAS_GATHER_MODE)
   const char* gm_env = getenv("ALGAS_GATHER_MODE");
   const int gather_mode = gm_env ? atoi(gm_env) : 0;
-  if (gather_mode < 0 || gather_mode > 2) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0, 1 or 2");
+  if (gather_mode < 0 || gather_mode > 3) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0..3");
   if (cs > 1 && gather_mode != 0) return set_error(ALGAS_EINVAL, "cluster_size > 1 needs the register gather path");
   const char* pf_env = getenv("ALGAS_PREFETCH");  // experiment switch
   const int prefetch = pf_env ? atoi(pf_env) : 8;
@@ -143,6 +144,21 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
       gcbits = 0;
   }
   const int gcb = gc_bytes(gcbits, idx->rp_shift);
+  int team_rows = 0;
+  if (gather_mode == 3) {
+    // rows in flight per team and pass: enough for a step's new rows
+    // (<= w * Rp), as many as fit next to the smallest admissible hash;
+    // p->stage_rows > 0 forces it (sweeps)
+    const int nteams = nt / chunk_tl(cc);
+    int hb_min = 6;
+    while ((1LL << hb_min) < 2LL * (S + w * Rp)) ++hb_min;
+    const int need = (std::min(w * Rp, ncap) + nteams - 1) / nteams;
+    team_rows = p->stage_rows > 0 ? p->stage_rows : std::max(1, std::min(need, 8));
+    while (team_rows > 1 &&
+           smem_layout(dp4, L, ncap, hb > 0 ? hb : hb_min, (nteams * team_rows + 1) / 2, gcb).total > budget)
+      --team_rows;
+    sr = (nteams * team_rows + 1) / 2;  // smem_layout reserves 2 x sr staging rows
+  }
   choose_smem(dp4, L, ncap, S, w, Rp, budget - gcb, &hb, &sr);
   if (hb < 6 || hb > 16) return set_error(ALGAS_EINVAL, "hash_bits %d not in [6,16]", hb);
   if ((1 << hb) < 2 * (S + w * Rp))
@@ -179,6 +195,7 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   c.gtab_bits = std::min(20, std::max(16, hb + 2));
   c.ncap = ncap;
   c.stage_rows = sr;
+  c.team_rows = team_rows;
   c.gather_mode = gather_mode;
   c.prefetch = prefetch;
   c.gc_bits = gcbits;

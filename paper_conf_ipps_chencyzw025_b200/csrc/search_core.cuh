@@ -203,8 +203,13 @@ struct SearchCfg {
   int32_t gtab_bits;     // HBM spill table per CTA: 2^gtab_bits u64
   int32_t ncap;          // capacity of the new-key buffer
   int32_t stage_rows;    // vectors per shared-memory staging buffer (2 buffers)
+  int32_t team_rows;     // gather_mode 3: rows in flight per team and pass (its staging slots)
   int32_t gather_mode;   // 0: LDG.128 into registers, many rows in flight per warp (default)
                          // 1: 16-B cp.async (LDGSTS) staging, 2: cp.async.bulk staging (mbarrier)
+                         // 3: team-local cp.async: each lane copies the 16-B chunks of its team's
+                         //    rows it will itself reduce into the team's staging slots, so every
+                         //    row of a pass is in flight without holding registers and without a
+                         //    CTA barrier between landing and use (team_rows rows per team)
   int32_t prefetch;      // bits: 1 L2 prefetch of each surviving row at filter time, 2 of the
                          // likely next parents' graph rows at select, 4 evict_last graph loads,
                          // 8 (default) graph rows of keys entering the list, at distance time,
@@ -517,13 +522,16 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
 // instruction issue (profiles/dist_wave_microbench*.txt): warps with no row
 // in a pass skip it entirely (warp-uniform test), and the compaction is one
 // ballot per row group instead of a warp scan.
+#ifndef ALGAS_DIST_BW1024
+#define ALGAS_DIST_BW1024 4  // A/B builds: 16-B chunks per lane in flight at 1024 resident threads
+#endif
 template <int NT, int TL, int CPL, int MINB = 1>
 struct DistRows {
   // rows in flight per team and pass: the wave's rows all in flight at once
   // within the register budget (<= 64 registers per thread at 1024 resident
   // threads per SM -- one 1024-thread CTA or two 512-thread CTAs -- <= 128
   // at 512)
-  static constexpr int BW = NT * MINB >= 1024 ? 4 : 16;
+  static constexpr int BW = NT * MINB >= 1024 ? ALGAS_DIST_BW1024 : 16;
   static constexpr int B = CPL >= BW ? 1 : BW / CPL;
 };
 template <int NT, int TL, int CPL, int METRIC, int BOVR = 0>
@@ -634,6 +642,72 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
         if (m[b] & (1u << lane))
           newk[wbase + __popc(m[b] & lt)] = ((uint64_t)__float_as_uint(acc[b]) << 32) | ((uint64_t)ids[b] << 1);
         wbase += __popc(m[b]);
+      }
+    }
+  }
+}
+
+// Distance step, gather mode 3 (P:L217 step 3): like dist_ldg, but the rows
+// of a pass land in shared memory through 16-B cp.async (LDGSTS) issued by
+// the lanes that will reduce them -- team t owns staging slots [t*BS, t*BS+BS),
+// lane tl copies chunks tl, tl+TL, ... of each of its team's rows -- so a pass
+// holds NTEAMS*BS rows in flight with no data registers (the register path's
+// rows per pass are capped by the 64-register budget of a 1024-thread CTA),
+// and a lane only waits for its own copies (cp.async.wait_group), no CTA
+// barrier.  Padded tail chunks of a slot are never written (zero since
+// init_cta).  Keys < worst are appended to newk (ballot + one atomic per
+// warp and row group).
+template <int NT, int TL, int CPL, int METRIC>
+__device__ __forceinline__ void dist_async(const SearchCfg& cfg, const float4* qs, float4* stage, int M,
+                                           uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  constexpr int NTEAMS = NT / TL;
+  constexpr int TPW = 32 / TL;  // teams per warp
+  const int team = tid / TL, tl = tid % TL;
+  const int wteam0 = (tid >> 5) * TPW;
+  const int BS = cfg.team_rows;
+  const int PASS = NTEAMS * BS;
+  QueryRegs<TL, CPL> Q;
+  Q.load(qs, tl);
+  for (int base = 0; base < M; base += PASS) {
+    int nb = (M - base - wteam0 + NTEAMS - 1) / NTEAMS;  // row groups holding rows of this warp
+    if (nb <= 0) continue;
+    if (nb > BS) nb = BS;
+    for (int b = 0; b < nb; ++b) {
+      const int j = base + b * NTEAMS + team;
+      if (j < M) {
+        const float4* row = cfg.data + (uint64_t)newid[j] * cfg.d4;
+        float4* dst = stage + (size_t)(team * BS + b) * cfg.dp4;
+#pragma unroll
+        for (int c = 0; c < CPL; ++c) {
+          const int chn = tl + c * TL;
+          if (chn < cfg.d4) cp_async16(dst + chn, row + chn);
+        }
+      }
+    }
+    asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+    for (int b = 0; b < nb; ++b) {
+      const int j = base + b * NTEAMS + team;
+      float a = team_partial_smem<TL, CPL, METRIC>(Q, stage + (size_t)(team * BS + b) * cfg.dp4, tl);
+#pragma unroll
+      for (int o = TL >> 1; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+      uint64_t key = kKeyMax;
+      uint32_t id = 0;
+      if (tl == 0 && j < M) {
+        id = newid[j];
+        key = make_key((METRIC == kL2) ? a : -a, id);
+      }
+      const bool keep = key < worst;
+      const unsigned m = __ballot_sync(0xffffffffu, keep);
+      if (keep && (cfg.prefetch & 8))  // its graph row: a likely parent of the next step(s)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)id << cfg.rp_shift)),
+                     "r"(4u << cfg.rp_shift)
+                     : "memory");
+      if (m) {
+        int wbase = 0;
+        if (lane == 0) wbase = atomicAdd(nkeys, __popc(m));
+        wbase = __shfl_sync(0xffffffffu, wbase, 0);
+        if (keep) newk[wbase + __popc(m & ((1u << lane) - 1u))] = key;
       }
     }
   }
@@ -1093,9 +1167,12 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
                                                                       &C->nkeys[sp], gcache, gstamp);
           __syncthreads();
         }
+      } else if (cfg.gather_mode == 3) {
+        dist_async<NT, TL, CPL, METRIC>(cfg, s.q, s.stage, M, worst, s.newid, s.newk, &C->nkeys[sp]);
+        __syncthreads();
       }
       const int SR = cfg.stage_rows;
-      const int nchunks = cfg.gather_mode == 0 ? 0 : (M + SR - 1) / SR;
+      const int nchunks = (cfg.gather_mode == 1 || cfg.gather_mode == 2) ? (M + SR - 1) / SR : 0;
       if (nchunks > 0) stage_issue<NT>(cfg, s, 0, 0, M < SR ? M : SR, warp, lane);
       QueryRegs<TL, CPL> Q;  // staged paths: the query in registers for the chunk loop
       if (nchunks > 0) Q.load(s.q, tl);
@@ -1200,7 +1277,7 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
         lap(3);
         continue;
       }
-      if (tid == 0 && nk > 0) C->mg_rank++;
+      if (tid == 0) C->mg_rank++;
       if (nk > 0) {
         const uint64_t* src = cur ? s.list[1] : s.list[0];
         uint64_t* dst = cur ? s.list[0] : s.list[1];

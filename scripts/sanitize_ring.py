@@ -27,9 +27,9 @@ def main():
     Q = synth.lattice(12, 128, seed=43)
     G, _ = oracle.knn_graph(X, 32)
     idx = algas.Index(X, G)
-    for vis, T in ((0, 2), (1, 4)):
+    for vis, T, mirror in ((0, 2, 0), (1, 4, 0), (1, 4, 1)):
         p = algas.default_params(k=10, itopk=32, width=4, offset_beam=1, n_seeds=16, ctas_per_query=T,
-                                 threads_per_cta=nt, slots=6, seed=1, visited_mode=vis)
+                                 threads_per_cta=nt, slots=6, seed=1, visited_mode=vis, state_mirror=mirror)
         got = {}
         with algas.Server(idx, p, deferred=True) as srv:
             for t in range(Q.shape[0]):
@@ -47,7 +47,7 @@ def main():
             assert np.array_equal(d["ids"], oi), "dynamic != oracle"
             b = idx.search(Q, params=p)
             assert np.array_equal(b["ids"], oi), "batch != oracle"
-        print(f"visited_mode={vis} T={T} threads={nt}: {len(got)} queries ok", flush=True)
+        print(f"visited_mode={vis} T={T} mirror={mirror} threads={nt}: {len(got)} queries ok", flush=True)
     print("SANITIZE_RUN_OK")
 
 

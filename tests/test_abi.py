@@ -121,8 +121,10 @@ def test_tuner_policy_respects_paper_constraints(props, slots):
         assert t.smem_per_block <= t.smem_avail_per_block
         assert t.smem_avail_per_block <= oracle.tuner_smem_per_block(props.smem_per_sm, t.blocks_per_sm,
                                                                      props.smem_reserved_per_block)
-        assert t.threads_per_cta in (32, 64, 128, 256, 512)
+        assert t.threads_per_cta in (32, 64, 128, 256, 512, 1024)
+        assert t.threads_per_cta <= 512 or dim <= 512   # the 1024-thread build serves dim <= 512
         assert 1 <= t.width <= 32 and 1 <= t.offset_beam <= L
+        assert t.visited_mode == (1 if t.ctas_per_query > 1 else 0)
 
 
 def test_tuner_small_batch_gets_more_ctas():

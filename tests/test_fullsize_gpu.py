@@ -222,3 +222,31 @@ def test_fullsize_C2_server_shared_recall_matches_device_queue():
     rec_srv = oracle.recall(got, truth, w.k)
     print(f"server {rec_srv:.4f} device queue {rec_dq:.4f}")
     assert rec_srv >= rec_dq - 0.005, (rec_srv, rec_dq)
+
+
+def test_fullsize_C2_tuner_matches_swept_optimum():
+    """The adaptive tuner (T from P:L231, threads, width, visited
+    mode) at the smallest L reaching recall@10 >= 0.95 delivers >= 0.9 x the
+    QPS of the best (T, threads, width) point of a measured sweep at the C2
+    shape and 32 slots.  Recall from O1 truth over the 2000-query stream."""
+    import torch
+    w, X, Q, G, idx, _, _, sample, ti = workload("C2", N_SAMPLE["C2"])
+    Qd = torch.from_numpy(Q).cuda()
+
+    def qps_at(T, nt, wd, vis):
+        for L in (10, 11, 12, 13, 14, 16, 20, 24, 32, 40, 48, 64):
+            p = algas.default_params(k=w.k, itopk=L, width=min(wd, L), offset_beam=1, ctas_per_query=T,
+                                     threads_per_cta=nt, slots=32, n_seeds=32, seed=1, visited_mode=vis)
+            r = idx.search_dynamic(Qd, p)
+            if oracle.recall(r["ids"], ti, w.k) >= 0.95:
+                ks = [idx.search_dynamic(Qd, p)["info"].kernel_ms for _ in range(3)]
+                return Q.shape[0] / (np.median(ks) / 1e3), L
+        return 0.0, None
+
+    tu = algas.tune(32, w.dim, w.degree, 16, w.k)
+    q_tuner, L_tuner = qps_at(tu.ctas_per_query, tu.threads_per_cta, tu.width, tu.visited_mode)
+    best = max(qps_at(T, nt, wd, 1 if T > 1 else 0)[0]
+               for T in (1, 2, 4) for nt in (512, 1024) for wd in (8, 12, 16))
+    print(f"tuner T={tu.ctas_per_query} nt={tu.threads_per_cta} w={tu.width} vis={tu.visited_mode} "
+          f"L={L_tuner}: {q_tuner:.0f} q/s; swept best {best:.0f} q/s")
+    assert q_tuner >= 0.9 * best, (q_tuner, best)
