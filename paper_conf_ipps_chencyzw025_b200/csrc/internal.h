@@ -41,6 +41,11 @@ struct Workspace {
   // counters, control block, SHARED bitmaps): no allocation per call
   void* d_scratch[4] = {nullptr, nullptr, nullptr, nullptr};
   size_t d_scratch_bytes[4] = {0, 0, 0, 0};
+  // host-mapped per-CTA results / counters / Finish words of the dynamic
+  // path's streaming merge (grow-only)
+  void* m_buf = nullptr;
+  size_t m_bytes = 0;
+  uint32_t call_id = 0;
 };
 
 }  // namespace algas
@@ -139,6 +144,11 @@ struct PersistArgs {
   int* queue_head;
   ResultEntry* dq_res;      // nq x T x kmax
   CtaStats* dq_stats;       // nq x T
+  // streaming merge (host-mapped dq_res / dq_stats): per (query, CTA) Finish
+  // word set to call_id with a system-scope release once its list and
+  // counters are written, so the host merges a query while the kernel runs
+  uint32_t* dq_done;        // nq x T, or null
+  uint32_t call_id;
   // host ring (mapped pointers)
   RingSlot* ring;
   const float4* ring_q;     // slots x d4

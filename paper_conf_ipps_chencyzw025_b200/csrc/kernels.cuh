@@ -324,6 +324,12 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       if (P.mode == 0) {
         __threadfence_system();
         st_release_sys(P.ring_done + (uint64_t)(2 * slot + sub) * P.T + rank, epoch);
+      } else if (P.dq_done) {
+        // streaming merge: this (query, CTA)'s list and counters are in host
+        // memory (written by the CTA's threads before the barrier above);
+        // release them to the host thread merging while the kernel runs
+        __threadfence_system();
+        st_release_sys(P.dq_done + (uint64_t)item * P.T + rank, P.call_id);
       } else {
         __threadfence();
       }

@@ -496,6 +496,7 @@ int algas_index_destroy(algas_index* idx) {
     if (idx->ws->counters) cudaFree(idx->ws->counters);
     if (idx->ws->h_res) cudaFreeHost(idx->ws->h_res);
     if (idx->ws->h_st) cudaFreeHost(idx->ws->h_st);
+    if (idx->ws->m_buf) cudaFreeHost(idx->ws->m_buf);
     for (void* p : idx->ws->d_scratch)
       if (p) cudaFree(p);
     delete idx->ws;
@@ -652,12 +653,86 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
     pa.vbm = (uint32_t*)vbp;
   }
   mark("alloc");
+  const size_t res_bytes = (size_t)items * pl.k * sizeof(ResultEntry), st_bytes = (size_t)items * sizeof(CtaStats);
+  // Streaming merge (GPU-CPU cooperation): with host outputs the
+  // CTAs write their lists and counters straight into host-mapped memory and
+  // raise a per-(query, CTA) Finish word; this thread merges each query the
+  // moment its T lists are in, while the kernel keeps running -- the host
+  // merge overlaps the search instead of following it.
+  const bool stream_merge = !is_device_ptr(out_ids) && !is_device_ptr(out_dists) && getenv("ALGAS_NO_STREAM_MERGE") == nullptr;
+  ResultEntry* mres = nullptr;
+  CtaStats* mst = nullptr;
+  uint32_t* mdone = nullptr;
+  if (stream_merge) {
+    const size_t done_bytes = (size_t)items * 4;
+    const size_t need = res_bytes + st_bytes + done_bytes + 256;
+    if (ws->m_bytes < need) {
+      if (ws->m_buf) cudaFreeHost(ws->m_buf);
+      ws->m_buf = nullptr;
+      ws->m_bytes = 0;
+      ALGAS_CUDA_TRY(cudaHostAlloc(&ws->m_buf, need, cudaHostAllocMapped | cudaHostAllocPortable));
+      memset(ws->m_buf, 0, need);
+      ws->m_bytes = need;
+    }
+    uint8_t* hb = (uint8_t*)ws->m_buf;
+    uint8_t* db = nullptr;
+    ALGAS_CUDA_TRY(cudaHostGetDevicePointer((void**)&db, ws->m_buf, 0));
+    const size_t o_st = (res_bytes + 127) & ~(size_t)127, o_done = (o_st + st_bytes + 127) & ~(size_t)127;
+    mres = (ResultEntry*)hb;
+    mst = (CtaStats*)(hb + o_st);
+    mdone = (uint32_t*)(hb + o_done);
+    pa.dq_res = (ResultEntry*)db;
+    pa.dq_stats = (CtaStats*)(db + o_st);
+    pa.dq_done = (uint32_t*)(db + o_done);
+    pa.call_id = ++ws->call_id;
+    if (pa.call_id == 0) pa.call_id = ++ws->call_id;  // 0 = never written
+  }
   EventTimer tm(st);
   if ((rc = tm.start())) return rc;
   if ((rc = launch_persistent(pl, pa, st))) return rc;
   if ((rc = tm.stop())) return rc;
   mark("launch");
-  const size_t res_bytes = (size_t)items * pl.k * sizeof(ResultEntry), st_bytes = (size_t)items * sizeof(CtaStats);
+  if (stream_merge) {
+    const auto t_merge = std::chrono::steady_clock::now();
+    bool ovf = false;
+    const uint32_t cid = pa.call_id;
+    const int T = pl.T, k = pl.k;
+    int spins = 0;
+    for (int64_t q = 0; q < nq; ++q) {
+      for (int c = 0; c < T; ++c) {
+        while (__atomic_load_n(mdone + q * T + c, __ATOMIC_ACQUIRE) != cid) {
+          if (++spins >= 4096) {  // a failed kernel is reported, not waited on
+            spins = 0;
+            const cudaError_t e = cudaStreamQuery(st);
+            if (e != cudaSuccess && e != cudaErrorNotReady)
+              return set_error(ALGAS_ECUDA, "search kernel failed: %s", cudaGetErrorString(e));
+            if (e == cudaSuccess && __atomic_load_n(mdone + q * T + c, __ATOMIC_ACQUIRE) != cid)
+              return set_error(ALGAS_ECUDA, "search kernel finished without publishing query %lld", (long long)q);
+          }
+        }
+      }
+      const ResultEntry* r = mres + (size_t)q * T * k;
+      if (T == 1) {
+        for (int i = 0; i < k; ++i) { out_ids[q * k + i] = r[i].id; out_dists[q * k + i] = r[i].dist; }
+      } else {
+        merge_cta_lists(r, T, k, k, out_ids + q * k, out_dists + q * k);
+      }
+      algas_query_stats qs;
+      aggregate_cta_stats(mst + q * T, T, &qs);
+      if (qs.overflows) ovf = true;
+      if (out_stats) out_stats[q] = qs;
+    }
+    ALGAS_CUDA_TRY(cudaStreamSynchronize(st));
+    ALGAS_CUDA_TRY(cudaGetLastError());
+    mark("merge");
+    if (info) {
+      fill_info(info, pl, ctas, tm.ms());
+      const auto t_end = std::chrono::steady_clock::now();
+      info->merge_ms = std::chrono::duration<float, std::milli>(t_end - t_merge).count();
+      info->call_ms = std::chrono::duration<float, std::milli>(t_end - t_entry).count();
+    }
+    return ovf ? set_error(ALGAS_EOVERFLOW, "a visited table overflowed") : ALGAS_OK;
+  }
   if ((rc = ensure_pinned(idx->ws, res_bytes, st_bytes))) return rc;
   ResultEntry* res = (ResultEntry*)idx->ws->h_res;
   CtaStats* cst = (CtaStats*)idx->ws->h_st;
