@@ -384,12 +384,23 @@ int algas_build_graph(const float *data, int64_t n, int32_t dim, int32_t metric,
  * [1, n_clusters], bad dim/metric. */
 int algas_knn_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric, int32_t k,
                           int32_t n_clusters, int32_t overlap, uint32_t *out_ids, float *out_dists);
-/* algas_build_graph with algas_knn_partitioned as its kNN step; rows the
+/* Neighbour-of-neighbour refinement of an approximate kNN list (DESIGN.md
+ * R33, the NN-descent step; not in the paper): `rounds` Jacobi rounds, each
+ * giving every point p the first k by (dist, id) of its list and the
+ * distances to the ids found in the first `fan` entries of the lists of its
+ * first `fan` neighbours (p and ids already listed excluded).  ids / dists:
+ * n x k in/out (rows sorted by (dist, id), SENTINEL / +inf padded), host or
+ * device.  EINVAL: fan outside [1, min(k, 64)], k > 1024, bad dim/metric. */
+int algas_knn_refine(const float *data, int64_t n, int32_t dim, int32_t metric, int32_t k, int32_t fan,
+                     int32_t rounds, uint32_t *ids, float *dists);
+/* algas_build_graph with algas_knn_partitioned (+ refine_rounds rounds of
+ * algas_knn_refine with refine_fan, 0 = none) as its kNN step; rows the
  * partition left short (clusters of <= knn_degree points) are completed
  * with the exact kNN of those rows over the whole set before the prune. */
 int algas_build_graph_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric,
                                   int32_t knn_degree, int32_t degree, int32_t prune,
-                                  int32_t n_clusters, int32_t overlap, uint32_t *out_graph);
+                                  int32_t n_clusters, int32_t overlap, int32_t refine_fan,
+                                  int32_t refine_rounds, uint32_t *out_graph);
 
 #if defined(__GNUC__)
 #pragma GCC visibility pop

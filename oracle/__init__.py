@@ -26,6 +26,9 @@ Parity status per function:
     build algorithm in it); pinned by m = 1 / overlap = m == O1 and two
     hand-worked 1-d examples, one where a Lloyd move and the capacity bound
     (4c < m) each change a cluster.
+  * orc_knn_refine (f4, R33)               parity unpinned by the paper; pinned
+    by its fixed point (an exact kNN list is unchanged), a hand-worked 1-d
+    example and monotonicity (no row's k-th distance grows).
   * orc_prune (K10)                        parity unpinned by the paper (the
     CAGRA algorithm is only cited); pinned by a hand-worked
     example and invariants.
@@ -112,6 +115,8 @@ def lib():
             L.orc_tuner_smem_per_block.restype = i64
             L.orc_prune.argtypes = [P, i64, i32, i32, P, P]
             L.orc_prune.restype = i32
+            L.orc_knn_refine.argtypes = [P, i64, i32, i32, i32, i32, P, P, P, P]
+            L.orc_knn_refine.restype = i32
             _lib = L
     return _lib
 
@@ -218,6 +223,22 @@ def knn_partitioned(X, k: int, n_clusters: int, overlap: int, metric: int = L2):
     ds = np.empty((n, k), np.float32)
     for i in range(n):
         ids[i], ds[i], _ = merge_topk(cand_i[i], cand_d[i], k)
+    return ids, ds
+
+
+def knn_refine(X, ids, ds, fan: int, rounds: int = 1, metric: int = L2):
+    """R33: `rounds` neighbour-of-neighbour refinement rounds (orc_knn_refine,
+    each a Jacobi round over the previous round's lists)."""
+    X = _f32(X)
+    ids, ds = _u32(ids).copy(), _f32(ds).copy()
+    n, k = ids.shape
+    for _ in range(rounds):
+        oi = np.empty_like(ids)
+        od = np.empty_like(ds)
+        rc = lib().orc_knn_refine(_ptr(X), n, X.shape[1], metric, k, fan, _ptr(ids), _ptr(ds), _ptr(oi), _ptr(od))
+        if rc != 0:
+            raise RuntimeError("orc_knn_refine failed")
+        ids, ds = oi, od
     return ids, ds
 
 

@@ -27,6 +27,11 @@
  *   orc_merge_topk   (A9)             host priority-queue merge
  *   orc_tuner_*                       adaptive tuning equations (P:L231,
  *                                     P:L235)
+ *   orc_knn_refine   (f4, R33)        one neighbour-of-neighbour refinement
+ *                                     round of an approximate kNN list
+ *                                     (R33; not in the paper:
+ *                                     parity unpinned by it, pinned by its
+ *                                     exact fixed point and a hand example)
  *   orc_prune        (K10)            CAGRA-style rank-based detour pruning +
  *                                     reverse edges (graph named at P:L293,
  *                                     algorithm from ref [25] P:L430, which is
@@ -514,5 +519,66 @@ int32_t orc_prune(const uint32_t *knn, int64_t n, int32_t K, int32_t R, uint32_t
         free(fill);
     }
     free(rev); free(P); free(e); free(nrev);
+    return 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* f4 reading R33: one neighbour-of-neighbour refinement round of an      */
+/* approximate kNN list (the NN-descent step).  For every point p, in     */
+/* id order, from the INPUT lists only (a Jacobi round):                  */
+/*   C(p) = { x = in[q][b] : q = in[p][a], a < fan, b < fan,              */
+/*            x != SENTINEL, x != p, x not in in[p] }, each x once        */
+/*   out[p] = first k of sort_by_(dist,id)( in[p] u {(F(p,x), x) : x in C} ) */
+/*   padded with (SENTINEL, +inf).  F is orc_distance.            */
+/* in/out: n x k, rows sorted by (dist, id), SENTINEL-padded.            */
+/* Returns 0, or -1 on bad arguments / allocation failure.               */
+/* ------------------------------------------------------------------ */
+int32_t orc_knn_refine(const float *X, int64_t n, int32_t d, int32_t metric, int32_t k, int32_t fan,
+                       const uint32_t *ids_in, const float *d_in, uint32_t *ids_out, float *d_out)
+{
+    uint8_t *mark;
+    orc_cand *c;
+    int64_t p;
+    int32_t a, b, i, m;
+    if (n < 1 || k < 1 || fan < 1 || fan > k) return -1;
+    mark = (uint8_t *)calloc((size_t)((n + 7) / 8), 1);
+    c = (orc_cand *)malloc(sizeof(orc_cand) * (size_t)(k + fan * fan));
+    if (!mark || !c) { free(mark); free(c); return -1; }
+    for (p = 0; p < n; p++) {
+        m = 0;
+        bm_set(mark, (uint32_t)p);
+        for (i = 0; i < k; i++) {             /* the current list */
+            uint32_t x = ids_in[p * k + i];
+            if (x == ORC_SENTINEL) continue;
+            bm_set(mark, x);
+            c[m].dist = d_in[p * k + i];
+            c[m].id = x;
+            c[m].checked = 0;
+            m++;
+        }
+        for (a = 0; a < fan; a++) {           /* neighbours of its first fan neighbours */
+            uint32_t q = ids_in[p * k + a];
+            if (q == ORC_SENTINEL) continue;
+            for (b = 0; b < fan; b++) {
+                uint32_t x = ids_in[(int64_t)q * k + b];
+                if (x == ORC_SENTINEL || bm_test(mark, x)) continue;
+                bm_set(mark, x);
+                c[m].dist = orc_distance(X + p * (int64_t)d, X + (int64_t)x * d, d, metric);
+                c[m].id = x;
+                c[m].checked = 0;
+                m++;
+            }
+        }
+        qsort(c, (size_t)m, sizeof(orc_cand), cand_cmp);
+        for (i = 0; i < k; i++) {
+            ids_out[p * k + i] = i < m ? c[i].id : ORC_SENTINEL;
+            d_out[p * k + i] = i < m ? c[i].dist : __builtin_inff();
+        }
+        /* clear the marks of this point */
+        mark[p >> 3] = 0;
+        for (i = 0; i < m; i++) mark[c[i].id >> 3] = 0;
+    }
+    free(mark);
+    free(c);
     return 0;
 }

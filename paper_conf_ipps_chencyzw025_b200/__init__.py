@@ -28,7 +28,7 @@ VISITED_SHARED = 1
 OK, EINVAL, ENOMEM, ECUDA, EAGAIN, ESTATE, ENCCL, EOVERFLOW = 0, -1, -2, -3, -4, -5, -6, -7
 
 __all__ = ["Index", "Server", "Params", "QueryStats", "RunInfo", "lib", "knn", "prune", "build_graph",
-           "merge_topk", "merge_topk_parts", "knn_partitioned", "build_graph_partitioned", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP", "COSINE"]
+           "merge_topk", "merge_topk_parts", "knn_partitioned", "build_graph_partitioned", "knn_refine", "tune", "device_props", "AlgasError", "SENTINEL", "L2", "IP", "COSINE"]
 
 
 class AlgasError(RuntimeError):
@@ -96,7 +96,7 @@ EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_i
            "algas_server_create", "algas_server_create_deferred", "algas_server_start", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
-           "algas_build_graph", "algas_knn_partitioned", "algas_build_graph_partitioned"]
+           "algas_build_graph", "algas_knn_partitioned", "algas_build_graph_partitioned", "algas_knn_refine"]
 
 _lock = threading.Lock()
 _lib = None
@@ -159,7 +159,8 @@ def lib(build_if_missing: bool = True):
         L.algas_prune.argtypes = [P, i64, i32, i32, P]
         L.algas_build_graph.argtypes = [P, i64, i32, i32, i32, i32, i32, P]
         L.algas_knn_partitioned.argtypes = [P, i64, i32, i32, i32, i32, i32, P, P]
-        L.algas_build_graph_partitioned.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i32, P]
+        L.algas_build_graph_partitioned.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i32, i32, i32, P]
+        L.algas_knn_refine.argtypes = [P, i64, i32, i32, i32, i32, i32, P, P]
         _lib = L
         return L
 
@@ -402,15 +403,26 @@ def knn_partitioned(data, k: int, n_clusters: int, overlap: int = 2, metric: int
 
 
 def build_graph_partitioned(data, degree: int, n_clusters: int, overlap: int = 2, knn_degree: int | None = None,
-                            metric: int = L2, prune: bool = True):
-    """algas_build_graph_partitioned: partitioned kNN + the same prune as build_graph."""
+                            metric: int = L2, prune: bool = True, refine_fan: int = 16, refine_rounds: int = 0):
+    """algas_build_graph_partitioned: partitioned kNN (+ refinement rounds) + the same prune as build_graph."""
     n, dim = int(data.shape[0]), int(data.shape[1])
     kd = knn_degree if knn_degree is not None else 2 * degree
     out = np.empty((n, degree), np.uint32)
     dp, _a = _ptr(data)
     _check(lib().algas_build_graph_partitioned(dp, n, dim, metric, kd, degree, 1 if prune else 0, n_clusters,
-                                               overlap, _ptr(out)[0]))
+                                               overlap, refine_fan, refine_rounds, _ptr(out)[0]))
     return out
+
+
+def knn_refine(data, ids, dists, fan: int, rounds: int = 1, metric: int = L2):
+    """algas_knn_refine: neighbour-of-neighbour refinement rounds (R33); returns new (ids, dists)."""
+    n, dim = int(data.shape[0]), int(data.shape[1])
+    ids = ids.clone() if _is_torch(ids) else np.array(ids, np.uint32, copy=True)
+    dists = dists.clone() if _is_torch(dists) else np.array(dists, np.float32, copy=True)
+    k = int(ids.shape[1])
+    dp, _a = _ptr(data)
+    _check(lib().algas_knn_refine(dp, n, dim, metric, k, fan, rounds, _ptr(ids)[0], _ptr(dists)[0]))
+    return ids, dists
 
 
 def knn_last_stats():

@@ -8,6 +8,7 @@
 #include <cstdint>
 #include <mutex>
 #include <string>
+#include <vector>
 
 #include "../../include/algas.h"
 #include "search_core.cuh"
@@ -232,6 +233,19 @@ inline void aggregate_cta_stats(const CtaStats* cs, int T, algas_query_stats* q)
   q->t_start_ns = t0 == ~0ull ? 0 : t0;
   q->t_end_ns = t1;
 }
+
+// partitioned graph build (build_part.cu, R30 / R33)
+struct ClusterBlock {
+  int32_t cluster;  // a CTA of the batched cluster kNN: 64 member rows of one cluster
+  int32_t row0;
+};
+int launch_cluster_knn(const float* X, int d, int metric, const uint32_t* mem, const int64_t* start,
+                       const std::vector<ClusterBlock>& blocks, int k, uint64_t* out);
+int launch_merge_lists(const uint64_t* lists, const uint32_t* slot_of, int64_t n, int c, int k, uint32_t* out_ids,
+                       float* out_d);
+int launch_refine(const float* X, int d, int metric, int64_t n, int k, int fan, const uint32_t* in_ids,
+                  const float* in_d, uint32_t* out_ids, float* out_d);
+constexpr int kPartMaxKnn = 128;  // list length the batched cluster kNN keeps in shared memory
 
 // host TopK merge (runtime.cpp)
 int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t* out_ids, float* out_d);

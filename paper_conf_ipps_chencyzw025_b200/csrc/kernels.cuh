@@ -108,6 +108,9 @@ struct PKArgs {
 };
 
 constexpr unsigned long long kMboxQuit = 0xFFFFFFFFull << 32;
+#ifndef ALGAS_FINISH_FENCE
+#define ALGAS_FINISH_FENCE 0
+#endif
 
 // MINB = resident CTAs per SM the build is for (1, or 2 when a persistent
 // grid of slots x T searches exceeds the SM count: half the registers)
@@ -320,20 +323,28 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     last_epoch = epoch;
     __syncthreads();
     // ---------------- Finish
+    // device-scope finish count, which gates the slot's next pickup: thread 0
     if (tid == 0) {
+      __threadfence();
+      atomicAdd(P.slot_fin + slot, 1u);
+    }
+    // host-visible Finish word: the CTA's list and counters (written by its
+    // threads before the barrier above) are released at system scope -- the
+    // ring's per-CTA Finish flag, or the streaming merge's (query, CTA) word.
+    // Issued by the LAST warp, so its release overlaps the next pickup
+    // instead of delaying thread 0's polling.  st.release.sys alone orders
+    // the CTA's earlier writes (ordered before it by the barrier, release is
+    // cumulative) before the flag; ALGAS_FINISH_FENCE=1 builds add a full
+    // fence.sc.sys in front (A/B).
+    if (tid == NT - 32) {
+#if ALGAS_FINISH_FENCE
+      if (P.mode == 0 || P.dq_done) __threadfence_system();
+#endif
       if (P.mode == 0) {
-        __threadfence_system();
         st_release_sys(P.ring_done + (uint64_t)(2 * slot + sub) * P.T + rank, epoch);
       } else if (P.dq_done) {
-        // streaming merge: this (query, CTA)'s list and counters are in host
-        // memory (written by the CTA's threads before the barrier above);
-        // release them to the host thread merging while the kernel runs
-        __threadfence_system();
         st_release_sys(P.dq_done + (uint64_t)item * P.T + rank, P.call_id);
-      } else {
-        __threadfence();
       }
-      atomicAdd(P.slot_fin + slot, 1u);  // the slot's rank 0 gates its next pickup on this
     }
     if (P.mode == 0) {  // the slot's next query is in its other ring entry
       if (sub) last_ep1 = epoch; else last_ep0 = epoch;

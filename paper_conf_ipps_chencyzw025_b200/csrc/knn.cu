@@ -886,10 +886,61 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
   }
   int64_t smax = 0;
   for (int64_t j = 0; j < m; ++j) smax = std::max(smax, start[j + 1] - start[j]);
-  // 4. exact kNN inside each cluster (rows gathered contiguously; local id
-  //    order == global id order, so (dist, id) ties resolve as globally)
   ALGAS_CUDA_TRY(cudaMalloc(&hmem.p, std::max<size_t>(mem.size() * 4, 16)));
   ALGAS_CUDA_TRY(cudaMemcpy(hmem.p, mem.data(), mem.size() * 4, cudaMemcpyHostToDevice));
+  if (k <= kPartMaxKnn && getenv("ALGAS_PART_PER_CLUSTER") == nullptr) {
+    // 4+5 on the GPU, all clusters in one launch (build_part.cu): a CTA takes
+    // 64 member rows of one cluster against all its members (fp32 direct
+    // form, running top-k in shared memory; lists keyed by GLOBAL id, so
+    // (dist, id) ties resolve as globally; a cluster of s points yields
+    // min(k, s - 1) entries, the rest padding); then every point merges its
+    // c cluster lists (repeated ids dropped, first k)
+    const float* Xm = X;
+    int met = metric;
+    Dev hxn;
+    if (metric == ALGAS_COSINE) {  // IP on unit-row copies (R29)
+      ALGAS_CUDA_TRY(cudaMalloc(&hxn.p, (size_t)n * dim * 4));
+      normalize_copy_kernel<<<(unsigned)((n + 7) / 8), 256>>>(reinterpret_cast<const float4*>(X), n, dim / 4,
+                                                              reinterpret_cast<float4*>(hxn.p));
+      ALGAS_CUDA_TRY(cudaGetLastError());
+      Xm = (const float*)hxn.p;
+      met = ALGAS_IP;
+    }
+    std::vector<ClusterBlock> blocks;
+    for (int64_t j = 0; j < m; ++j)
+      for (int64_t r0 = 0; r0 < start[j + 1] - start[j]; r0 += 64) blocks.push_back(ClusterBlock{(int32_t)j, (int32_t)r0});
+    std::vector<uint32_t> slot_of((size_t)n * c);
+    for (int64_t j = 0; j < m; ++j)
+      for (int64_t t = start[j]; t < start[j + 1]; ++t) {
+        const uint32_t i = mem[t];
+        int r = 0;
+        while (asg[(size_t)i * c + r] != (uint32_t)j) ++r;
+        slot_of[(size_t)i * c + r] = (uint32_t)t;
+      }
+    Dev hstart, hlists, hslot, hoi, hod;
+    ALGAS_CUDA_TRY(cudaMalloc(&hstart.p, (size_t)(m + 1) * 8));
+    ALGAS_CUDA_TRY(cudaMemcpy(hstart.p, start.data(), (size_t)(m + 1) * 8, cudaMemcpyHostToDevice));
+    ALGAS_CUDA_TRY(cudaMalloc(&hlists.p, std::max<size_t>(mem.size() * (size_t)k * 8, 16)));
+    ALGAS_CUDA_TRY(cudaMalloc(&hslot.p, slot_of.size() * 4));
+    ALGAS_CUDA_TRY(cudaMemcpy(hslot.p, slot_of.data(), slot_of.size() * 4, cudaMemcpyHostToDevice));
+    phase("members");
+    if ((rc = launch_cluster_knn(Xm, dim, met, (const uint32_t*)hmem.p, (const int64_t*)hstart.p, blocks, k,
+                                 (uint64_t*)hlists.p)))
+      return rc;
+    phase("clusters");
+    ALGAS_CUDA_TRY(cudaMalloc(&hoi.p, (size_t)n * k * 4));
+    ALGAS_CUDA_TRY(cudaMalloc(&hod.p, (size_t)n * k * 4));
+    if ((rc = launch_merge_lists((const uint64_t*)hlists.p, (const uint32_t*)hslot.p, n, c, k, (uint32_t*)hoi.p,
+                                 (float*)hod.p)))
+      return rc;
+    phase("merge");
+    ALGAS_CUDA_TRY(cudaMemcpy(out_ids, hoi.p, (size_t)n * k * 4, cudaMemcpyDefault));
+    ALGAS_CUDA_TRY(cudaMemcpy(out_dists, hod.p, (size_t)n * k * 4, cudaMemcpyDefault));
+    return ALGAS_OK;
+  }
+  // 4. exact kNN inside each cluster, one algas_knn call per cluster (k >
+  //    kPartMaxKnn, or ALGAS_PART_PER_CLUSTER): rows gathered contiguously;
+  //    local id order == global id order, so (dist, id) ties resolve as globally
   ALGAS_CUDA_TRY(cudaMalloc(&hB.p, (size_t)smax * dim * 4));
   phase("members");
   std::vector<uint32_t> cand((size_t)n * c * k, kSentinel);
@@ -948,10 +999,48 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
   return ALGAS_OK;
 }
 
+int algas_knn_refine(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t k, int32_t fan,
+                     int32_t rounds, uint32_t* ids, float* dists) {
+  if (!data || !ids || !dists || n < 1 || n >= (1LL << 31) || dim < 4 || dim % 4 != 0 || k < 1 || k > 1024 ||
+      fan < 1 || fan > k || fan > 64 || rounds < 0 || (metric != ALGAS_L2 && metric != ALGAS_IP && metric != ALGAS_COSINE))
+    return set_error(ALGAS_EINVAL, "algas_knn_refine: bad arguments");
+  if (rounds == 0) return ALGAS_OK;
+  Dev hx, hxn, a_i, a_d, b_i, b_d;
+  const float* X = nullptr;
+  int rc;
+  if ((rc = to_device(data, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
+  int met = metric;
+  if (metric == ALGAS_COSINE) {  // IP on unit-row copies (R29)
+    ALGAS_CUDA_TRY(cudaMalloc(&hxn.p, (size_t)n * dim * 4));
+    normalize_copy_kernel<<<(unsigned)((n + 7) / 8), 256>>>(reinterpret_cast<const float4*>(X), n, dim / 4,
+                                                            reinterpret_cast<float4*>(hxn.p));
+    ALGAS_CUDA_TRY(cudaGetLastError());
+    X = (const float*)hxn.p;
+    met = ALGAS_IP;
+  }
+  const size_t bytes = (size_t)n * k * 4;
+  ALGAS_CUDA_TRY(cudaMalloc(&a_i.p, bytes));
+  ALGAS_CUDA_TRY(cudaMalloc(&a_d.p, bytes));
+  ALGAS_CUDA_TRY(cudaMalloc(&b_i.p, bytes));
+  ALGAS_CUDA_TRY(cudaMalloc(&b_d.p, bytes));
+  ALGAS_CUDA_TRY(cudaMemcpy(a_i.p, ids, bytes, cudaMemcpyDefault));
+  ALGAS_CUDA_TRY(cudaMemcpy(a_d.p, dists, bytes, cudaMemcpyDefault));
+  for (int r = 0; r < rounds; ++r) {  // Jacobi rounds (R33)
+    if ((rc = launch_refine(X, dim, met, n, k, fan, (const uint32_t*)a_i.p, (const float*)a_d.p, (uint32_t*)b_i.p,
+                            (float*)b_d.p)))
+      return rc;
+    std::swap(a_i.p, b_i.p);
+    std::swap(a_d.p, b_d.p);
+  }
+  ALGAS_CUDA_TRY(cudaMemcpy(ids, a_i.p, bytes, cudaMemcpyDefault));
+  ALGAS_CUDA_TRY(cudaMemcpy(dists, a_d.p, bytes, cudaMemcpyDefault));
+  return ALGAS_OK;
+}
+
 int algas_build_graph_partitioned(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t knn_degree,
                                   int32_t degree, int32_t prune, int32_t n_clusters, int32_t overlap,
-                                  uint32_t* out_graph) {
-  if (!data || !out_graph || n < 2 || knn_degree < degree || degree < 1)
+                                  int32_t refine_fan, int32_t refine_rounds, uint32_t* out_graph) {
+  if (!data || !out_graph || n < 2 || knn_degree < degree || degree < 1 || refine_rounds < 0)
     return set_error(ALGAS_EINVAL, "algas_build_graph_partitioned: bad arguments");
   const int K = (int)std::min<int64_t>(knn_degree, n - 1);
   Dev guard_k, guard_d;
@@ -960,6 +1049,10 @@ int algas_build_graph_partitioned(const float* data, int64_t n, int32_t dim, int
   int rc = algas_knn_partitioned(data, n, dim, metric, K, n_clusters, overlap, (uint32_t*)guard_k.p,
                                  (float*)guard_d.p);
   if (rc) return rc;
+  if (refine_rounds > 0 &&
+      (rc = algas_knn_refine(data, n, dim, metric, K, std::min(std::max(refine_fan, 1), std::min(K, 64)),
+                             refine_rounds, (uint32_t*)guard_k.p, (float*)guard_d.p)))
+    return rc;
   // rows the partition left short (clusters of <= K points) are completed by
   // the exact kNN of those rows over the whole set (the prune needs full rows)
   std::vector<uint32_t> hk((size_t)n * K);

@@ -25,6 +25,9 @@ def main():
     ap.add_argument("workload", default="C2")
     ap.add_argument("--clusters", type=int, nargs="+", default=[64, 128])
     ap.add_argument("--overlap", type=int, nargs="+", default=[2])
+    ap.add_argument("--refine", type=int, nargs="+", default=[0, 1], help="refinement rounds (DESIGN.md R33)")
+    ap.add_argument("--fan", type=int, default=16)
+    ap.add_argument("--no-exact", action="store_true")
     ap.add_argument("--nq", type=int, default=2000)
     a = ap.parse_args()
     w = synth.WORKLOADS[a.workload]
@@ -40,33 +43,44 @@ def main():
     p = algas.default_params(k=w.k, itopk=64, width=8, offset_beam=1, n_seeds=32, ctas_per_query=1,
                              threads_per_cta=512, seed=3)
     out = {"workload": w.name, "n": w.n, "dim": w.dim, "knn_degree": w.knn_degree, "degree": w.degree}
-    torch.cuda.synchronize()
-    t0 = time.time()
-    ge = algas.build_graph(Xd, w.degree, knn_degree=w.knn_degree, metric=w.metric)
-    torch.cuda.synchronize()
-    out["exact_build_s"] = time.time() - t0
-    r = algas.Index(Xd, ge, w.metric).search(Q, params=p)
-    out["exact_search_recall"] = float((r["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
+    if not a.no_exact:
+        torch.cuda.synchronize()
+        t0 = time.time()
+        ge = algas.build_graph(Xd, w.degree, knn_degree=w.knn_degree, metric=w.metric)
+        torch.cuda.synchronize()
+        out["exact_build_s"] = time.time() - t0
+        r = algas.Index(Xd, ge, w.metric).search(Q, params=p)
+        out["exact_search_recall"] = float((r["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
+        print(json.dumps({"exact_build_s": out["exact_build_s"], "exact_search_recall": out["exact_search_recall"]}),
+              flush=True)
     out["partitioned"] = []
     for m in a.clusters:
         for c in a.overlap:
             torch.cuda.synchronize()
             t0 = time.time()
-            ids, _ = algas.knn_partitioned(Xd, w.knn_degree, m, c, w.metric)
+            ids, dd = algas.knn_partitioned(Xd, w.knn_degree, m, c, w.metric)
             torch.cuda.synchronize()
             t_knn = time.time() - t0
-            ids = ids.cpu().numpy().view(np.uint32)
-            hit = np.mean([len(set(ids[i].tolist()) & set(se[j, 1:].tolist())) / (w.knn_degree - 1)
-                           for j, i in enumerate(sample)])
-            t0 = time.time()
-            gp = algas.build_graph_partitioned(Xd, w.degree, m, c, knn_degree=w.knn_degree, metric=w.metric)
-            torch.cuda.synchronize()
-            t_build = time.time() - t0
-            rp = algas.Index(Xd, gp, w.metric).search(Q, params=p)
-            rec = float((rp["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
-            out["partitioned"].append({"clusters": m, "overlap": c, "knn_s": t_knn, "build_s": t_build,
-                                       "knn_graph_recall_sample": float(hit), "search_recall": rec})
-            print(json.dumps(out["partitioned"][-1]), flush=True)
+            for rounds in a.refine:
+                torch.cuda.synchronize()
+                t0 = time.time()
+                ri, _ = algas.knn_refine(Xd, ids, dd, fan=a.fan, rounds=rounds, metric=w.metric) if rounds else (ids, dd)
+                torch.cuda.synchronize()
+                t_ref = time.time() - t0
+                rih = ri.cpu().numpy().view(np.uint32)
+                hit = np.mean([len(set(rih[i].tolist()) & set(se[j, 1:].tolist())) / (w.knn_degree - 1)
+                               for j, i in enumerate(sample)])
+                t0 = time.time()
+                gp = algas.build_graph_partitioned(Xd, w.degree, m, c, knn_degree=w.knn_degree, metric=w.metric,
+                                                   refine_fan=a.fan, refine_rounds=rounds)
+                torch.cuda.synchronize()
+                t_build = time.time() - t0
+                rp = algas.Index(Xd, gp, w.metric).search(Q, params=p)
+                rec = float((rp["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
+                out["partitioned"].append({"clusters": m, "overlap": c, "refine_rounds": rounds, "fan": a.fan,
+                                           "knn_s": t_knn, "refine_s": t_ref, "build_s": t_build,
+                                           "knn_graph_recall_sample": float(hit), "search_recall": rec})
+                print(json.dumps(out["partitioned"][-1]), flush=True)
     print(json.dumps(out))
 
 

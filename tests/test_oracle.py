@@ -587,3 +587,61 @@ def test_knn_partitioned_entries_are_true_neighbours():
             assert np.all(np.diff(ds[i, :len(real)]) >= 0)
         rec.append(oracle.recall(ids, ei, 10))
     assert rec[1] > rec[0] and rec[1] > 0.8, rec
+
+
+# ---------------------------------------------------------------- refinement round (f4, R33)
+def _line_lists(n, k=2):
+    """1-d points x_i = i (d padded to 4); input lists in[p] = [p+1, p+3]
+    (distances 1, 9), SENTINEL past the end."""
+    X = np.zeros((n, 4), np.float32)
+    X[:, 0] = np.arange(n)
+    ids = np.full((n, k), SENT, np.uint32)
+    ds = np.full((n, k), np.inf, np.float32)
+    for p in range(n):
+        row = [(float((q - p) ** 2), q) for q in (p + 1, p + 3) if q < n]
+        for e, (dd, q) in enumerate(row):
+            ids[p, e], ds[p, e] = q, dd
+    return X, ids, ds
+
+
+def test_knn_refine_hand_example():
+    """k = 2, fan = 2, in[p] = [p+1, p+3].  For p <= 5: the neighbours' lists
+    are in[p+1] = [p+2, p+4] and in[p+3] = [p+4, p+6], so the candidates are
+    p+2, p+4, p+6 at 4, 16, 36; merged with (p+1: 1, p+3: 9) the first two are
+    p+1, p+2 at 1, 4.  A second round finds nothing closer (the lists only
+    point forward: p-1, as close as p+1, is never reached)."""
+    X, ids, ds = _line_lists(12)
+    o1, d1 = oracle.knn_refine(X, ids, ds, fan=2, rounds=1)
+    for p in range(6):
+        assert o1[p].tolist() == [p + 1, p + 2] and d1[p].tolist() == [1.0, 4.0]
+    o2, d2 = oracle.knn_refine(X, ids, ds, fan=2, rounds=2)
+    np.testing.assert_array_equal(o2[:6], o1[:6])
+
+
+@pytest.mark.parametrize("metric", [oracle.L2, oracle.IP])
+def test_knn_refine_exact_list_is_a_fixed_point(metric):
+    """An exact kNN list cannot be improved: refinement returns it unchanged."""
+    X = synth.lattice(400, 16, seed=61, metric=metric)
+    ei, ed = oracle.knn_graph(X, 12, metric)
+    for fan in (1, 4, 12):
+        ri, rd = oracle.knn_refine(X, ei, ed, fan=fan, rounds=1, metric=metric)
+        np.testing.assert_array_equal(ri, ei)
+        np.testing.assert_array_equal(rd, ed)
+
+
+def test_knn_refine_monotone_and_improves_partitioned_lists():
+    """From the partitioned lists (overlap 2, so lists cross partition
+    borders): every row's k-th distance never grows, all entries are true
+    distances, and recall vs the exact graph rises."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 1500)
+    ei, _ = oracle.knn_graph(X, 10)
+    pi, pd = oracle.knn_partitioned(X, 10, 12, 2)   # overlap 2: lists link the partitions
+    ri, rd = oracle.knn_refine(X, pi, pd, fan=8, rounds=1)
+    assert np.all(rd[:, -1] <= pd[:, -1])
+    for i in range(0, 1500, 53):
+        real = ri[i][ri[i] != SENT]
+        ref = ((X[real].astype(np.float64) - X[i]) ** 2).sum(1)
+        np.testing.assert_allclose(rd[i, :len(real)], ref, rtol=1e-5)
+        assert i not in real.tolist() and len(set(real.tolist())) == len(real)
+    assert oracle.recall(ri, ei, 10) > oracle.recall(pi, ei, 10) + 0.05

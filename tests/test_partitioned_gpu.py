@@ -70,3 +70,44 @@ def test_build_graph_partitioned_short_clusters_completed():
     g = algas.build_graph_partitioned(X, 24, n_clusters=200, overlap=1, knn_degree=48)
     assert (g < X.shape[0]).mean() > 0.999
     assert not (g == np.arange(X.shape[0])[:, None]).any()
+
+
+# ------------------------------------------------------------------ refinement round (R33)
+@pytest.mark.parametrize("metric", [algas.L2, algas.IP])
+@pytest.mark.parametrize("fan,rounds", [(4, 1), (12, 2)])
+def test_knn_refine_lattice_bit_exact(metric, fan, rounds):
+    """algas_knn_refine == oracle.knn_refine bit for bit on lattice data,
+    from the (oracle's) partitioned lists."""
+    X = synth.lattice(900, 32, seed=43, metric=metric)
+    pi, pd = oracle.knn_partitioned(X, 16, 9, 2, metric)
+    gi, gd = algas.knn_refine(X, pi, pd, fan=fan, rounds=rounds, metric=metric)
+    oi, od = oracle.knn_refine(X, pi, pd, fan=fan, rounds=rounds, metric=metric)
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(_bits(gd), _bits(od))
+
+
+def test_knn_refine_hand_example_gpu():
+    """The oracle's hand-worked example (tests/test_oracle.py) on the GPU."""
+    from test_oracle import _line_lists
+    X, ids, ds = _line_lists(12)
+    gi, gd = algas.knn_refine(X, ids, ds, fan=2, rounds=1)
+    for p in range(6):
+        assert gi[p].tolist() == [p + 1, p + 2] and gd[p].tolist() == [1.0, 4.0]
+
+
+def test_knn_refine_raises_recall_float():
+    """Float data: one round from partitioned lists raises kNN recall; every
+    entry is a true distance (1e-5) and rows stay sorted and duplicate-free."""
+    w = synth.WORKLOADS["C1"]
+    X = synth.base_vectors(w, 6000)
+    ei, _ = oracle.knn_graph(X, 16)
+    pi, pd = algas.knn_partitioned(X, 16, 24, 2)
+    ri, rd = algas.knn_refine(X, pi, pd, fan=16, rounds=1)
+    assert oracle.recall(ri, ei, 16) > oracle.recall(pi, ei, 16) + 0.05
+    assert np.all(rd[:, -1] <= pd[:, -1])
+    for i in range(0, 6000, 97):
+        real = ri[i][ri[i] != algas.SENTINEL]
+        assert i not in real.tolist() and len(set(real.tolist())) == len(real)
+        ref = ((X[real].astype(np.float64) - X[i]) ** 2).sum(1)
+        np.testing.assert_allclose(rd[i, :len(real)], ref, rtol=1e-5)
+        assert np.all(np.diff(rd[i, :len(real)]) >= 0)
