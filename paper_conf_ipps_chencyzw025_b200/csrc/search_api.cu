@@ -126,7 +126,11 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   // (ALGAS_GATHER_MODE)
   const char* gm_env = getenv("ALGAS_GATHER_MODE");
   const int gather_mode = gm_env ? atoi(gm_env) : 0;
-  if (gather_mode < 0 || gather_mode > 3) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0..3");
+  if (gather_mode < 0 || gather_mode > 4) return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE must be 0..4");
+#if !ALGAS_GATHER_EXPERIMENTS
+  if (gather_mode != 0)
+    return set_error(ALGAS_EINVAL, "ALGAS_GATHER_MODE %d needs a build with -DALGAS_GATHER_EXPERIMENTS=1", gather_mode);
+#endif
   if (cs > 1 && gather_mode != 0) return set_error(ALGAS_EINVAL, "cluster_size > 1 needs the register gather path");
   const char* pf_env = getenv("ALGAS_PREFETCH");  // experiment switch
   const int prefetch = pf_env ? atoi(pf_env) : 8;
@@ -145,7 +149,12 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   }
   const int gcb = gc_bytes(gcbits, idx->rp_shift);
   int team_rows = 0;
-  if (gather_mode == 3) {
+  if (gather_mode == 4) {
+    // hybrid: one register pass + team_rows staged rows per team in flight
+    const int nteams = nt / chunk_tl(cc);
+    team_rows = p->stage_rows > 0 ? p->stage_rows : 1;
+    sr = (nteams * team_rows + 1) / 2;
+  } else if (gather_mode == 3) {
     // rows in flight per team and pass: enough for a step's new rows
     // (<= w * Rp), as many as fit next to the smallest admissible hash;
     // p->stage_rows > 0 forces it (sweeps)

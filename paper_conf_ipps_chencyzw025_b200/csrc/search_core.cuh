@@ -522,6 +522,12 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
 // instruction issue (profiles/dist_wave_microbench*.txt): warps with no row
 // in a pass skip it entirely (warp-uniform test), and the compaction is one
 // ballot per row group instead of a warp scan.
+#ifndef ALGAS_GATHER_EXPERIMENTS
+#define ALGAS_GATHER_EXPERIMENTS 0  // 1: compile gather modes 1-4 (A/B builds, ALGAS_GATHER_MODE)
+#endif
+#ifndef ALGAS_QCHUNK
+#define ALGAS_QCHUNK 0  // A/B builds: 1 = query chunk loaded per chunk inside the FMA loop
+#endif
 #ifndef ALGAS_DIST_BW1024
 #define ALGAS_DIST_BW1024 4  // A/B builds: 16-B chunks per lane in flight at 1024 resident threads
 #endif
@@ -571,10 +577,35 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
     // the query chunks are read (volatile) only after every row load of the
     // pass was issued; the FMAs depend on them, so no FMA can be scheduled
     // between the row loads (which would serialise the DRAM round trips)
+    float acc[B];
+#if ALGAS_QCHUNK
+    // one query chunk in registers at a time (chunk-outer, row-inner): with
+    // B > 1 rows per team the query would otherwise hold CPL float4 next to
+    // the B x CPL row chunks.  Each row's sum runs in the same order as below.
+#pragma unroll
+    for (int b = 0; b < B; ++b) acc[b] = 0.f;
+#pragma unroll
+    for (int c = 0; c < CPL; ++c) {
+      const float4 q = lds_f4_ordered(qs + tl + c * TL);
+#pragma unroll
+      for (int b = 0; b < B; ++b) {
+        if (b >= nbw) continue;
+        const float4 x = v[b][c];
+        float a = acc[b];
+        if (METRIC == kL2) {
+          float d0 = q.x - x.x, d1 = q.y - x.y, d2 = q.z - x.z, d3 = q.w - x.w;
+          a = fmaf(d0, d0, a); a = fmaf(d1, d1, a); a = fmaf(d2, d2, a); a = fmaf(d3, d3, a);
+        } else {
+          a = fmaf(q.x, x.x, a); a = fmaf(q.y, x.y, a);
+          a = fmaf(q.z, x.z, a); a = fmaf(q.w, x.w, a);
+        }
+        acc[b] = a;
+      }
+    }
+#else
     QueryRegs<TL, CPL> Q;
 #pragma unroll
     for (int c = 0; c < CPL; ++c) Q.q[c] = lds_f4_ordered(qs + tl + c * TL);
-    float acc[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       float a = 0.f;
@@ -595,6 +626,7 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
       }
       acc[b] = a;
     }
+#endif
 #pragma unroll
     for (int o = TL >> 1; o > 0; o >>= 1)
 #pragma unroll
@@ -711,6 +743,72 @@ __device__ __forceinline__ void dist_async(const SearchCfg& cfg, const float4* q
       }
     }
   }
+}
+
+// Distance step, gather mode 4 (hybrid): the rows beyond the first register
+// pass (rows NTEAMS .. NTEAMS*(1+BS)) are put in flight FIRST as team-local
+// cp.async copies into shared memory, then the first NTEAMS rows go through
+// the register pass (dist_ldg), then each lane waits for its own copies and
+// reduces the staged rows -- the two waves' memory latencies overlap instead
+// of following each other.  Rows past both waves: further register passes.
+template <int NT, int TL, int CPL, int METRIC, int MINB>
+__device__ __forceinline__ void dist_hybrid(const SearchCfg& cfg, const float4* qs, float4* stage, int M,
+                                            uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  constexpr int B1 = DistRows<NT, TL, CPL, MINB>::B;  // rows per team of the register wave
+  constexpr int NTEAMS = NT / TL;
+  constexpr int W1 = NTEAMS * B1;                     // rows of the register wave
+  constexpr int TPW = 32 / TL;
+  const int team = tid / TL, tl = tid % TL;
+  const int wteam0 = (tid >> 5) * TPW;
+  const int BS = cfg.team_rows;
+  // wave 2 in flight first (no registers held)
+  for (int b = 0; b < BS; ++b) {
+    const int j = W1 + b * NTEAMS + team;
+    if (j < M) {
+      const float4* row = cfg.data + (uint64_t)newid[j] * cfg.d4;
+      float4* dst = stage + (size_t)(team * BS + b) * cfg.dp4;
+#pragma unroll
+      for (int c = 0; c < CPL; ++c) {
+        const int chn = tl + c * TL;
+        if (chn < cfg.d4) cp_async16(dst + chn, row + chn);
+      }
+    }
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+  // wave 1: the register pass over rows [0, W1)
+  dist_ldg<NT, TL, CPL, METRIC, B1>(cfg, qs, M < W1 ? M : W1, 0, 1, worst, newid, newk, nkeys);
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+  QueryRegs<TL, CPL> Q;
+  Q.load(qs, tl);
+  for (int b = 0; b < BS; ++b) {
+    if (W1 + b * NTEAMS + wteam0 >= M) break;  // warp-uniform: no row of this warp left
+    const int j = W1 + b * NTEAMS + team;
+    float a = team_partial_smem<TL, CPL, METRIC>(Q, stage + (size_t)(team * BS + b) * cfg.dp4, tl);
+#pragma unroll
+    for (int o = TL >> 1; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+    uint64_t key = kKeyMax;
+    uint32_t id = 0;
+    if (tl == 0 && j < M) {
+      id = newid[j];
+      key = make_key((METRIC == kL2) ? a : -a, id);
+    }
+    const bool keep = key < worst;
+    const unsigned m = __ballot_sync(0xffffffffu, keep);
+    if (keep && (cfg.prefetch & 8))
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cfg.graph + ((uint64_t)id << cfg.rp_shift)),
+                   "r"(4u << cfg.rp_shift)
+                   : "memory");
+    if (m) {
+      int wbase = 0;
+      if (lane == 0) wbase = atomicAdd(nkeys, __popc(m));
+      wbase = __shfl_sync(0xffffffffu, wbase, 0);
+      if (keep) newk[wbase + __popc(m & ((1u << lane) - 1u))] = key;
+    }
+  }
+  // rows past both waves (large steps): more register passes
+  const int done = W1 + NTEAMS * BS;
+  if (M > done) dist_ldg<NT, TL, CPL, METRIC, B1>(cfg, qs, M, done, 1, worst, newid, newk, nkeys);
 }
 
 // Warp-level bitonic merge ("parallel-friendly bitonic sort", the
@@ -1167,8 +1265,16 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
                                                                       &C->nkeys[sp], gcache, gstamp);
           __syncthreads();
         }
-      } else if (cfg.gather_mode == 3) {
+      }
+#if ALGAS_GATHER_EXPERIMENTS
+      // measured alternatives of the vector gather (compiled
+      // only into A/B builds: their code paths cost the production kernel
+      // registers)
+      else if (cfg.gather_mode == 3) {
         dist_async<NT, TL, CPL, METRIC>(cfg, s.q, s.stage, M, worst, s.newid, s.newk, &C->nkeys[sp]);
+        __syncthreads();
+      } else if (cfg.gather_mode == 4) {
+        dist_hybrid<NT, TL, CPL, METRIC, MINB>(cfg, s.q, s.stage, M, worst, s.newid, s.newk, &C->nkeys[sp]);
         __syncthreads();
       }
       const int SR = cfg.stage_rows;
@@ -1226,6 +1332,7 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
         }
         __syncthreads();  // buffer b fully read before it is re-issued (chunk ch+2)
       }
+#endif
       if (tid == 0) C->dist_evals += M;
       lap(2);
     }

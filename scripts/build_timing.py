@@ -28,6 +28,8 @@ def main():
     ap.add_argument("--refine", type=int, nargs="+", default=[0, 1], help="refinement rounds (DESIGN.md R33)")
     ap.add_argument("--fan", type=int, default=16)
     ap.add_argument("--no-exact", action="store_true")
+    ap.add_argument("--search-L", type=int, nargs="*", default=[],
+                    help="also search each partitioned graph at these L (T=4, 1024 threads, SHARED, w=12/16)")
     ap.add_argument("--nq", type=int, default=2000)
     a = ap.parse_args()
     w = synth.WORKLOADS[a.workload]
@@ -77,9 +79,19 @@ def main():
                 t_build = time.time() - t0
                 rp = algas.Index(Xd, gp, w.metric).search(Q, params=p)
                 rec = float((rp["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean())
+                curve = []
+                idx_p = algas.Index(Xd, gp, w.metric)
+                for L in a.search_L:
+                    ps = algas.default_params(k=w.k, itopk=L, width=min(L, 12 if L <= 32 else 16), offset_beam=1,
+                                              n_seeds=32, ctas_per_query=4, threads_per_cta=1024, slots=32, seed=3,
+                                              visited_mode=1)
+                    rr = idx_p.search_dynamic(Qd, ps)
+                    curve.append([L, float((rr["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean()),
+                                  round(a.nq / (rr["info"].kernel_ms / 1e3))])
                 out["partitioned"].append({"clusters": m, "overlap": c, "refine_rounds": rounds, "fan": a.fan,
                                            "knn_s": t_knn, "refine_s": t_ref, "build_s": t_build,
-                                           "knn_graph_recall_sample": float(hit), "search_recall": rec})
+                                           "knn_graph_recall_sample": float(hit), "search_recall": rec,
+                                           "search_T4_L_recall_qps": curve})
                 print(json.dumps(out["partitioned"][-1]), flush=True)
     print(json.dumps(out))
 
