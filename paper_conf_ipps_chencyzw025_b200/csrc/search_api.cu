@@ -695,6 +695,10 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
     pa.dq_done = (uint32_t*)(db + o_done);
     pa.call_id = ++ws->call_id;
     if (pa.call_id == 0) pa.call_id = ++ws->call_id;  // 0 = never written
+    // the Finish words of THIS call's layout: the region may hold an earlier
+    // call's results or counters (other T / nq => other offsets), whose
+    // values could equal call_id -- clear it before the launch
+    memset(mdone, 0, (size_t)items * 4);
   }
   EventTimer tm(st);
   if ((rc = tm.start())) return rc;
