@@ -105,6 +105,10 @@ typedef struct algas_params {
                                 stream, P:L255-272's GDRCopy state copy without GDRCopy), so
                                 the slots' CTAs poll HBM instead of host memory over PCIe;
                                 0 (default) = CTAs poll the host-mapped ring */
+    int32_t watchdog_ms;     /* persistent server: a query in a slot longer than this is
+                                reported (algas_poll -> ALGAS_ESTATE, the stuck tag in
+                                algas_last_error): a hung or dead kernel never leaves the
+                                caller waiting silently; 0 -> 10000 ms, < 0 -> off */
     uint64_t seed;           /* entry-point generator seed (R5)                      */
 } algas_params;
 

@@ -44,7 +44,7 @@ class Params(ctypes.Structure):
                 ("max_iter", ctypes.c_int32), ("visited_mode", ctypes.c_int32), ("slots", ctypes.c_int32),
                 ("hash_bits", ctypes.c_int32), ("stage_rows", ctypes.c_int32),
                 ("cluster_size", ctypes.c_int32), ("host_threads", ctypes.c_int32),
-                ("state_mirror", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("state_mirror", ctypes.c_int32), ("watchdog_ms", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class QueryStats(ctypes.Structure):

@@ -129,6 +129,10 @@ struct algas_server {
   // accepted, and every ring entry that becomes free is set to QUIT, so the
   // persistent kernel exits once the staged queries are done
   std::atomic<bool> quit_when_idle{false};
+  // watchdog: a query in a slot longer than watchdog_ns marks the server failed
+  int64_t watchdog_ns = 0;
+  std::atomic<bool> stuck{false};
+  std::atomic<uint64_t> stuck_tag{0};
   bool launched = false;
   PersistArgs pa;  // launch arguments (kept for a deferred launch)
   // state mirror: host staging of every ring entry (RingSlot line
@@ -274,11 +278,14 @@ static void poller_main(algas_server* s, int me, int nth) {
   std::vector<uint32_t> ids(s->kmax);
   std::vector<float> ds(s->kmax);
   int idle = 0;
+  uint64_t sweep = 0;
   while (!s->stop.load(std::memory_order_acquire)) {
     bool any = false;
+    int watching = 0;  // this poller's queries in flight
     for (int q = 0; q < 2 * s->slots; ++q) {  // sub-slots of this poller's slots
       if ((q >> 1) % nth != me) continue;
       if ((*s->hstate)[q].load(std::memory_order_acquire) != 2) continue;
+      ++watching;
       const uint32_t ep = s->epoch[q];
       bool all = true;
       for (int c = 0; c < T; ++c) {
@@ -286,7 +293,18 @@ static void poller_main(algas_server* s, int me, int nth) {
         uint32_t v = __atomic_load_n(&s->done_h[(size_t)q * T + c], __ATOMIC_ACQUIRE);
         if (v != ep) { all = false; break; }
       }
-      if (!all) continue;
+      if (!all) {
+        // watchdog: checked every 1024 sweeps (a steady_clock read per sweep would cost the merge path)
+        if (s->watchdog_ns > 0 && (sweep & 1023) == 0 && !s->stuck.load(std::memory_order_relaxed)) {
+          const int64_t age = std::chrono::duration_cast<std::chrono::nanoseconds>(
+                                  std::chrono::steady_clock::now() - s->t_submit[q]).count();
+          if (age > s->watchdog_ns) {
+            s->stuck_tag.store(s->tags[q], std::memory_order_relaxed);
+            s->stuck.store(true, std::memory_order_release);
+          }
+        }
+        continue;
+      }
       any = true;
       algas_server::Done d;
       d.tag = s->tags[q];
@@ -320,7 +338,10 @@ static void poller_main(algas_server* s, int me, int nth) {
         s->cq.push_back(std::move(d));
       }
     }
-    if (!any) {
+    // spin while queries are in flight (a yield can cost several us of
+    // rescheduling latency on the merge path); back off only when idle
+    ++sweep;
+    if (!any && watching == 0) {
       if (++idle > 64) {
         std::this_thread::yield();
         idle = 0;
@@ -356,6 +377,10 @@ int algas_server_start(algas_server* s, int32_t quit_when_idle) {
       }
     if (s->mirror) cudaStreamSynchronize(io_stream(s));
   }
+  // staged queries: their time in the slot (latency, watchdog) starts now
+  const auto now = std::chrono::steady_clock::now();
+  for (int u = 0; u < 2 * s->slots; ++u)
+    if ((*s->hstate)[u].load(std::memory_order_acquire) == 2) s->t_submit[u] = now;
   const int rc = launch_persistent(s->plan, s->pa, s->stream);
   if (rc) return rc;
   s->launched = true;
@@ -401,6 +426,7 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)nsub * s->T);
 #undef SRV_ALLOC
   s->uid = g_server_uid.fetch_add(1);
+  s->watchdog_ns = params->watchdog_ms < 0 ? 0 : (int64_t)(params->watchdog_ms > 0 ? params->watchdog_ms : 10000) * 1000000;
   s->mirror = params->state_mirror != 0;
   if (s->mirror) {
     s->mir_stride = (int64_t)sizeof(RingSlot) + (int64_t)s->dim * 4;  // 16-B multiple (dim % 4 == 0)
@@ -553,6 +579,9 @@ int algas_poll(algas_server* s, uint64_t* tags, uint32_t* ids, float* dists, alg
   cudaError_t e = cudaStreamQuery(s->stream);
   if (e != cudaSuccess && e != cudaErrorNotReady)
     return set_error(ALGAS_ECUDA, "persistent kernel failed: %s", cudaGetErrorString(e));
+  if (s->stuck.load(std::memory_order_acquire))
+    return set_error(ALGAS_ESTATE, "watchdog: query tag %llu has been in its slot for more than %lld ms",
+                     (unsigned long long)s->stuck_tag.load(), (long long)(s->watchdog_ns / 1000000));
   std::lock_guard<std::mutex> lk(s->cq_mu);
   int n = 0;
   while (n < max_results && !s->cq.empty()) {

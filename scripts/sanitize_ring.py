@@ -29,7 +29,8 @@ def main():
     idx = algas.Index(X, G)
     for vis, T, mirror in ((0, 2, 0), (1, 4, 0), (1, 4, 1)):
         p = algas.default_params(k=10, itopk=32, width=4, offset_beam=1, n_seeds=16, ctas_per_query=T,
-                                 threads_per_cta=nt, slots=6, seed=1, visited_mode=vis, state_mirror=mirror)
+                                 threads_per_cta=nt, slots=6, seed=1, visited_mode=vis, state_mirror=mirror,
+                                 watchdog_ms=-1)  # a sanitized kernel runs orders of magnitude slower
         got = {}
         with algas.Server(idx, p, deferred=True) as srv:
             for t in range(Q.shape[0]):

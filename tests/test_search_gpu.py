@@ -591,3 +591,22 @@ def test_server_enqueue_fifo_equals_batch(slots, T, shared, mirror):
         np.testing.assert_array_equal(_bits(ds), _bits(b["dists"]))
     else:
         _check_invariants(X, Q, ids, ds, algas.L2, 10)
+
+
+def test_server_watchdog_reports_a_stuck_slot():
+    """A query that never completes (here: staged into a deferred server whose
+    kernel is never started) is reported by algas_poll after watchdog_ms
+    instead of being waited on forever."""
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=501)
+    p = algas.default_params(k=10, itopk=16, width=2, n_seeds=4, ctas_per_query=1, threads_per_cta=64, slots=2,
+                             seed=1, watchdog_ms=200)
+    idx = algas.Index(X, G)
+    srv = algas.Server(idx, p, deferred=True)
+    try:
+        assert srv.submit(Q[0], tag=77)
+        srv.poll(4)                                   # fine before the deadline
+        time.sleep(0.5)
+        with pytest.raises(algas.AlgasError, match="watchdog: query tag 77"):
+            srv.poll(4)
+    finally:
+        srv.close()
