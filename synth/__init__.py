@@ -10,7 +10,9 @@ Workloads (BASELINE.json ``configs``):
   C2  1M  x 128  fp32 L2 (SIFT1M-shaped),  R=64, k=10
   C3  1M  x 960  fp32 L2 (GIST1M-shaped),  R=64, k=10
   C4  1.2M x 100 inner product (GloVe-100-shaped, unit-normalised), R=64, k=100
-  C5  100M x 96  fp32 L2 (DEEP-shaped, unit-normalised), sharded
+  C5  100M x 96  fp32 L2 (DEEP-shaped, unit-normalised), sharded: 8 shards
+      generated on the device from (seed, shard) (shard_vectors_device);
+      C5s = one of them (12.5M x 96), what one B200 holds at G = 8
 """
 from __future__ import annotations
 
@@ -44,6 +46,12 @@ class Workload:
     seed_base: int
     seed_query: int
     center_scale: float = 1.0  # centers ~ N(0, center_scale^2 I)
+    shards: int = 0            # > 0: the base set is shard 0 of `shards` per-shard generated parts (C5)
+    build: str = "exact"       # graph build: "exact" (kNN + prune) or "partitioned" (R30 / R33)
+    part_clusters: int = 0     # partitioned build: clusters (0: n / 4096), overlap, refinement rounds / fan
+    part_overlap: int = 2
+    refine_rounds: int = 8
+    refine_fan: int = 32
 
 
 WORKLOADS = {
@@ -61,7 +69,11 @@ WORKLOADS = {
     "C4": Workload("C4-GloVe100-shaped-1.2Mx100-IP", 1_200_000, 100, IP, 64, 100, 10_000, 128, True,
                    1000, 24, 4.0, 0.3, 1.0, 0.0, False, True, 4001, 4002, 0.5),
     "C5": Workload("C5-DEEP100M-shaped-100Mx96-L2", 100_000_000, 96, L2, 64, 10, 10_000, 128, True,
-                   10000, 24, 4.0, 0.3, 1.0, 0.0, False, True, 5001, 5002, 0.5),
+                   10000, 24, 4.0, 0.3, 1.0, 0.0, False, True, 5001, 5002, 0.5, shards=8, build="partitioned"),
+    # one shard of C5 at G = 8 (12.5M x 96), generated on the device from (seed, shard) --
+    # what one B200 holds and builds in the sharded mode
+    "C5s": Workload("C5-shard0of8-DEEP-shaped-12.5Mx96-L2", 12_500_000, 96, L2, 64, 10, 10_000, 128, True,
+                    10000, 24, 4.0, 0.3, 1.0, 0.0, False, True, 5001, 5002, 0.5, shards=8, build="partitioned"),
 }
 
 
@@ -109,6 +121,38 @@ def base_vectors(w: Workload, n: int | None = None) -> np.ndarray:
     centers, bases = _model(w, w.dim)
     rng = np.random.default_rng(w.seed_base)
     return _finish(w, _mixture(rng, n, w.dim, centers, bases, w.spread, w.noise))
+
+
+def shard_vectors_device(w: Workload, shard: int, device, n: int | None = None, chunk: int = 1 << 18):
+    """Shard `shard` of a sharded base set (C5), generated ON THE DEVICE from
+    (seed_base + shard) with torch's generator: the same mixture model (the
+    K centres and bases of `_model`, shared by all shards) as base_vectors,
+    another random stream.  Returns an (n x dim) float32 CUDA tensor
+    (n = w.n, the shard's size)."""
+    import torch
+    n = w.n if n is None else n
+    centers, bases = _model(w, w.dim)
+    C = torch.from_numpy(centers).to(device)
+    B = torch.from_numpy(bases).to(device)
+    g = torch.Generator(device=device)
+    g.manual_seed(int(w.seed_base) * 1000 + int(shard))
+    out = torch.empty((n, w.dim), dtype=torch.float32, device=device)
+    K = B.shape[0]
+    for s in range(0, n, chunk):
+        m = min(chunk, n - s)
+        c = torch.randint(0, K, (m,), generator=g, device=device)
+        z = torch.randn((m, w.rank), generator=g, device=device)
+        x = torch.randn((m, w.dim), generator=g, device=device) * w.noise
+        x += C[c] + w.spread * torch.einsum("mr,mrd->md", z, B[c])
+        x = x * w.value_scale + w.value_shift
+        if w.clip0:
+            x.clamp_(min=0)
+        if w.normalize:
+            nrm = x.double().pow(2).sum(1, keepdim=True).sqrt()
+            nrm[nrm == 0] = 1.0
+            x = (x.double() / nrm).float()
+        out[s:s + m] = x
+    return out
 
 
 def query_vectors(w: Workload, nq: int | None = None, stream: int = 0) -> np.ndarray:
