@@ -12,7 +12,7 @@ CSRC = os.path.join(HERE, "csrc")
 # same sources with extra -D flags from ALGAS_BUILD_DEFS, e.g. build/*.so)
 LIB = os.environ.get("ALGAS_LIB") or os.path.join(HERE, "libalgas.so")
 EXTRA_DEFS = os.environ.get("ALGAS_BUILD_DEFS", "").split()
-SOURCES = ["search_kernels.cu", "search_api.cu", "runtime.cu", "knn.cu", "build_part.cu"]
+SOURCES = ["search_kernels.cu", "search_api.cu", "runtime.cu", "knn.cu", "build_part.cu", "knn_tc.cu"]
 # the search kernels, one object per thread count (compiled in parallel)
 THREAD_COUNTS = [32, 64, 128, 256, 512, 1024]
 KERNEL_TU = "kernels_nt.cu"

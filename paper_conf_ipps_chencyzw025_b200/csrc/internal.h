@@ -247,6 +247,11 @@ int launch_refine(const float* X, int d, int metric, int64_t n, int k, int fan, 
                   const float* in_d, uint32_t* out_ids, float* out_d);
 constexpr int kPartMaxKnn = 128;  // list length the batched cluster kNN keeps in shared memory
 
+// graph build's contraction on the tensor cores (knn_tc.cu): D (qb x nb, row
+// stride ldD) = Q . X^T from TF32 hi/lo splits (3xTF32), tcgen05 + TMEM
+int tc_dot_3xtf32(const float* Qh, const float* Ql, int64_t qb, const float* Xh, const float* Xl, int64_t nb, int d,
+                  float* D, int64_t ldD, cudaStream_t st);
+
 // host TopK merge (runtime.cpp)
 int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t* out_ids, float* out_d);
 

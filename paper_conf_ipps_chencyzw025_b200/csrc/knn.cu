@@ -508,8 +508,10 @@ static int knn_screened(const float* X, int64_t n, const float* Q, int64_t nq, i
   const double u = std::ldexp(1.0, -24);
   const double gam = (d + 8) * u / (1.0 - (d + 8) * u);
   const float eps_c = (float)(1.05 * (4.0 * gam + 8.0 * std::ldexp(1.0, -22)));
-  cublasHandle_t h = cublas_handle();
-  ALGAS_CUBLAS_TRY(cublasSetStream(h, 0));
+  const char* gemm_env = getenv("ALGAS_KNN_GEMM");
+  const bool use_cublas = gemm_env != nullptr && strcmp(gemm_env, "cublas") == 0;
+  cublasHandle_t h = use_cublas ? cublas_handle() : nullptr;
+  if (use_cublas) ALGAS_CUBLAS_TRY(cublasSetStream(h, 0));
   const int sel_smem = SEL_WARPS * (2 * K2 + SEL_BUF) * 8;
   void* sel = metric == ALGAS_L2 ? (void*)select_kernel<1> : (void*)select_kernel<2>;
   ALGAS_CUDA_TRY(cudaFuncSetAttribute(sel, cudaFuncAttributeMaxDynamicSharedMemorySize, sel_smem));
@@ -524,13 +526,20 @@ static int knn_screened(const float* X, int64_t n, const float* Q, int64_t nq, i
     split_tf32_kernel<<<(unsigned)((qb * d + 255) / 256), 256>>>(Q + q0 * d, (size_t)qb * d, Qh, Ql);
     for (int64_t x0 = 0; x0 < n; x0 += NB) {
       const int64_t nb = std::min<int64_t>(NB, n - x0);
-      // D^T (col-major nb x qb, ld NB) = X_blk . Q_blk^T: hi.hi + lo.hi + hi.lo
-      const float* A[3] = {Xh + x0 * d, Xl + x0 * d, Xh + x0 * d};
-      const float* B[3] = {Qh, Qh, Ql};
-      for (int g = 0; g < 3; ++g)
-        ALGAS_CUBLAS_TRY(cublasGemmEx(h, CUBLAS_OP_T, CUBLAS_OP_N, (int)nb, (int)qb, d, &one, A[g], CUDA_R_32F, d,
-                                      B[g], CUDA_R_32F, d, g == 0 ? &zero : &one, D, CUDA_R_32F, (int)NB,
-                                      CUBLAS_COMPUTE_32F_FAST_TF32, CUBLAS_GEMM_DEFAULT));
+      // D (row-major qb x nb, ld NB) = Q_blk . X_blk^T: hi.hi + lo.hi + hi.lo
+      if (use_cublas) {
+        // library path (A/B: ALGAS_KNN_GEMM=cublas): D^T col-major = X_blk . Q_blk^T
+        const float* A[3] = {Xh + x0 * d, Xl + x0 * d, Xh + x0 * d};
+        const float* B[3] = {Qh, Qh, Ql};
+        for (int g = 0; g < 3; ++g)
+          ALGAS_CUBLAS_TRY(cublasGemmEx(h, CUBLAS_OP_T, CUBLAS_OP_N, (int)nb, (int)qb, d, &one, A[g], CUDA_R_32F, d,
+                                        B[g], CUDA_R_32F, d, g == 0 ? &zero : &one, D, CUDA_R_32F, (int)NB,
+                                        CUBLAS_COMPUTE_32F_FAST_TF32, CUBLAS_GEMM_DEFAULT));
+      } else {
+        // hand-written tcgen05 kernel (knn_tc.cu)
+        int rc = tc_dot_3xtf32(Qh, Ql, qb, Xh + x0 * d, Xl + x0 * d, nb, d, D, NB, 0);
+        if (rc) return rc;
+      }
       if (metric == ALGAS_L2)
         select_kernel<1><<<(unsigned)((qb + SEL_WARPS - 1) / SEL_WARPS), SEL_WARPS * 32, sel_smem>>>(
             D, NB, (int)qb, nb, x0, q0, self_base, K2, (unsigned long long*)hstate.p, qn, xn, nullptr);

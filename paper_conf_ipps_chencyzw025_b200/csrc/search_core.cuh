@@ -540,10 +540,17 @@ struct DistRows {
   static constexpr int BW = NT * MINB >= 1024 ? ALGAS_DIST_BW1024 : 16;
   static constexpr int B = CPL >= BW ? 1 : BW / CPL;
 };
+// claim_vbm (SHARED mode with the query's bitmap): the rows are
+// claimed HERE -- lane 0 of the team issues the row's atomicOr right before
+// the row's loads, so the claim's L2 round trip overlaps the row's DRAM
+// fetch; a row another CTA of the query claimed first is gathered but its
+// key dropped (the node is scored by exactly one CTA, as with a claim at
+// filter time, which costs a separate round trip before the wave).
 template <int NT, int TL, int CPL, int METRIC, int BOVR = 0>
 __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs, int M, int r0, int rstep,
                                          uint64_t worst, const uint32_t* newid, uint64_t* newk, int* nkeys,
-                                         uint32_t* gcache = nullptr, uint32_t gc_stamp = 0) {
+                                         uint32_t* gcache = nullptr, uint32_t gc_stamp = 0,
+                                         uint32_t* claim_vbm = nullptr) {
   const int tid = threadIdx.x, lane = tid & 31;
   constexpr int NTEAMS = NT / TL;
   constexpr int TPW = 32 / TL;  // teams per warp
@@ -559,10 +566,16 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
     if (nbw <= 0) continue;
     float4 v[B][CPL];
     uint32_t ids[B];
+    uint32_t lost[B];  // claim_vbm: another CTA claimed the row first
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       const int j = base + b * NTEAMS + team;
       ids[b] = j < Mc ? newid[r0 + j * rstep] : 0u;
+      lost[b] = 0u;
+      if (claim_vbm != nullptr && tl == 0 && b < nbw && j < Mc) {
+        const uint32_t bit = 1u << (ids[b] & 31);
+        lost[b] = atomicOr(claim_vbm + (ids[b] >> 5), bit) & bit;
+      }
     }
 #pragma unroll
     for (int b = 0; b < B; ++b) {
@@ -639,7 +652,7 @@ __device__ __forceinline__ void dist_ldg(const SearchCfg& cfg, const float4* qs,
     for (int b = 0; b < B; ++b) {
       const int j = base + b * NTEAMS + team;
       uint64_t key = kKeyMax;
-      if (b < nbw && tl == 0 && j < Mc) key = make_key((METRIC == kL2) ? acc[b] : -acc[b], ids[b]);
+      if (b < nbw && tl == 0 && j < Mc && !lost[b]) key = make_key((METRIC == kL2) ? acc[b] : -acc[b], ids[b]);
       m[b] = b < nbw ? __ballot_sync(0xffffffffu, key < worst) : 0u;
       tot += __popc(m[b]);
       // a key that enters the list is a likely parent of the next step(s):
@@ -1191,9 +1204,13 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
                 for (int o = 0; o < cfg.d4 * 16; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rp + o));
               }
               if (keep && cfg.shared) {  // new to this CTA: claim it in the query's table (P:L211, P:L217 step 2)
-                if (vbm) {                // the paper's bitmap: one L2 atomic, no probing
-                  const uint32_t bit = 1u << (id & 31);
-                  keep = (atomicOr(vbm + (id >> 5), bit) & bit) == 0u;
+                if (vbm) {                // the paper's bitmap: one L2 atomic, no probing --
+                  if (!(cfg.prefetch & 256)) {  // (A/B, bit 256: with the row's loads in dist_ldg instead --
+                                                  //  measured slower: the rows other CTAs won cost more
+                                                  //  than the round trip saved, profiles/round2_ab.md)
+                    const uint32_t bit = 1u << (id & 31);
+                    keep = (atomicOr(vbm + (id >> 5), bit) & bit) == 0u;
+                  }
                 } else {
                   const int g = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
                   keep = (g == kVisNew);
@@ -1229,6 +1246,7 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
         lap(1);
       }
     }
+    const bool first_pass = first;  // the seeding pass: its ids are the CTA's seeds
     first = false;
 
     // ================= distances (P:L217 step 3) + prefilter =================
@@ -1261,8 +1279,12 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
           __syncthreads();
         } else {
           ++gstamp;
+          // prefetch bit 256 (A/B): SHARED bitmap claims ride with the row
+          // loads (not for the seeds: a CTA keeps its own seeds, R21; not
+          // after a spill, whose filter claims at filter time)
+          uint32_t* claim = (vbm != nullptr && !first_pass && !C->spilled && (cfg.prefetch & 256)) ? vbm : nullptr;
           dist_ldg<NT, TL, CPL, METRIC, DistRows<NT, TL, CPL, MINB>::B>(cfg, s.q, M, 0, 1, worst, s.newid, s.newk,
-                                                                      &C->nkeys[sp], gcache, gstamp);
+                                                                      &C->nkeys[sp], gcache, gstamp, claim);
           __syncthreads();
         }
       }

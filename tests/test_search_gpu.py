@@ -150,11 +150,36 @@ def test_knn_screened_equals_direct_float(knn_mode, metric, d):
     np.testing.assert_array_equal(_bits(sd), _bits(dd))
 
 
+@pytest.mark.parametrize("d", [128, 100, 960])
+def test_knn_tcgen05_screen_certifies_and_matches_cublas(knn_mode, monkeypatch, d):
+    """The screen's contraction on the hand-written tcgen05 kernel (3xTF32 in
+    TMEM, knn_tc.cu): the certificate holds for (nearly) every row -- an
+    inaccurate product would send rows to the fallback -- and the kNN equals
+    the cuBLAS-screened and the direct (CUDA-core) results bit for bit."""
+    X = synth.uniform(30_000, d, seed=31)
+    Q = synth.uniform(500, d, seed=32)
+    knn_mode("screened")
+    algas.knn_last_stats()  # reset the per-thread counters
+    ti, td = algas.knn(X, Q, 32, algas.L2)
+    screened, fallback = algas.knn_last_stats()
+    assert screened == Q.shape[0] and fallback <= 0.02 * Q.shape[0], (screened, fallback)
+    monkeypatch.setenv("ALGAS_KNN_GEMM", "cublas")
+    ci, cd = algas.knn(X, Q, 32, algas.L2)
+    monkeypatch.delenv("ALGAS_KNN_GEMM")
+    knn_mode("direct")
+    di, dd = algas.knn(X, Q, 32, algas.L2)
+    algas.knn_last_stats()
+    np.testing.assert_array_equal(ti, ci)
+    np.testing.assert_array_equal(ti, di)
+    np.testing.assert_array_equal(_bits(td), _bits(dd))
+
+
 def test_knn_screened_lattice_matches_oracle(knn_mode):
     """Integer lattice: the screened path equals O1 bit for bit, including
     (dist, id) tie order (ties defeat the certificate -> direct fallback)."""
     X = synth.lattice(5000, 64, seed=23)
     knn_mode("screened")
+    algas.knn_last_stats()  # reset the per-thread counters
     gi, gd = algas.knn(X, X[:200], 20, algas.L2, self_base=0)
     screened, fallback = algas.knn_last_stats()
     assert screened == 200
