@@ -96,6 +96,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_dot_kernel(const float* __re
   for (int kb = 0; kb < nkb; ++kb) {
     const int k0 = kb * TC_K;
     // ---- stage the K block: 16-B chunks, zero past the matrix edges
+    // (unrolled so several loads of a thread are in flight at once)
+#pragma unroll 4
     for (int t = tid; t < TC_M * (TC_K / 4); t += TC_THREADS) {
       const int r = t >> 3, c = t & 7;
       float4 h = make_float4(0.f, 0.f, 0.f, 0.f), l = h;
@@ -106,6 +108,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_dot_kernel(const float* __re
       *reinterpret_cast<float4*>(a_hi + tile_off(r, c)) = h;
       *reinterpret_cast<float4*>(a_lo + tile_off(r, c)) = l;
     }
+#pragma unroll 4
     for (int t = tid; t < TC_N * (TC_K / 4); t += TC_THREADS) {
       const int r = t >> 3, c = t & 7;
       float4 h = make_float4(0.f, 0.f, 0.f, 0.f), l = h;
