@@ -12,7 +12,8 @@
 // the cuBLAS path computes (error bound: knn.cu, eps_c).
 //
 // One CTA = a 128 (queries) x 256 (base points) tile, 128 threads:
-//   * per K block of 32 dims, all threads stage the four operand tiles
+//   * per K block of 32 dims (two stage buffers: block kb+1 is staged while
+//     the tensor core runs block kb), all threads stage the four operand tiles
 //     (Q hi/lo 128 x 32, X hi/lo 256 x 32) into shared memory in the
 //     canonical K-major no-swizzle UMMA layout (8-row x 16-byte core
 //     matrices: core (g, c) of row group g and 16-byte K chunk c at
@@ -62,16 +63,49 @@ __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b
 
 }  // namespace
 
+constexpr int kStageBytes = (TC_M + TC_N) * TC_K * 4 * 2;  // Q hi/lo + X hi/lo tiles of one K block: 96 KB
+
+// stage K block k0 of the four operand tiles into buffer `buf`: 16-B
+// cp.async (LDGSTS) per chunk into its canonical-layout slot, zero-filled
+// past the matrix edges (src-size 0); nothing is waited for here -- a thread
+// has all 48 of its chunk copies in flight (cp.async.commit_group after)
+__device__ __forceinline__ void cp16_zfill(uint8_t* dst, const float* src, bool valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(valid ? 16 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void tc_stage(uint8_t* buf, const float* Qh, const float* Ql, int64_t qb, int64_t q0,
+                                         const float* Xh, const float* Xl, int64_t nb, int64_t x0, int d, int k0,
+                                         int tid) {
+  uint8_t* a_hi = buf;
+  uint8_t* a_lo = a_hi + TC_M * TC_K * 4;
+  uint8_t* b_hi = a_lo + TC_M * TC_K * 4;
+  uint8_t* b_lo = b_hi + TC_N * TC_K * 4;
+#pragma unroll 8
+  for (int t = tid; t < TC_M * (TC_K / 4); t += TC_THREADS) {
+    const int r = t >> 3, c = t & 7;
+    const bool ok = q0 + r < qb && k0 + c * 4 < d;
+    const int64_t o = ok ? (q0 + r) * d + k0 + c * 4 : 0;
+    cp16_zfill(a_hi + tile_off(r, c), Qh + o, ok);
+    cp16_zfill(a_lo + tile_off(r, c), Ql + o, ok);
+  }
+#pragma unroll 8
+  for (int t = tid; t < TC_N * (TC_K / 4); t += TC_THREADS) {
+    const int r = t >> 3, c = t & 7;
+    const bool ok = x0 + r < nb && k0 + c * 4 < d;
+    const int64_t o = ok ? (x0 + r) * d + k0 + c * 4 : 0;
+    cp16_zfill(b_hi + tile_off(r, c), Xh + o, ok);
+    cp16_zfill(b_lo + tile_off(r, c), Xl + o, ok);
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
 __global__ void __launch_bounds__(TC_THREADS, 1) tc_dot_kernel(const float* __restrict__ Qh, const float* __restrict__ Ql,
                                                                int64_t qb, const float* __restrict__ Xh,
                                                                const float* __restrict__ Xl, int64_t nb, int d,
                                                                float* __restrict__ D, int64_t ldD) {
+  // two stage buffers: block kb+1 is staged while the tensor core runs block kb
   extern __shared__ __align__(1024) uint8_t sm[];
-  uint8_t* a_hi = sm;                          // 128 x 32 fp32 = 16 KB
-  uint8_t* a_lo = a_hi + TC_M * TC_K * 4;      // 16 KB
-  uint8_t* b_hi = a_lo + TC_M * TC_K * 4;      // 256 x 32 fp32 = 32 KB
-  uint8_t* b_lo = b_hi + TC_N * TC_K * 4;      // 32 KB
-  __shared__ __align__(8) uint64_t mbar;
+  __shared__ __align__(8) uint64_t mbar[2];
   __shared__ uint32_t tmem_base_sh;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t q0 = (int64_t)blockIdx.y * TC_M, x0 = (int64_t)blockIdx.x * TC_N;
@@ -83,7 +117,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_dot_kernel(const float* __re
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
   if (tid == 0) {
-    mbar_init(&mbar, 1);
+    mbar_init(&mbar[0], 1);
+    mbar_init(&mbar[1], 1);
     mbar_fence_init();
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -91,55 +126,45 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_dot_kernel(const float* __re
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = tmem_base_sh;
 
-  uint32_t phase = 0;
+  uint32_t ph0 = 0, ph1 = 0;  // parity of the next completion of mbar[0] / mbar[1]
   const int nkb = (d + TC_K - 1) / TC_K;
+  tc_stage(sm, Qh, Ql, qb, q0, Xh, Xl, nb, x0, d, 0, tid);
   for (int kb = 0; kb < nkb; ++kb) {
-    const int k0 = kb * TC_K;
-    // ---- stage the K block: 16-B chunks, zero past the matrix edges
-    // (unrolled so several loads of a thread are in flight at once)
-#pragma unroll 4
-    for (int t = tid; t < TC_M * (TC_K / 4); t += TC_THREADS) {
-      const int r = t >> 3, c = t & 7;
-      float4 h = make_float4(0.f, 0.f, 0.f, 0.f), l = h;
-      if (q0 + r < qb && k0 + c * 4 < d) {
-        h = *reinterpret_cast<const float4*>(Qh + (q0 + r) * d + k0 + c * 4);
-        l = *reinterpret_cast<const float4*>(Ql + (q0 + r) * d + k0 + c * 4);
-      }
-      *reinterpret_cast<float4*>(a_hi + tile_off(r, c)) = h;
-      *reinterpret_cast<float4*>(a_lo + tile_off(r, c)) = l;
-    }
-#pragma unroll 4
-    for (int t = tid; t < TC_N * (TC_K / 4); t += TC_THREADS) {
-      const int r = t >> 3, c = t & 7;
-      float4 h = make_float4(0.f, 0.f, 0.f, 0.f), l = h;
-      if (x0 + r < nb && k0 + c * 4 < d) {
-        h = *reinterpret_cast<const float4*>(Xh + (x0 + r) * d + k0 + c * 4);
-        l = *reinterpret_cast<const float4*>(Xl + (x0 + r) * d + k0 + c * 4);
-      }
-      *reinterpret_cast<float4*>(b_hi + tile_off(r, c)) = h;
-      *reinterpret_cast<float4*>(b_lo + tile_off(r, c)) = l;
-    }
-    fence_proxy_async_smem();  // generic-proxy tile writes -> visible to the tensor core (async proxy)
+    const int b = kb & 1;
+    uint8_t* buf = sm + (size_t)b * kStageBytes;
+    asm volatile("cp.async.wait_group 0;" ::: "memory");  // this thread's copies of block kb landed
+    fence_proxy_async_smem();  // tile writes -> visible to the tensor core (async proxy)
     __syncthreads();
     if (tid == 0) {
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const uint32_t a_hi = smem_u32(buf), a_lo = a_hi + TC_M * TC_K * 4;
+      const uint32_t b_hi = a_lo + TC_M * TC_K * 4, b_lo = b_hi + TC_N * TC_K * 4;
       // 4 K steps of 8 (two 16-B chunks each) x 3 products
 #pragma unroll
       for (int s = 0; s < TC_K / 8; ++s) {
         const uint32_t off = (uint32_t)s * 256;
-        const uint64_t ah = smem_desc(smem_u32(a_hi) + off, 128, 1024), al = smem_desc(smem_u32(a_lo) + off, 128, 1024);
-        const uint64_t bh = smem_desc(smem_u32(b_hi) + off, 128, 1024), bl = smem_desc(smem_u32(b_lo) + off, 128, 1024);
+        const uint64_t ah = smem_desc(a_hi + off, 128, 1024), al = smem_desc(a_lo + off, 128, 1024);
+        const uint64_t bh = smem_desc(b_hi + off, 128, 1024), bl = smem_desc(b_lo + off, 128, 1024);
         mma_tf32(tmem, ah, bh, (kb | s) ? 1u : 0u);  // Q hi . X hi
         mma_tf32(tmem, ah, bl, 1u);                  // Q hi . X lo
         mma_tf32(tmem, al, bh, 1u);                  // Q lo . X hi
       }
-      asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(&mbar))
+      asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                       smem_u32(&mbar[b]))
                    : "memory");
     }
-    mbar_wait(&mbar, phase);  // the MMAs have read the tiles (and, at the end, D is complete)
-    phase ^= 1u;
-    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if (kb + 1 < nkb) {
+      // the other buffer was last read by block kb-1's MMAs
+      if (kb >= 1) {
+        if (b == 0) { mbar_wait(&mbar[1], ph1); ph1 ^= 1u; }
+        else        { mbar_wait(&mbar[0], ph0); ph0 ^= 1u; }
+      }
+      tc_stage(sm + (size_t)(b ^ 1) * kStageBytes, Qh, Ql, qb, q0, Xh, Xl, nb, x0, d, (kb + 1) * TC_K, tid);
+    }
   }
+  // the last block's commit covers every earlier MMA (they complete in order)
+  if (((nkb - 1) & 1) == 0) mbar_wait(&mbar[0], ph0); else mbar_wait(&mbar[1], ph1);
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 
   // ---- epilogue: TMEM lanes 32w.. of warp w = its query rows; 32 columns per load
   const int64_t row = q0 + warp * 32 + lane;
@@ -181,7 +206,7 @@ int tc_dot_3xtf32(const float* Qh, const float* Ql, int64_t qb, const float* Xh,
                   float* D, int64_t ldD, cudaStream_t st) {
   if (qb <= 0 || nb <= 0) return ALGAS_OK;
   if (d % 4 != 0 || ldD % 4 != 0) return set_error(ALGAS_EINVAL, "tc_dot: d and ldD must be multiples of 4");
-  const int smem = (TC_M + TC_N) * TC_K * 4 * 2;  // 96 KB
+  const int smem = 2 * kStageBytes;  // two stages of 96 KB
   ALGAS_CUDA_TRY(cudaFuncSetAttribute(tc_dot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   const dim3 grid((unsigned)((nb + TC_N - 1) / TC_N), (unsigned)((qb + TC_M - 1) / TC_M));
   tc_dot_kernel<<<grid, TC_THREADS, smem, st>>>(Qh, Ql, qb, Xh, Xl, nb, d, D, ldD);
