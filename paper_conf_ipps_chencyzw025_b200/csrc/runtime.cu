@@ -23,20 +23,43 @@ namespace algas {
 
 // ------------------------------------------------------------------ A9 merge
 int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t* out_ids, float* out_d) {
-  // heap entry: (dist, id, cta, pos) -- min-heap on (dist, id)
+  // binary min-heap on (dist, id) over the T list heads, in a per-thread
+  // buffer (the poller merges every query: no allocation on this path)
   struct H {
     float d;
     uint32_t id;
     int c, p;
   };
-  auto greater = [](const H& a, const H& b) {
-    if (a.d != b.d) return a.d > b.d;
-    return a.id > b.id;
+  auto less = [](const H& a, const H& b) { return a.d < b.d || (a.d == b.d && a.id < b.id); };
+  thread_local std::vector<H> heap;
+  if ((int)heap.size() < T) heap.resize(T);
+  int hn = 0;
+  auto push = [&](H h) {
+    int i = hn++;
+    while (i > 0) {
+      const int par = (i - 1) >> 1;
+      if (!less(h, heap[par])) break;
+      heap[i] = heap[par];
+      i = par;
+    }
+    heap[i] = h;
   };
-  std::priority_queue<H, std::vector<H>, decltype(greater)> pq(greater);
+  auto pop_top = [&]() {
+    const H last = heap[--hn];
+    int i = 0;
+    for (;;) {
+      int c = 2 * i + 1;
+      if (c >= hn) break;
+      if (c + 1 < hn && less(heap[c + 1], heap[c])) ++c;
+      if (!less(heap[c], last)) break;
+      heap[i] = heap[c];
+      i = c;
+    }
+    heap[i] = last;
+  };
   for (int c = 0; c < T; ++c) {
     const ResultEntry& e = res[(size_t)c * kin];
-    if (kin > 0 && e.id != kSentinel) pq.push(H{e.dist, e.id, c, 0});
+    if (kin > 0 && e.id != kSentinel) push(H{e.dist, e.id, c, 0});
   }
   int n = 0;
   // repeated ids (R11): a linear scan of the emitted ids for small k, an
@@ -54,9 +77,9 @@ int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t*
       if (set[h] == kSentinel) { set[h] = id; return false; }
     }
   };
-  while (!pq.empty() && n < k) {
-    H h = pq.top();
-    pq.pop();
+  while (hn > 0 && n < k) {
+    const H h = heap[0];
+    pop_top();
     bool dup = false;
     if (use_set) {
       dup = seen_insert(h.id);
@@ -71,7 +94,7 @@ int32_t merge_cta_lists(const ResultEntry* res, int T, int kin, int k, uint32_t*
     }
     if (h.p + 1 < kin) {
       const ResultEntry& e = res[(size_t)h.c * kin + h.p + 1];
-      if (e.id != kSentinel) pq.push(H{e.dist, e.id, h.c, h.p + 1});
+      if (e.id != kSentinel) push(H{e.dist, e.id, h.c, h.p + 1});
     }
   }
   for (int i = n; i < k; ++i) {
@@ -153,6 +176,7 @@ struct algas_server {
     algas_query_stats st;
   };
   std::deque<Done> cq;
+  std::vector<Done> done_pool;  // recycled completion records (their vectors keep their capacity)
   std::atomic<int64_t> inflight{0};
   // host FIFO of enqueued queries not yet in a slot (algas_enqueue): the
   // poller thread moves the head into a slot the moment one is recycled
@@ -307,6 +331,13 @@ static void poller_main(algas_server* s, int me, int nth) {
       }
       any = true;
       algas_server::Done d;
+      {
+        std::lock_guard<std::mutex> lk(s->cq_mu);
+        if (!s->done_pool.empty()) {
+          d = std::move(s->done_pool.back());
+          s->done_pool.pop_back();
+        }
+      }
       d.tag = s->tags[q];
       const int k = s->kq[q];
       const ResultEntry* r = s->res_h + (size_t)q * T * s->kmax;
@@ -590,6 +621,7 @@ int algas_poll(algas_server* s, uint64_t* tags, uint32_t* ids, float* dists, alg
     if (ids) memcpy(ids + (size_t)n * s->kmax, d.ids.data(), sizeof(uint32_t) * s->kmax);
     if (dists) memcpy(dists + (size_t)n * s->kmax, d.d.data(), sizeof(float) * s->kmax);
     if (stats) stats[n] = d.st;
+    if (s->done_pool.size() < 4096) s->done_pool.push_back(std::move(d));  // keep its buffers for the poller
     s->cq.pop_front();
     ++n;
   }
