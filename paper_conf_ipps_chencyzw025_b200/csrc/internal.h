@@ -107,7 +107,9 @@ inline void choose_smem(int dp4, int L, int ncap, int S, int w, int Rp, int64_t 
   *hash_bits = hb;
   *stage_rows = sr;
 }
-int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent);
+int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent,
+              bool allow_dsmem = true);
+int launch_cluster_size(const Plan& pl);
 
 // spill tables: ensure >= entries, returns base pointer (workspace locked by caller)
 int ensure_gtab(algas_index* idx, size_t entries);

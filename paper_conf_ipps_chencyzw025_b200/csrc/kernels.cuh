@@ -77,7 +77,7 @@ template <int NT, int TL, int CPL, int METRIC>
 __global__ void __launch_bounds__(NT) batch_kernel(BatchArgs a) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const SmemLayout lay = smem_layout(a.cfg.dp4, a.cfg.L, a.cfg.ncap, a.cfg.hash_bits, a.cfg.stage_rows,
-                                       gc_bytes(a.cfg.gc_bits, a.cfg.rp_shift));
+                                       gc_bytes(a.cfg.gc_bits, a.cfg.rp_shift), a.cfg.vis_dsmem * a.cfg.vis_words * 4);
   const Smem s = carve(smem_raw, lay);
   init_cta<NT>(s, a.cfg);
   __shared__ int s_item;
@@ -118,7 +118,7 @@ template <int NT, int TL, int CPL, int METRIC, int CS, int MINB = 1>
 __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const SmemLayout lay = smem_layout(A.cfg.dp4, A.cfg.L, A.cfg.ncap, A.cfg.hash_bits, A.cfg.stage_rows,
-                                       gc_bytes(A.cfg.gc_bits, A.cfg.rp_shift));
+                                       gc_bytes(A.cfg.gc_bits, A.cfg.rp_shift), A.cfg.vis_dsmem * A.cfg.vis_words * 4);
   const Smem s = carve(smem_raw, lay);
   init_cta<NT>(s, A.cfg, CS);
   if constexpr (CS > 1) cluster_barrier();  // every CTA's mbarriers exist before any remote arrive
@@ -247,6 +247,9 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     const unsigned long long mb = s_mbox;
     if (mb == kMboxQuit) {
       if constexpr (CS > 1) post_quit<CS>(s);
+      // DSMEM bitmap: no CTA of the cluster leaves while another may still
+      // address its shared memory (every CTA of a slot sees the same quit)
+      if (A.cfg.vis_dsmem) cluster_barrier();
       break;
     }
     const uint32_t epoch = (uint32_t)(mb >> 32);
@@ -295,9 +298,21 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       const uint4 z = make_uint4(0u, 0u, 0u, 0u);
       for (int64_t i = lo + tid; i < hi; i += NT) o4[i] = z;
     }
+    if (A.cfg.vis_dsmem) {
+      // SHARED bitmap in distributed shared memory (vis_claim): this CTA
+      // clears its share for the new query; the cluster barrier below orders
+      // every share's clear before any CTA's first claim.  No CTA of the slot
+      // still claims into a share for the previous query: rank 0 picks a
+      // query up only after the slot's finish counter shows all T CTAs done
+      // (both feeds), and the others start it only through rank 0's mailbox.
+      uint4* v4 = reinterpret_cast<uint4*>(s.vsh);
+      const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+      for (int i = tid; i < (A.cfg.vis_words >> 2); i += NT) v4[i] = z;
+    }
     if (A.cfg.cosine) normalize_query<NT>(s.q, A.cfg.d4);  // COSINE (R29), before the cluster push
     if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
-    __syncthreads();
+    if (A.cfg.vis_dsmem) cluster_barrier();  // also a CTA barrier
+    else __syncthreads();
 
     const QPar qp{par.y, par.z, A.cfg.off < par.y ? A.cfg.off : par.y};
     const int k = par.x;

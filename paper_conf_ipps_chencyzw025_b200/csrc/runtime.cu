@@ -492,7 +492,7 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   if ((e = cudaMalloc(&s->gtab, gent * 8)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc spill tables: %s", cudaGetErrorString(e)));
   cudaMemset(s->gtab, 0, gent * 8);
-  const int64_t vw = s->plan.cfg.shared ? shared_bitmap_words(idx->n) : 0;
+  const int64_t vw = (s->plan.cfg.shared && !s->plan.cfg.vis_dsmem) ? shared_bitmap_words(idx->n) : 0;
   if (vw > 0 && (e = cudaMalloc(&s->vbm, (size_t)slots * 2 * vw * 4)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc visited bitmaps: %s", cudaGetErrorString(e)));
   if (vw > 0) cudaMemset(s->vbm, 0, (size_t)slots * 2 * vw * 4);

@@ -78,7 +78,7 @@ static int take_epochs(algas_index* idx, uint64_t count, uint32_t* base, cudaStr
   return ALGAS_OK;
 }
 
-int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent) {
+int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* out, bool persistent, bool allow_dsmem) {
   Plan pl;
   memset(&pl, 0, sizeof(pl));
   const int L = p->itopk, k = p->k, w = p->width;
@@ -148,6 +148,29 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
       gcbits = 0;
   }
   const int gcb = gc_bytes(gcbits, idx->rp_shift);
+  // SHARED visited bitmap in distributed shared memory (vis_claim): a
+  // persistent grid of single-CTA searches whose T (a power of two <= 8) CTAs
+  // of a slot form one thread-block cluster, each holding 1/T of the n-bit
+  // bitmap, if that share fits next to a visited hash of >= 2^12 entries;
+  // else the slot's bitmap in HBM.  ALGAS_VIS_DSMEM=0 turns it off (A/B).
+  int vis_dsmem = 0, vis_words = 0, vis_tshift = 0;
+  if (allow_dsmem && persistent && cs == 1 && gather_mode == 0 && p->visited_mode == ALGAS_VISITED_SHARED && T <= 8 &&
+      (T & (T - 1)) == 0) {
+    const char* ve = getenv("ALGAS_VIS_DSMEM");
+    if (!ve || atoi(ve) != 0) {
+      while ((1 << vis_tshift) < T) ++vis_tshift;
+      const int64_t words = (idx->n + 31) / 32;
+      const int64_t share = (((words + T - 1) / T) + 3) & ~int64_t(3);
+      int hb_min = 12;
+      while ((1LL << hb_min) < 2LL * (S + w * Rp)) ++hb_min;
+      if (share * 4 <= (1 << 20) &&
+          smem_layout(dp4, L, ncap, p->hash_bits > 0 ? p->hash_bits : hb_min, 0, gcb, (int)share * 4).total <= budget) {
+        vis_dsmem = 1;
+        vis_words = (int)share;
+      }
+    }
+  }
+  const int vsb = vis_dsmem ? vis_words * 4 : 0;
   int team_rows = 0;
   if (gather_mode == 4) {
     // hybrid: one register pass + team_rows staged rows per team in flight
@@ -168,11 +191,11 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
       --team_rows;
     sr = (nteams * team_rows + 1) / 2;  // smem_layout reserves 2 x sr staging rows
   }
-  choose_smem(dp4, L, ncap, S, w, Rp, budget - gcb, &hb, &sr);
+  choose_smem(dp4, L, ncap, S, w, Rp, budget - gcb - vsb, &hb, &sr);
   if (hb < 6 || hb > 16) return set_error(ALGAS_EINVAL, "hash_bits %d not in [6,16]", hb);
   if ((1 << hb) < 2 * (S + w * Rp))
     return set_error(ALGAS_EINVAL, "visited hash 2^%d too small for seeds + one step (%d)", hb, S + w * Rp);
-  SmemLayout lay = smem_layout(dp4, L, ncap, hb, sr, gcb);
+  SmemLayout lay = smem_layout(dp4, L, ncap, hb, sr, gcb, vsb);
   if (lay.total + reserved > optin)
     return set_error(ALGAS_EINVAL, "search needs %d B shared memory per CTA, device allows %d", lay.total, optin);
 
@@ -211,16 +234,32 @@ int make_plan(const algas_index* idx, const algas_params* p, int slots, Plan* ou
   c.seed = p->seed;
   c.cosine = idx->metric == ALGAS_COSINE ? 1 : 0;
   c.shared = p->visited_mode == ALGAS_VISITED_SHARED ? 1 : 0;
+  c.vis_dsmem = vis_dsmem;
+  c.vis_tshift = vis_tshift;
+  c.vis_words = vis_words;
   if (c.shared && cs > 1) return set_error(ALGAS_EINVAL, "SHARED visited mode needs cluster_size 1");
   int nb = 0;
   int rc = max_blocks_per_sm(pl, persistent, &nb);
   if (rc != ALGAS_OK) return rc;
   if (nb < 1) return set_error(ALGAS_EINVAL, "search kernel does not fit on an SM (smem %d)", pl.smem);
   pl.blocks_per_sm = nb;
-  (void)slots;
+  if (vis_dsmem && T > 1) {
+    // the slots' clusters of T CTAs must all be co-resident; if
+    // they are not, plan again with the HBM bitmap
+    int ncl = 0;
+    rc = max_active_clusters(pl, &ncl);
+    if (rc != ALGAS_OK || ncl < slots) {
+      (void)cudaGetLastError();
+      return make_plan(idx, p, slots, out, persistent, false);
+    }
+  }
   *out = pl;
   return ALGAS_OK;
 }
+
+// CTAs per thread-block cluster of a persistent launch: a cluster-split
+// search (cluster_size), or the T CTAs of a slot sharing a DSMEM bitmap
+int launch_cluster_size(const Plan& pl) { return pl.cluster > 1 ? pl.cluster : (pl.cfg.vis_dsmem ? pl.T : 1); }
 
 static int num_sms() {
   int dev = 0, n = 0;
@@ -232,7 +271,7 @@ static int num_sms() {
 // Every slot's searches must be co-resident for the persistent kernel to
 // make progress (Eq. P:L231 with the measured occupancy).
 int check_coresident(const Plan& pl, int slots) {
-  if (pl.cluster <= 1) {
+  if (launch_cluster_size(pl) <= 1) {
     if ((int64_t)slots * pl.T > (int64_t)pl.blocks_per_sm * num_sms())
       return set_error(ALGAS_EINVAL, "%d slots x %d CTAs exceed co-resident capacity %d x %d SMs (P:L231)", slots,
                        pl.T, pl.blocks_per_sm, num_sms());
@@ -241,9 +280,10 @@ int check_coresident(const Plan& pl, int slots) {
   int nc = 0;
   int rc = max_active_clusters(pl, &nc);
   if (rc) return rc;
-  if ((int64_t)slots * pl.T > nc)
+  const int64_t need = pl.cluster > 1 ? (int64_t)slots * pl.T : (int64_t)slots;
+  if (need > nc)
     return set_error(ALGAS_EINVAL, "%d slots x %d searches exceed the %d co-resident %d-CTA clusters (P:L231)", slots,
-                     pl.T, nc, pl.cluster);
+                     pl.T, nc, launch_cluster_size(pl));
   return ALGAS_OK;
 }
 
@@ -655,7 +695,7 @@ int algas_search_dynamic(const algas_index* cidx, const float* queries_dev, int6
   pa.gtab = ws->gtab;
   pa.epoch_base = ebase;
   // SHARED visited bitmaps: two per slot (zeroed here; each query's CTAs clear the other one)
-  if (pl.cfg.shared && (pa.vbm_words = shared_bitmap_words(idx->n)) > 0) {
+  if (pl.cfg.shared && !pl.cfg.vis_dsmem && (pa.vbm_words = shared_bitmap_words(idx->n)) > 0) {
     void* vbp = nullptr;
     if ((rc = ensure_scratch(ws, 3, (size_t)slots * 2 * pa.vbm_words * 4, &vbp))) return rc;
     ALGAS_CUDA_TRY(cudaMemsetAsync(vbp, 0, (size_t)slots * 2 * pa.vbm_words * 4, st));

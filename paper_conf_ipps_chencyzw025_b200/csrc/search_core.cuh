@@ -225,6 +225,11 @@ struct SearchCfg {
                          //    hash is this CTA's cache of it
   int32_t cosine;        // 1: COSINE index (unit data rows, METRIC = kIP): the staged query is
                          //    normalised in shared memory (normalize_query) before the search
+  int32_t vis_dsmem;     // 1: SHARED visited bitmap in distributed shared memory -- the query's
+                         //    T CTAs form a thread-block cluster and CTA r holds bitmap words
+                         //    w with w % T == r (vis_words u32 each); claims are DSMEM atomics
+  int32_t vis_tshift;    //    log2 T (T = 1, 2, 4, 8)
+  int32_t vis_words;     //    u32 words of this CTA's share (multiple of 4)
   uint64_t seed;
 };
 
@@ -269,7 +274,7 @@ constexpr int kMergeParts = 1024;
 
 struct SmemLayout {
   int off_q, off_listA, off_listB, off_newk, off_newid, off_sel, off_part, off_hash, off_stage, off_bar, off_ctrl,
-      off_gc, total;
+      off_gc, off_vsh, total;
 };
 // bytes of a graph-row cache of 2^gc_bits rows of Rp ids + tag + stamp per row
 __host__ __device__ inline int gc_bytes(int gc_bits, int rp_shift) {
@@ -277,7 +282,7 @@ __host__ __device__ inline int gc_bytes(int gc_bits, int rp_shift) {
 }
 __host__ __device__ inline int align16(int x) { return (x + 15) & ~15; }
 __host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int hash_bits, int stage_rows,
-                                                   int gcb = 0) {
+                                                   int gcb = 0, int vsh_bytes = 0) {
   SmemLayout s;
   int o = 0;
   s.off_stage = o; o += 2 * stage_rows * dp4 * 16;  // 128-B aligned at offset 0
@@ -292,6 +297,7 @@ __host__ __device__ inline SmemLayout smem_layout(int dp4, int L, int ncap, int 
   s.off_bar = o;   o += 32;
   s.off_ctrl = o;  o += align16((int)sizeof(Ctrl));
   s.off_gc = o;    o += align16(gcb);
+  s.off_vsh = o;   o += align16(vsh_bytes);
   s.total = o;
   return s;
 }
@@ -308,6 +314,7 @@ struct Smem {
   uint64_t* bar;    // 2 mbarriers
   Ctrl* ctrl;
   uint32_t* gcache; // graph-row cache: rows [2^gc_bits][Rp], then tags, then stamps
+  uint32_t* vsh;    // vis_dsmem: this CTA's share of the query's SHARED visited bitmap
 };
 __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
   Smem s;
@@ -323,6 +330,7 @@ __device__ __forceinline__ Smem carve(uint8_t* base, const SmemLayout& l) {
   s.bar = reinterpret_cast<uint64_t*>(base + l.off_bar);
   s.gcache = reinterpret_cast<uint32_t*>(base + l.off_gc);
   s.ctrl = reinterpret_cast<Ctrl*>(base + l.off_ctrl);
+  s.vsh = reinterpret_cast<uint32_t*>(base + l.off_vsh);
   return s;
 }
 // once per CTA lifetime (kernel start): staging barriers; zero staging and
@@ -380,6 +388,24 @@ __device__ __forceinline__ bool smem_contains(const uint32_t* tab, int bits, uin
   }
   return false;
 }
+// SHARED visited bitmap: atomic test-and-set of id's bit in the
+// query's bitmap; true if this call set it.  vis_dsmem: the bitmap is spread
+// over the shared memory of the query's T CTAs (one thread-block cluster),
+// word w in CTA w % T -- one DSMEM atomic (~200 cycles) instead of an L2
+// atomic that queues behind the step's row traffic; else the slot's HBM
+// bitmap (vbm).
+__device__ __forceinline__ bool vis_claim(const SearchCfg& cfg, uint32_t* vsh, uint32_t* vbm, uint32_t id) {
+  const uint32_t bit = 1u << (id & 31), w = id >> 5;
+  if (cfg.vis_dsmem) {
+    const uint32_t owner = w & ((1u << cfg.vis_tshift) - 1u), lw = w >> cfg.vis_tshift;
+    uint32_t ra, old;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(vsh + lw)), "r"(owner));
+    asm volatile("atom.relaxed.cluster.shared::cluster.or.b32 %0, [%1], %2;" : "=r"(old) : "r"(ra), "r"(bit) : "memory");
+    return (old & bit) == 0u;
+  }
+  return (atomicOr(vbm + w, bit) & bit) == 0u;
+}
+
 // epoch-tagged HBM table: entry = (epoch << 32) | id; an entry of another
 // epoch counts as empty, so the table never needs clearing.
 __device__ __forceinline__ int gmem_visit(unsigned long long* tab, int bits, uint32_t epoch, uint32_t id) {
@@ -1056,7 +1082,7 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
       keep = smem_visit(s.hash, hbits, e) == kVisNew;
       // SHARED: a CTA keeps its own seeds even when another CTA of the
       // query claimed them first (R21), but marks them for the others
-      if (keep && cfg.shared && vbm) atomicOr(vbm + (e >> 5), 1u << (e & 31));
+      if (keep && cfg.shared && (vbm || cfg.vis_dsmem)) (void)vis_claim(cfg, s.vsh, vbm, e);
       else if (keep && cfg.shared && gtab) (void)gmem_visit(gtab, cfg.gtab_bits, epoch, e);
     }
     const unsigned m = __ballot_sync(0xffffffffu, keep);
@@ -1204,12 +1230,11 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
                 for (int o = 0; o < cfg.d4 * 16; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rp + o));
               }
               if (keep && cfg.shared) {  // new to this CTA: claim it in the query's table (P:L211, P:L217 step 2)
-                if (vbm) {                // the paper's bitmap: one L2 atomic, no probing --
-                  if (!(cfg.prefetch & 256)) {  // (A/B, bit 256: with the row's loads in dist_ldg instead --
+                if (vbm || cfg.vis_dsmem) {  // the paper's bitmap: one atomic, no probing --
+                  if (!(cfg.prefetch & 256) || cfg.vis_dsmem) {  // (A/B, bit 256: with the row's loads in dist_ldg instead --
                                                   //  measured slower: the rows other CTAs won cost more
                                                   //  than the round trip saved, profiles/round2_ab.md)
-                    const uint32_t bit = 1u << (id & 31);
-                    keep = (atomicOr(vbm + (id >> 5), bit) & bit) == 0u;
+                    keep = vis_claim(cfg, s.vsh, vbm, id);
                   }
                 } else {
                   const int g = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
@@ -1217,11 +1242,8 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
                   if (g == kVisFull) atomicOr(&C->overflow, 1);
                 }
               }
-            } else if (vbm) {
-              if (!smem_contains(s.hash, hbits, id)) {
-                const uint32_t bit = 1u << (id & 31);
-                keep = (atomicOr(vbm + (id >> 5), bit) & bit) == 0u;
-              }
+            } else if (vbm || cfg.vis_dsmem) {
+              if (!smem_contains(s.hash, hbits, id)) keep = vis_claim(cfg, s.vsh, vbm, id);
             } else if (!smem_contains(s.hash, hbits, id)) {
               const int r = gmem_visit(gtab, cfg.gtab_bits, epoch, id);
               keep = (r == kVisNew);

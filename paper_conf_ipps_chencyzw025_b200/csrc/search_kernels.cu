@@ -48,13 +48,14 @@ int max_active_clusters(const Plan& pl, int* out) {
   void* fn = kernel_for(pl, pl.metric, true);
   if (!fn) return set_error(ALGAS_EINVAL, "no persistent kernel for cluster=%d", pl.cluster);
   ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem));
+  const int csz = launch_cluster_size(pl);
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(pl.cluster);
+  cfg.gridDim = dim3(csz);
   cfg.blockDim = dim3(pl.nt);
   cfg.dynamicSmemBytes = pl.smem;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeClusterDimension;
-  at[0].val.clusterDim.x = pl.cluster;
+  at[0].val.clusterDim.x = csz;
   at[0].val.clusterDim.y = 1;
   at[0].val.clusterDim.z = 1;
   cfg.attrs = at;
@@ -108,9 +109,9 @@ int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st) {
   at[na].id = cudaLaunchAttributeCooperative;
   at[na].val.cooperative = 1;
   ++na;
-  if (pl.cluster > 1) {
+  if (launch_cluster_size(pl) > 1) {
     at[na].id = cudaLaunchAttributeClusterDimension;
-    at[na].val.clusterDim.x = pl.cluster;
+    at[na].val.clusterDim.x = launch_cluster_size(pl);
     at[na].val.clusterDim.y = 1;
     at[na].val.clusterDim.z = 1;
     ++na;
