@@ -129,9 +129,17 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
   const int slot = unit / P.T;
   const int rank = unit % P.T;
   const int tid = threadIdx.x;
-  __shared__ unsigned long long s_mbox;
-  __shared__ int4 s_par;
-  __shared__ unsigned long long s_tag, s_t0;
+  // start message of a query: mailbox word, tag, params (32 B, one unit for
+  // the DSMEM push of cluster slots)
+  struct __align__(16) StartMsg {
+    unsigned long long mbox, tag;
+    int4 par;
+  };
+  __shared__ StartMsg s_start;
+  __shared__ unsigned long long s_t0;
+  unsigned long long& s_mbox = s_start.mbox;
+  unsigned long long& s_tag = s_start.tag;
+  int4& s_par = s_start.par;
 
   if constexpr (CS > 1) {
     if (crank != 0) {
@@ -168,7 +176,10 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         // CTAs consumed them, and in SHARED mode the bitmap share a CTA
         // clears at its next pickup is no longer in use by a slower CTA
         // (R26).  Wrap-safe difference of u32 counters.
-        while ((int)(ld_acquire_gpu32(P.slot_fin + slot) - served * (uint32_t)P.T) < 0) __nanosleep(32);
+        // (DSMEM-bitmap slots: the first cluster barrier below gives the same
+        // guarantee)
+        if (!A.cfg.vis_dsmem)
+          while ((int)(ld_acquire_gpu32(P.slot_fin + slot) - served * (uint32_t)P.T) < 0) __nanosleep(32);
         if (P.mode == 0) {
           // host ring: poll the slot state in host memory, or its
           // device mirror in HBM (state_mirror: no PCIe read while polling)
@@ -203,7 +214,33 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         s_t0 = globaltimer();
       }
       __syncthreads();
-      if (s_mbox != kMboxQuit && P.mode == 0) {
+      if (A.cfg.vis_dsmem) {
+        // cluster slot: the query, params and tag go to this CTA's shared
+        // memory only; the other CTAs receive them through DSMEM below
+        if (s_mbox != kMboxQuit) {
+          if (P.mode == 0) {
+            const uint8_t* ment = P.mir ? P.mir + (size_t)(2 * slot + sub) * P.mir_stride : nullptr;
+            const RingSlot* rs = ment ? reinterpret_cast<const RingSlot*>(ment) : &P.ring[2 * slot + sub];
+            const float4* src = ment ? reinterpret_cast<const float4*>(ment + sizeof(RingSlot))
+                                     : P.ring_q + (uint64_t)(2 * slot + sub) * A.cfg.d4;
+            for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = ld_volatile_f4(src + i);
+            if (tid == NT - 1) {
+              const int4 sp4 = ld_volatile_i4(reinterpret_cast<const int4*>(rs));
+              s_par = make_int4(sp4.y, sp4.z, sp4.w, 0);
+            }
+            if (tid == NT - 2) s_tag = *((const volatile unsigned long long*)&rs->tag);
+          } else {
+            const uint32_t item = (uint32_t)s_mbox;
+            const float4* qsrc = P.queries + (uint64_t)item * A.cfg.d4;
+            for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = qsrc[i];
+            if (tid == 0) {
+              s_par = make_int4(P.kmax, A.cfg.L, A.cfg.w, 0);
+              s_tag = P.tag0 + (uint64_t)item;
+            }
+          }
+          if (A.cfg.cosine) normalize_query<NT>(s.q, A.cfg.d4);  // COSINE (R29): pushed normalised
+        }
+      } else if (s_mbox != kMboxQuit && P.mode == 0) {
         // payload from mapped host memory in ONE PCIe round trip: the query
         // chunks, {state, k, L, w} and the tag are read by different threads
         // at once (volatile: never a stale line; ordered after thread 0's
@@ -226,11 +263,11 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
         if (tid == NT - 2) P.dtag[slot] = *((const volatile unsigned long long*)&rs->tag);
       }
       __syncthreads();
-      if (tid == 0) {
+      if (tid == 0 && !A.cfg.vis_dsmem) {
         __threadfence();
         st_release_gpu64(P.mbox + slot, s_mbox);
       }
-    } else {
+    } else if (!A.cfg.vis_dsmem) {
       if (tid == 0) {
         unsigned long long mb;
         for (;;) {
@@ -244,19 +281,45 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       }
       __syncthreads();
     }
+    if (A.cfg.vis_dsmem) {
+      // cluster slot start: barrier 1 -- every CTA finished the previous
+      // query (so no share is claimed into and no query buffer is read any
+      // more) and rank 0 holds the next item; rank 0 then writes {mailbox,
+      // params, tag} and the query into the other CTAs' shared memory
+      // (DSMEM), every CTA clears its bitmap share; barrier 2 publishes both.
+      cluster_barrier();
+      if (tid == 0) s_t0 = globaltimer();  // the slot is free: the query starts now
+      if (rank == 0) {
+        const int nq4 = A.cfg.d4 + 2;  // query chunks + the 32-B start message
+        for (int i = tid; i < nq4 * (P.T - 1); i += NT) {
+          const int r = 1 + i / nq4, c = i % nq4;
+          const uint4* lp = c < A.cfg.d4 ? reinterpret_cast<const uint4*>(s.q + c)
+                                          : reinterpret_cast<const uint4*>(&s_start) + (c - A.cfg.d4);
+          uint32_t ra;
+          asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(lp)), "r"(r));
+          const uint4 v = *lp;
+          asm volatile("st.shared::cluster.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(ra), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                       : "memory");
+        }
+      }
+      uint4* v4 = reinterpret_cast<uint4*>(s.vsh);
+      const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+      for (int i = tid; i < (A.cfg.vis_words >> 2); i += NT) v4[i] = z;
+      cluster_barrier();
+    }
     const unsigned long long mb = s_mbox;
     if (mb == kMboxQuit) {
       if constexpr (CS > 1) post_quit<CS>(s);
-      // DSMEM bitmap: no CTA of the cluster leaves while another may still
-      // address its shared memory (every CTA of a slot sees the same quit)
-      if (A.cfg.vis_dsmem) cluster_barrier();
-      break;
+      break;  // (cluster slots: no CTA addresses another's shared memory after barrier 2)
     }
     const uint32_t epoch = (uint32_t)(mb >> 32);
     const uint32_t item = (uint32_t)mb;
     int4 par;
     uint64_t tag;
-    if (P.mode == 0) {
+    if (A.cfg.vis_dsmem) {
+      par = s_par;  // delivered with the query (cluster slot start)
+      tag = s_tag;
+    } else if (P.mode == 0) {
       // host ring: per-query params published by rank 0 with the mailbox
       if (tid == 0) {
         const volatile int* vp = reinterpret_cast<const volatile int*>(P.dparams + slot);
@@ -274,7 +337,9 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
 
     // ---------------- stage the query into shared memory (rank 0 of a ring
     // slot already holds it from the PCIe read)
-    if (P.mode == 1) {
+    if (A.cfg.vis_dsmem) {
+      // (the query is in s.q already, normalised for COSINE)
+    } else if (P.mode == 1) {
       const float4* qsrc = P.queries + (uint64_t)item * A.cfg.d4;
       for (int i = tid; i < A.cfg.d4; i += NT) s.q[i] = qsrc[i];
     } else if (rank != 0) {
@@ -298,21 +363,11 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       const uint4 z = make_uint4(0u, 0u, 0u, 0u);
       for (int64_t i = lo + tid; i < hi; i += NT) o4[i] = z;
     }
-    if (A.cfg.vis_dsmem) {
-      // SHARED bitmap in distributed shared memory (vis_claim): this CTA
-      // clears its share for the new query; the cluster barrier below orders
-      // every share's clear before any CTA's first claim.  No CTA of the slot
-      // still claims into a share for the previous query: rank 0 picks a
-      // query up only after the slot's finish counter shows all T CTAs done
-      // (both feeds), and the others start it only through rank 0's mailbox.
-      uint4* v4 = reinterpret_cast<uint4*>(s.vsh);
-      const uint4 z = make_uint4(0u, 0u, 0u, 0u);
-      for (int i = tid; i < (A.cfg.vis_words >> 2); i += NT) v4[i] = z;
+    if (!A.cfg.vis_dsmem) {
+      if (A.cfg.cosine) normalize_query<NT>(s.q, A.cfg.d4);  // COSINE (R29), before the cluster push
+      if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
+      __syncthreads();
     }
-    if (A.cfg.cosine) normalize_query<NT>(s.q, A.cfg.d4);  // COSINE (R29), before the cluster push
-    if constexpr (CS > 1) push_query<NT, CS>(s, A.cfg.d4);  // released by the first step signal
-    if (A.cfg.vis_dsmem) cluster_barrier();  // also a CTA barrier
-    else __syncthreads();
 
     const QPar qp{par.y, par.z, A.cfg.off < par.y ? A.cfg.off : par.y};
     const int k = par.x;
