@@ -1198,6 +1198,10 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
         np_step = np;
         const int spilled = C->spilled;
         const int total = np << cfg.rp_shift;  // one neighbour id per thread and pass
+        // SHARED with the query's bitmap: no CTA-local hash in the step
+        // (prefetch bit 2048 keeps it as a filter in front of the claim, A/B)
+        const bool bitmap_only =
+            cfg.shared && (cfg.vis_dsmem || (vbm != nullptr && !(cfg.prefetch & 256))) && !(cfg.prefetch & 2048);
         for (int base = 0; base < total; base += NT) {
           const int idx = base + tid;
           uint32_t id = kSentinel;
@@ -1213,7 +1217,13 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
           }
           bool keep = false;
           if (id != kSentinel) {
-            if (!spilled) {
+            if (bitmap_only) {
+              // SHARED bitmap: it holds every point this CTA has
+              // visited too (own seeds included, R21), so it alone is the
+              // visited set -- one atomic, no shared-memory hash probe
+              // (measured ~900 cycles per step, the ATOMS.CAS test-and-set)
+              keep = vis_claim(cfg, s.vsh, vbm, id);
+            } else if (!spilled) {
               const int r = smem_visit(s.hash, hbits, id);
               keep = (r == kVisNew);
               if (r == kVisFull) atomicOr(&C->overflow, 1);

@@ -71,10 +71,11 @@ def main():
                                 ("select", "gather", "dist", "sort")},
                "hist_max_iters": np.bincount(st["max_iters"], minlength=1).tolist()[:30]}
         if os.environ.get("SUBLAP"):  # -DALGAS_SUBLAP=1 build: per-warp gather sub-phases (first pass)
-            ws = np.maximum(st["merges_rank"].astype(np.float64), 1)
-            out["sub_idhash_cyc"] = round(float(st["cyc_select"].sum() / ws.sum()))
-            out["sub_claim_cyc"] = round(float(st["merges_bitonic"].astype(np.float64).sum() / ws.sum()))
-            out["sub_warps_per_step"] = round(float(ws.sum() / np.maximum(st["iters"], 1).sum()), 1)
+            ws = max(float(st["merges_rank"].astype(np.float64).sum()), 1.0)
+            out["sub_id_cyc"] = round(float(st["cyc_select"].astype(np.float64).sum() / ws))
+            out["sub_hash_cyc"] = round(float(st["merges_bitonic"].astype(np.float64).sum() / ws))
+            out["sub_claim_cyc"] = round(float(st["cap_hits"].astype(np.float64).sum() / ws))
+            out["sub_warps_per_step"] = round(ws / max(float(st["iters"].astype(np.float64).sum()), 1.0), 1)
         print(json.dumps(out), flush=True)
 
 
