@@ -885,6 +885,59 @@ __device__ __forceinline__ uint64_t warp_bitonic_merge32(uint64_t list, uint64_t
   return m;
 }
 
+// ---- select (P:L217 step 1) from the registers of warp 0 (list striped:
+// lane l, register e = position 32e + l): the first w unchecked keys in list
+// order (one under greedy search), R6/R7, marked checked; the first L keys
+// are written to dst and the step's control words updated.
+template <int E>
+__device__ __forceinline__ void warp_select_store(const SearchCfg& cfg, const Smem& s, Ctrl* C, int lane,
+                                                  uint64_t (&x)[E], uint64_t* dst, int L, int W, int OFF, int sp,
+                                                  uint32_t liters, int cur, int lcnt) {
+  int tot = 0, first_un = -1;
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const unsigned um = __ballot_sync(0xffffffffu, 32 * e + lane < lcnt && !(x[e] & 1ull));
+    if (first_un < 0 && um) first_un = 32 * e + __ffs(um) - 1;
+    tot += __popc(um);
+  }
+  const int diff0 = __shfl_sync(0xffffffffu, lane == 0 ? C->diffusing : 0, 0);
+  int done = 0, np = 0, diff = diff0;
+  if (tot == 0) {
+    done = 1;
+  } else if ((int)liters >= cfg.max_iter) {
+    done = 1;
+    if (lane == 0) C->cap_hit = 1;
+  } else {
+    if (first_un >= OFF) diff = 1;        // P:L249 (sticky, R6)
+    np = diff ? (tot < W ? tot : W) : 1;  // P:L200
+    int base = 0;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const bool un = 32 * e + lane < lcnt && !(x[e] & 1ull);
+      const unsigned um = __ballot_sync(0xffffffffu, un);
+      const int rank = base + __popc(um & ((1u << lane) - 1u));
+      if (un && rank < np) {
+        s.sel[32 + rank] = (int)key_id(x[e]);
+        x[e] |= 1ull;                           // mark checked (Alg.1 l.7)
+      }
+      base += __popc(um);
+    }
+  }
+#pragma unroll
+  for (int e = 0; e < E; ++e)
+    if (32 * e + lane < L) dst[32 * e + lane] = x[e];
+  if (lane == 0) {
+    C->diffusing = diff;
+    C->done = done;
+    C->np = np;
+    C->nnew[sp ^ 1] = 0;
+    C->nkeys[sp ^ 1] = 0;
+    if (!done) C->parents += np;
+    C->cur = cur;
+    C->cnt = lcnt;
+  }
+}
+
 // Candidate update of the fused path ("parallel-friendly bitonic
 // sort ... merges the candidate list and expand list"), for lists of up to
 // Lp = 32*E keys: warp 0 holds the sorted list in registers, STRIPED (lane l,
@@ -949,50 +1002,53 @@ __device__ __forceinline__ void warp_merge_select(const SearchCfg& cfg, const Sm
     dst = const_cast<uint64_t*>(src);
   }
   liters += np_step > 0 ? 1 : 0;
-  // ---- select (P:L217 step 1) from the registers: the first w unchecked
-  // keys in list order (one under greedy search), R6/R7
-  int tot = 0, first_un = -1;
-#pragma unroll
-  for (int e = 0; e < E; ++e) {
-    const unsigned um = __ballot_sync(0xffffffffu, 32 * e + lane < lcnt && !(x[e] & 1ull));
-    if (first_un < 0 && um) first_un = 32 * e + __ffs(um) - 1;
-    tot += __popc(um);
-  }
-  const int diff0 = __shfl_sync(0xffffffffu, lane == 0 ? C->diffusing : 0, 0);
-  int done = 0, np = 0, diff = diff0;
-  if (tot == 0) {
-    done = 1;
-  } else if ((int)liters >= cfg.max_iter) {
-    done = 1;
-    if (lane == 0) C->cap_hit = 1;
-  } else {
-    if (first_un >= OFF) diff = 1;        // P:L249 (sticky, R6)
-    np = diff ? (tot < W ? tot : W) : 1;  // P:L200
-    int base = 0;
-#pragma unroll
-    for (int e = 0; e < E; ++e) {
-      const bool un = 32 * e + lane < lcnt && !(x[e] & 1ull);
-      const unsigned um = __ballot_sync(0xffffffffu, un);
-      const int rank = base + __popc(um & ((1u << lane) - 1u));
-      if (un && rank < np) {
-        s.sel[32 + rank] = (int)key_id(x[e]);
-        x[e] |= 1ull;                           // mark checked (Alg.1 l.7)
+  warp_select_store<E>(cfg, s, C, lane, x, dst, L, W, OFF, sp, liters, cur, lcnt);
+}
+
+// Candidate update for lists of <= 32 keys, fused with the next
+// select: a merge BY RANK in parallel warps instead of warp 0's bitonic
+// networks.  New key i goes to position #(new keys < it) + #(list keys < it)
+// (a lower bound in the sorted list), list key j to j + #(new keys < it);
+// keys are unique, so the positions are a permutation and the first L form
+// the merged list -- the same list the bitonic merge produces.  Warps
+// 0..nblk-1 place the new keys (32 each, <= 128), warp nblk the list keys,
+// each comparison a shared-memory broadcast read; one named barrier, then
+// warp 0 selects from the merged list.  Needs NT >= 160.
+template <int NT>
+__device__ __forceinline__ void rank_merge_select32(const SearchCfg& cfg, const Smem& s, Ctrl* C, int warp, int lane,
+                                                    int cnt, int nk, int L, int W, int OFF, int sp, uint32_t& liters,
+                                                    int np_step, int& cur, int& lcnt) {
+  const uint64_t* src = cur ? s.list[1] : s.list[0];
+  uint64_t* dst = cur ? s.list[0] : s.list[1];
+  const int nblk = (nk + 31) >> 5;
+  if (nk > 0 && warp <= nblk) {
+    if (warp < nblk) {
+      const int i = 32 * warp + lane;
+      if (i < nk) {
+        const uint64_t key = s.newk[i];
+        int r = lower_bound_u64(src, cnt, key);
+        for (int j = 0; j < nk; ++j) r += (s.newk[j] < key) ? 1 : 0;
+        if (r < L) dst[r] = key;
       }
-      base += __popc(um);
+    } else if (lane < cnt) {
+      const uint64_t key = src[lane];
+      int r = lane;
+      for (int j = 0; j < nk; ++j) r += (s.newk[j] < key) ? 1 : 0;
+      if (r < L) dst[r] = key;
     }
+    asm volatile("bar.sync 1, %0;" ::"r"(32 * (nblk + 1)) : "memory");
   }
-#pragma unroll
-  for (int e = 0; e < E; ++e)
-    if (32 * e + lane < L) dst[32 * e + lane] = x[e];
-  if (lane == 0) {
-    C->diffusing = diff;
-    C->done = done;
-    C->np = np;
-    C->nnew[sp ^ 1] = 0;
-    C->nkeys[sp ^ 1] = 0;
-    if (!done) C->parents += np;
-    C->cur = cur;
-    C->cnt = lcnt;
+  if (warp == 0) {
+    if (nk > 0) {
+      cur ^= 1;
+      lcnt = (cnt + nk) < L ? cnt + nk : L;
+    } else {
+      dst = const_cast<uint64_t*>(src);
+    }
+    liters += np_step > 0 ? 1 : 0;
+    uint64_t x[1];
+    x[0] = lane < lcnt ? dst[lane] : kKeyMax;
+    warp_select_store<1>(cfg, s, C, lane, x, dst, L, W, OFF, sp, liters, cur, lcnt);
   }
 }
 
@@ -1407,15 +1463,24 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
       if (CS == 1 && L <= 32 * kMaxE && nk <= kWarpMergeMax && !(cfg.prefetch & (64 | 2))) {
         uint64_t* sorted2 = reinterpret_cast<uint64_t*>(s.part);  // blocks 1..3, sorted
         const int nblk = (nk + 31) >> 5;
+        // lists of <= 32 keys: merge by rank in parallel warps (prefetch bit
+        // 4096: warp 0's bitonic networks instead, A/B)
+        const bool by_rank = (NT >= 160) && L <= 32 && !(cfg.prefetch & 4096);
+        if (by_rank) {
+          if constexpr (NT >= 160) {
+            if (tid == 0) C->mg_bitonic++;
+            rank_merge_select32<NT>(cfg, s, C, warp, lane, cnt, nk, L, W, OFF, sp, liters, np_step, cur, lcnt);
+          }
+        }
         if constexpr (NT >= 128) {
-          if (warp >= 1 && warp < nblk) {
+          if (!by_rank && warp >= 1 && warp < nblk) {
             const uint64_t x = (32 * warp + lane < nk) ? s.newk[32 * warp + lane] : kKeyMax;
             sorted2[32 * warp + lane] = warp_bitonic_sort32(x, lane);
             __threadfence_block();
             asm volatile("bar.arrive 1, %0;" ::"r"(32 * nblk) : "memory");
           }
         }
-        if (warp == 0) {
+        if (warp == 0 && !by_rank) {
           if (tid == 0) C->mg_bitonic++;
           if (L <= 32)
             warp_merge_select<1, NT>(cfg, s, C, lane, cnt, nk, nblk, sorted2, L, W, OFF, sp, liters, np_step, cur, lcnt);
