@@ -23,6 +23,8 @@ graph and parameters) timed on the host cores, rank 0 only.
 from __future__ import annotations
 
 import argparse
+import csv
+import io
 import json
 import os
 import subprocess
@@ -376,6 +378,45 @@ def cpu_baseline(W, w, p, gpu_ids, budget_s=8.0):
             "unique_parents_T1": round(float(st1["parents"].mean()), 1)}
 
 
+def ncu_traffic(a, p, W):
+    """DRAM bytes (read + write) of ONE launch of the persistent kernel at the
+    chosen operating point, from an ncu pass over the same index, queries and
+    parameters in a child process (ncu replays the kernel; nothing timed here
+    comes from it).  Returns (bytes per launch, source) or (None, reason)."""
+    import shutil
+    import subprocess
+    import tempfile
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return None, "ncu not found"
+    d = tempfile.mkdtemp(prefix="algas_ncu_")
+    try:
+        np.save(os.path.join(d, "X.npy"), W["X"].cpu().numpy() if hasattr(W["X"], "cpu") else W["X"])
+        np.save(os.path.join(d, "G.npy"), W["G"].cpu().numpy() if hasattr(W["G"], "cpu") else W["G"])
+        pj = {f: getattr(p, f) for f, _ in p._fields_ if not f.startswith("reserved")}
+        cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum", "--print-units", "base", "--csv",
+               "--clock-control", "none", "-k", "regex:persistent_kernel", "-c", "1", sys.executable,
+               os.path.join(ROOT, "scripts", "profile_run.py"), a.config, "--nq", str(a.nq), "--load", d,
+               "--params-json", json.dumps(pj), "--reps", "1"]
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=a.ncu_timeout)
+        tot = 0.0
+        seen = 0
+        for row in csv.reader(io.StringIO(r.stdout)):
+            if len(row) >= 3 and row[-3] in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+                tot += float(row[-1].replace(",", ""))
+                seen += 1
+        if seen != 2 or not np.isfinite(tot) or tot <= 0:
+            os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+            with open(os.path.join(ROOT, "gpurun_out", "ncu_traffic.log"), "w") as f:
+                f.write(" ".join(cmd[:12]) + "\n--- stdout\n" + r.stdout[-20000:] + "\n--- stderr\n" + r.stderr[-20000:])
+            return None, f"ncu rc={r.returncode}: no dram counters (gpurun_out/ncu_traffic.log)"
+        return tot, "ncu dram__bytes_read.sum + dram__bytes_write.sum, one launch, this run"
+    except Exception as e:  # noqa: BLE001 -- the bench line must still print
+        return None, f"ncu failed: {type(e).__name__}"
+    finally:
+        shutil.rmtree(d, ignore_errors=True)
+
+
 def run_algas(a, rank, world, local):
     import torch
     import torch.distributed as dist
@@ -461,9 +502,11 @@ def run_algas(a, rank, world, local):
     kernel_s = float(np.mean(kern_ms)) / 1e3
     achieved = algo_bytes_per_launch / kernel_s / 1e9
     peak, peak_src = _peaks()
-    traffic = None
+    traffic, traffic_src = None, None
+    if rank == 0 and not a.no_ncu:
+        traffic, traffic_src = ncu_traffic(a, p, W)
     tp = os.path.join(ROOT, "profiles", f"traffic_{a.config}.json")
-    if os.path.exists(tp):
+    if traffic is None and os.path.exists(tp):
         # an ncu capture only counts for the same launch configuration
         try:
             tj = json.load(open(tp))
@@ -471,6 +514,7 @@ def run_algas(a, rank, world, local):
                        for f in ("itopk", "width", "ctas_per_query", "threads_per_cta", "slots", "visited_mode"))
             if same and tj.get("dram_bytes_per_launch_per_query") is not None:
                 traffic = float(tj["dram_bytes_per_launch_per_query"]) * a.nq
+                traffic_src = os.path.relpath(tp, ROOT)
         except Exception:
             traffic = None
 
@@ -550,7 +594,8 @@ def run_algas(a, rank, world, local):
         "e2e": e2e,
         "gpu_launches": a.steps,
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
+                     "frac": round(achieved / peak, 4), "traffic": traffic, "traffic_source": traffic_src,
+                     "peak_source": peak_src,
                      "kernel": "persistent_kernel", "algo_bytes_per_query": round(float(bytes_q.mean())),
                      "unique_bytes_per_query": unique_b,
                      "kernel_ms": round(float(np.mean(kern_ms)), 3)},
@@ -770,6 +815,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--no-ncu", action="store_true", help="no in-run ncu pass for roofline.traffic")
+    ap.add_argument("--ncu-timeout", type=float, default=240.0)
     a = ap.parse_args()
     if a.warmup < 3:
         a.warmup = 3

@@ -106,9 +106,15 @@ int launch_persistent(const Plan& pl, const PersistArgs& pa, cudaStream_t st) {
   cfg.stream = st;
   cudaLaunchAttribute at[2];
   int na = 0;
-  at[na].id = cudaLaunchAttributeCooperative;
-  at[na].val.cooperative = 1;
-  ++na;
+  // cooperative launch for single-CTA units (the runtime refuses a grid that
+  // cannot be co-resident); cluster grids are checked against
+  // cudaOccupancyMaxActiveClusters by make_plan / check_coresident instead
+  // (a cooperative cluster launch fails under ncu's kernel replay)
+  if (launch_cluster_size(pl) <= 1) {
+    at[na].id = cudaLaunchAttributeCooperative;
+    at[na].val.cooperative = 1;
+    ++na;
+  }
   if (launch_cluster_size(pl) > 1) {
     at[na].id = cudaLaunchAttributeClusterDimension;
     at[na].val.clusterDim.x = launch_cluster_size(pl);

@@ -76,6 +76,12 @@ def main():
             out["sub_hash_cyc"] = round(float(st["merges_bitonic"].astype(np.float64).sum() / ws))
             out["sub_claim_cyc"] = round(float(st["cap_hits"].astype(np.float64).sum() / ws))
             out["sub_warps_per_step"] = round(ws / max(float(st["iters"].astype(np.float64).sum()), 1.0), 1)
+        if os.environ.get("SUBLAP") == "2":  # merge-phase probes (diagnosis build)
+            its = max(float(st["iters"].astype(np.float64).sum()), 1.0)
+            out["m_entry"] = round(float(st["cyc_select"].astype(np.float64).sum() / its))
+            out["m_keyload"] = round(float(st["merges_bitonic"].astype(np.float64).sum() / its))
+            out["m_lowerbound"] = round(float(st["cap_hits"].astype(np.float64).sum() / its))
+            out["m_loop"] = round(float(st["merges_rank"].astype(np.float64).sum() / its), 1)
         print(json.dumps(out), flush=True)
 
 

@@ -31,18 +31,28 @@ def main():
     ap.add_argument("--slots", type=int, default=32)
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--batch-kernel", action="store_true")
+    ap.add_argument("--load", default=None, help="directory with X.npy / G.npy (bench.py's built index)")
+    ap.add_argument("--params-json", default=None, help="algas_params fields (overrides the flags)")
     a = ap.parse_args()
     w = synth.WORKLOADS[a.cfg]
-    X = synth.base_vectors(w)
     Q = synth.query_vectors(w, a.nq)
-    Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
-    knn, _ = algas.knn(Xd, Xd, w.knn_degree, w.metric, self_base=0)
-    G = algas.prune(knn, w.degree) if w.prune else knn[:, :w.degree].contiguous()
-    del knn
+    Qd = torch.from_numpy(Q).cuda()
+    if a.load:
+        Xd = torch.from_numpy(np.load(os.path.join(a.load, "X.npy"))).cuda()
+        G = np.load(os.path.join(a.load, "G.npy"))
+    else:
+        Xd = torch.from_numpy(synth.base_vectors(w)).cuda()
+        knn, _ = algas.knn(Xd, Xd, w.knn_degree, w.metric, self_base=0)
+        G = algas.prune(knn, w.degree) if w.prune else knn[:, :w.degree].contiguous()
+        del knn
     idx = algas.Index(Xd, G, w.metric)
-    p = algas.default_params(k=w.k, itopk=a.itopk, width=a.width, offset_beam=a.offset if a.offset > 0 else max(1, a.itopk // 4),
-                             ctas_per_query=a.ctas, threads_per_cta=a.threads, slots=a.slots, seed=1,
-                             visited_mode=1 if a.visited == "shared" else 0)
+    if a.params_json:
+        p = algas.default_params(**json.loads(a.params_json))
+    else:
+        p = algas.default_params(k=w.k, itopk=a.itopk, width=a.width,
+                                 offset_beam=a.offset if a.offset > 0 else max(1, a.itopk // 4),
+                                 ctas_per_query=a.ctas, threads_per_cta=a.threads, slots=a.slots, seed=1,
+                                 visited_mode=1 if a.visited == "shared" else 0)
     out = []
     for _ in range(a.reps):
         if a.batch_kernel:
@@ -52,8 +62,8 @@ def main():
         st = r["stats"]
         out.append(dict(kernel_ms=r["info"].kernel_ms, parents=float(st["parents"].mean()),
                         dist_evals=float(st["dist_evals"].mean()), iters=float(st["iters"].mean())))
-    print(json.dumps(dict(cfg=a.cfg, nq=a.nq, itopk=a.itopk, width=a.width, offset=p.offset_beam, threads=a.threads,
-                          ctas=a.ctas,
+    print(json.dumps(dict(cfg=a.cfg, nq=a.nq, itopk=p.itopk, width=p.width, offset=p.offset_beam,
+                          threads=p.threads_per_cta, ctas=p.ctas_per_query,
                           slots=a.slots, runs=out)))
 
 
