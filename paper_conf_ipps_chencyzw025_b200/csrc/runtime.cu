@@ -141,6 +141,8 @@ struct algas_server {
   std::vector<uint32_t> next_ep; // per slot: epoch of its next query
   std::vector<int> next_sub;     // per slot: sub-slot of its next query
   std::unique_ptr<std::atomic<int>[]> slot_lock;  // per slot: claim lock
+  std::unique_ptr<std::atomic<int>[]> slot_busy;  // per slot: sub-slots not free (0..2)
+  std::atomic<int> n_idle_slots{0};               // slots with both sub-slots free
   std::vector<uint64_t> tags;
   std::vector<int> kq;
   std::vector<std::chrono::steady_clock::time_point> t_submit;
@@ -257,7 +259,10 @@ void write_slot(algas_server* s, int u, const float* query, uint64_t tag, int32_
 // 0 -> 1) and give it the slot's next epoch, scanning slots from `start`, a
 // slot with nothing in flight first; returns the sub-slot index or -1
 int claim_slot(algas_server* s, int start) {
-  for (int pass = 0; pass < 2; ++pass) {
+  // pass 0 (a slot with nothing in flight) only while such a slot exists:
+  // under load every slot is busy and the scan would cost the poller ~1 us
+  // per query (the count is advisory: a stale value only changes placement)
+  for (int pass = s->n_idle_slots.load(std::memory_order_relaxed) > 0 ? 0 : 1; pass < 2; ++pass) {
     for (int i = 0; i < s->slots; ++i) {
       const int q = (start + i) % s->slots;
       int unlocked = 0;
@@ -270,6 +275,8 @@ int claim_slot(algas_server* s, int start) {
         const uint32_t ne = (s->next_ep[q] + 1) & 0xFFFFFFu;
         s->next_ep[q] = ne == 0 ? 1 : ne;
         s->next_sub[q] ^= 1;
+        if (s->slot_busy[q].fetch_add(1, std::memory_order_relaxed) == 0)
+          s->n_idle_slots.fetch_sub(1, std::memory_order_relaxed);
         s->slot_lock[q].store(0, std::memory_order_release);
         return u;
       }
@@ -362,6 +369,8 @@ static void poller_main(algas_server* s, int me, int nth) {
       __atomic_store_n(&s->ring_h[q].state, quit ? (uint32_t)kSlotQuit : (ep << 8) | kSlotEmpty, __ATOMIC_RELEASE);
       if (quit && s->mirror) mirror_publish(s, q, kSlotQuit, false);
       s->queue_ns[q] = 0;
+      if (s->slot_busy[q >> 1].fetch_sub(1, std::memory_order_relaxed) == 1)
+        s->n_idle_slots.fetch_add(1, std::memory_order_relaxed);
       (*s->hstate)[q].store(0, std::memory_order_release);
       drain_pending(s, q >> 1);
       {
@@ -479,6 +488,9 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   s->next_sub.assign(slots, 1);  // the kernel serves sub-slot 1 first, then alternates
   s->slot_lock.reset(new std::atomic<int>[slots]);
   for (int q = 0; q < slots; ++q) s->slot_lock[q].store(0);
+  s->slot_busy.reset(new std::atomic<int>[slots]);
+  for (int q = 0; q < slots; ++q) s->slot_busy[q].store(0);
+  s->n_idle_slots.store(slots);
   const size_t ctl_bytes = control_bytes(slots);
   if ((e = cudaMalloc(&s->ctl, ctl_bytes)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc: %s", cudaGetErrorString(e)));
