@@ -410,7 +410,7 @@ def ncu_traffic(a, p, W):
             with open(os.path.join(ROOT, "gpurun_out", "ncu_traffic.log"), "w") as f:
                 f.write(" ".join(cmd[:12]) + "\n--- stdout\n" + r.stdout[-20000:] + "\n--- stderr\n" + r.stderr[-20000:])
             return None, f"ncu rc={r.returncode}: no dram counters (gpurun_out/ncu_traffic.log)"
-        return tot, "ncu dram__bytes_read.sum + dram__bytes_write.sum, one launch, this run"
+        return tot, "ncu dram rd+wr, 1 launch, this run"
     except Exception as e:  # noqa: BLE001 -- the bench line must still print
         return None, f"ncu failed: {type(e).__name__}"
     finally:
@@ -589,7 +589,7 @@ def run_algas(a, rank, world, local):
                    "target_met": target_met, "graph": w.build,
                    "parallelism": f"replicas x{world}", "l2": "256MB flush/step"},
         "latency_us": {"p50": round(float(np.percentile(lat, 50)), 1), "p99": round(float(np.percentile(lat, 99)), 1),
-                       "def": "device: pickup->published"},
+                       "def": "device pickup->publish"},
         "clocks": clk.summary(),
         "e2e": e2e,
         "gpu_launches": a.steps,

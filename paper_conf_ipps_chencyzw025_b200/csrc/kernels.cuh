@@ -287,7 +287,11 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
       // more) and rank 0 holds the next item; rank 0 then writes {mailbox,
       // params, tag} and the query into the other CTAs' shared memory
       // (DSMEM), every CTA clears its bitmap share; barrier 2 publishes both.
-      cluster_barrier();
+      // Barrier 1 needs no release: the previous query's DSMEM claims all
+      // returned their words (performed), and the shared-memory data rank 0
+      // pushes was ordered by its own __syncthreads; the results still in
+      // flight to host memory are ordered by their Finish word's release.
+      cluster_barrier_relaxed();
       if (tid == 0) s_t0 = globaltimer();  // the slot is free: the query starts now
       if (rank == 0) {
         const int nq4 = A.cfg.d4 + 2;  // query chunks + the 32-B start message
@@ -394,7 +398,7 @@ __global__ void __launch_bounds__(NT, MINB) persistent_kernel(PKArgs A) {
     __syncthreads();
     // ---------------- Finish
     // device-scope finish count, which gates the slot's next pickup: thread 0
-    if (tid == 0) {
+    if (tid == 0 && !A.cfg.vis_dsmem) {  // (cluster slots start on a cluster barrier instead)
       __threadfence();
       atomicAdd(P.slot_fin + slot, 1u);
     }

@@ -505,6 +505,12 @@ __device__ __forceinline__ void stage_issue(const SearchCfg& cfg, const Smem& s,
 __device__ __forceinline__ void cluster_barrier() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+// the same barrier without release semantics on the arrive: a thread's
+// earlier writes (e.g. results still on their way to host memory) need not
+// be performed before it arrives
+__device__ __forceinline__ void cluster_barrier_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+}
 template <typename T>
 __device__ __forceinline__ T* rank_ptr(T* local, int rank) {
   // generic address of the same shared-memory object in cluster CTA `rank`
@@ -1138,7 +1144,12 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
       keep = smem_visit(s.hash, hbits, e) == kVisNew;
       // SHARED: a CTA keeps its own seeds even when another CTA of the
       // query claimed them first (R21), but marks them for the others
-      if (keep && cfg.shared && (vbm || cfg.vis_dsmem)) (void)vis_claim(cfg, s.vsh, vbm, e);
+      if (keep && cfg.shared && (vbm || cfg.vis_dsmem)) {
+        // (the returned word is consumed: the claim is performed before this
+        // thread reaches the next query's relaxed start barrier)
+        const bool c = vis_claim(cfg, s.vsh, vbm, e);
+        asm volatile("" ::"r"((int)c));
+      }
       else if (keep && cfg.shared && gtab) (void)gmem_visit(gtab, cfg.gtab_bits, epoch, e);
     }
     const unsigned m = __ballot_sync(0xffffffffu, keep);
