@@ -175,8 +175,10 @@ def _search_case(name, n_sample, itopk, width, T, threads, shared):
         # SHARED over the whole 2000-query stream x 3 seeds (6000 query runs,
         # paired SE ~0.001): the GPU's asynchronous claiming is another
         # admissible interleaving than the oracle's step-by-step round robin
-        # (R25); measured gap 0.0035-0.0056 over four boxes -> bound 0.008
-        assert np.mean(rg) >= np.mean(ro) - 0.008, (rg, ro)
+        # (R25).  With the DSMEM bitmap the measured gap at the bench point
+        # (L=12, T=4) is 0.0021-0.0026 over three boxes -> the north-star
+        # bound; at L=24, T=2 it is 0.0027-0.0042 -> bound 0.008
+        assert np.mean(rg) >= np.mean(ro) - (0.005 if T == 4 else 0.008), (rg, ro)
     if shared:
         # SHARED: which CTA claims a point first is timing-dependent
         # on the GPU; the oracle's step-by-step round robin is one admissible
