@@ -1011,23 +1011,25 @@ __device__ __forceinline__ void warp_merge_select(const SearchCfg& cfg, const Sm
   warp_select_store<E>(cfg, s, C, lane, x, dst, L, W, OFF, sp, liters, cur, lcnt);
 }
 
-// Candidate update for lists of <= 32 keys, fused with the next
+// Candidate update for lists of <= 32*E keys, fused with the next
 // select: a merge BY RANK in parallel warps instead of warp 0's bitonic
 // networks.  New key i goes to position #(new keys < it) + #(list keys < it)
 // (a lower bound in the sorted list), list key j to j + #(new keys < it);
 // keys are unique, so the positions are a permutation and the first L form
 // the merged list -- the same list the bitonic merge produces.  Warps
-// 0..nblk-1 place the new keys (32 each, <= 128), warp nblk the list keys,
-// each comparison a shared-memory broadcast read; one named barrier, then
-// warp 0 selects from the merged list.  Needs NT >= 160.
-template <int NT>
-__device__ __forceinline__ void rank_merge_select32(const SearchCfg& cfg, const Smem& s, Ctrl* C, int warp, int lane,
-                                                    int cnt, int nk, int L, int W, int OFF, int sp, uint32_t& liters,
-                                                    int np_step, int& cur, int& lcnt) {
+// 0..nblk-1 place the new keys (32 each, <= 128), warps nblk..nblk+E-1 the
+// list keys (32 each), each comparison a shared-memory broadcast read; one
+// named barrier, then warp 0 selects from the merged list.  Needs
+// NT >= 32 * (4 + E).
+template <int E, int NT>
+__device__ __forceinline__ void rank_merge_select(const SearchCfg& cfg, const Smem& s, Ctrl* C, int warp, int lane,
+                                                  int cnt, int nk, int L, int W, int OFF, int sp, uint32_t& liters,
+                                                  int np_step, int& cur, int& lcnt) {
   const uint64_t* src = cur ? s.list[1] : s.list[0];
   uint64_t* dst = cur ? s.list[0] : s.list[1];
   const int nblk = (nk + 31) >> 5;
-  if (nk > 0 && warp <= nblk) {
+  const int nlw = (cnt + 31) >> 5;  // list warps (<= E)
+  if (nk > 0 && warp < nblk + nlw) {
     if (warp < nblk) {
       const int i = 32 * warp + lane;
       if (i < nk) {
@@ -1036,13 +1038,16 @@ __device__ __forceinline__ void rank_merge_select32(const SearchCfg& cfg, const 
         for (int j = 0; j < nk; ++j) r += (s.newk[j] < key) ? 1 : 0;
         if (r < L) dst[r] = key;
       }
-    } else if (lane < cnt) {
-      const uint64_t key = src[lane];
-      int r = lane;
-      for (int j = 0; j < nk; ++j) r += (s.newk[j] < key) ? 1 : 0;
-      if (r < L) dst[r] = key;
+    } else {
+      const int i = 32 * (warp - nblk) + lane;
+      if (i < cnt) {
+        const uint64_t key = src[i];
+        int r = i;
+        for (int j = 0; j < nk; ++j) r += (s.newk[j] < key) ? 1 : 0;
+        if (r < L) dst[r] = key;
+      }
     }
-    asm volatile("bar.sync 1, %0;" ::"r"(32 * (nblk + 1)) : "memory");
+    asm volatile("bar.sync 1, %0;" ::"r"(32 * (nblk + nlw)) : "memory");
   }
   if (warp == 0) {
     if (nk > 0) {
@@ -1052,9 +1057,10 @@ __device__ __forceinline__ void rank_merge_select32(const SearchCfg& cfg, const 
       dst = const_cast<uint64_t*>(src);
     }
     liters += np_step > 0 ? 1 : 0;
-    uint64_t x[1];
-    x[0] = lane < lcnt ? dst[lane] : kKeyMax;
-    warp_select_store<1>(cfg, s, C, lane, x, dst, L, W, OFF, sp, liters, cur, lcnt);
+    uint64_t x[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) x[e] = 32 * e + lane < lcnt ? dst[32 * e + lane] : kKeyMax;
+    warp_select_store<E>(cfg, s, C, lane, x, dst, L, W, OFF, sp, liters, cur, lcnt);
   }
 }
 
@@ -1474,13 +1480,20 @@ __device__ void search_cta(const SearchCfg& cfg, const QPar qp, const Smem& s, u
       if (CS == 1 && L <= 32 * kMaxE && nk <= kWarpMergeMax && !(cfg.prefetch & (64 | 2))) {
         uint64_t* sorted2 = reinterpret_cast<uint64_t*>(s.part);  // blocks 1..3, sorted
         const int nblk = (nk + 31) >> 5;
-        // lists of <= 32 keys: merge by rank in parallel warps (prefetch bit
-        // 4096: warp 0's bitonic networks instead, A/B)
-        const bool by_rank = (NT >= 160) && L <= 32 && !(cfg.prefetch & 4096);
+        // merge by rank in parallel warps (lists of <= 128 keys; <= 32 with
+        // prefetch bit 16384, A/B) -- prefetch bit 4096: warp 0's bitonic
+        // networks instead (A/B)
+        const int rank_lmax = (cfg.prefetch & 16384) ? 32 : 128;
+        const bool by_rank = (NT >= 256) && L <= rank_lmax && !(cfg.prefetch & 4096);
         if (by_rank) {
-          if constexpr (NT >= 160) {
+          if constexpr (NT >= 256) {
             if (tid == 0) C->mg_bitonic++;
-            rank_merge_select32<NT>(cfg, s, C, warp, lane, cnt, nk, L, W, OFF, sp, liters, np_step, cur, lcnt);
+            if (L <= 32)
+              rank_merge_select<1, NT>(cfg, s, C, warp, lane, cnt, nk, L, W, OFF, sp, liters, np_step, cur, lcnt);
+            else if (L <= 64)
+              rank_merge_select<2, NT>(cfg, s, C, warp, lane, cnt, nk, L, W, OFF, sp, liters, np_step, cur, lcnt);
+            else
+              rank_merge_select<4, NT>(cfg, s, C, warp, lane, cnt, nk, L, W, OFF, sp, liters, np_step, cur, lcnt);
           }
         }
         if constexpr (NT >= 128) {
