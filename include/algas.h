@@ -250,6 +250,23 @@ int algas_server_create(const algas_index *idx, const algas_params *params, alga
  * host cannot submit while the launch call blocks. */
 int algas_server_create_deferred(const algas_index *idx, const algas_params *params,
                                  algas_server **out);
+/* TEST HARNESS, not a search: a server whose device side is a host thread
+ * that follows the persistent kernel's ring protocol (P:L166-172 states;
+ * the kernel's mode-0 loop in kernels.cuh) -- for tests of the host state
+ * machine (slot claim, two ring entries per slot, epochs, poller, host merge,
+ * recycle, FIFO drain, watchdog, bounded sessions) on machines without a
+ * GPU.  No CUDA call is made.  params: slots, ctas_per_query (T), k, itopk,
+ * width, host_threads, watchdog_ms are used; dim: query length (multiple of
+ * 4).  The emulated device returns a fixed function of each query, not
+ * neighbours: CTA r's list entry i is (tag*1000 + i*T + r, q[0] + i*T + r),
+ * and for T > 1 CTA 1 repeats CTA 0's first id at a larger distance, so a
+ * query's merged result is ids tag*1000 + j, dists q[0] + j, j < k.
+ * deferred != 0: the device thread starts with algas_server_start (bounded
+ * sessions).  Destroy with algas_server_destroy. */
+int algas_server_create_emulated(const algas_params *params, int32_t dim, int32_t deferred, algas_server **out);
+/* Emulated server only: the query with this tag is never finished (it stays
+ * in its slot; the watchdog reports it).  ALGAS_EINVAL on a real server. */
+int algas_server_emulated_stall(algas_server *s, uint64_t tag);
 /* Launch a deferred server's kernel.  quit_when_idle != 0 makes it a bounded
  * session: every free ring entry becomes QUIT -- now and whenever a
  * finished query's entry is recycled -- so the kernel exits after the staged

@@ -93,7 +93,8 @@ class Tuning(ctypes.Structure):
 # every symbol include/algas.h declares (checked by tests/test_abi.py)
 EXPORTS = ["algas_params_default", "algas_last_error", "algas_version", "algas_index_create",
            "algas_index_destroy", "algas_index_info", "algas_search", "algas_search_ex", "algas_search_dynamic",
-           "algas_server_create", "algas_server_create_deferred", "algas_server_start", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
+           "algas_server_create", "algas_server_create_deferred", "algas_server_create_emulated",
+           "algas_server_emulated_stall", "algas_server_start", "algas_submit", "algas_submit_many", "algas_enqueue", "algas_poll", "algas_server_inflight", "algas_server_destroy",
            "algas_merge_topk", "algas_merge_topk_parts", "algas_device_query", "algas_tuner_max_parallel", "algas_tuner_blocks_per_sm",
            "algas_tuner_smem_per_block", "algas_tune", "algas_knn", "algas_knn_last_stats", "algas_prune",
            "algas_build_graph", "algas_knn_partitioned", "algas_build_graph_partitioned", "algas_knn_refine"]
@@ -135,6 +136,8 @@ def lib(build_if_missing: bool = True):
                                            ctypes.POINTER(RunInfo)]
         L.algas_server_create.argtypes = [P, ctypes.POINTER(Params), ctypes.POINTER(P)]
         L.algas_server_create_deferred.argtypes = [P, ctypes.POINTER(Params), ctypes.POINTER(P)]
+        L.algas_server_create_emulated.argtypes = [ctypes.POINTER(Params), i32, i32, ctypes.POINTER(P)]
+        L.algas_server_emulated_stall.argtypes = [P, u64]
         L.algas_server_start.argtypes = [P, i32]
         L.algas_submit.argtypes = [P, P, u64, i32, i32, i32]
         L.algas_submit_many.argtypes = [P, P, i64, u64, i32, i32, i32, ctypes.POINTER(i64)]
@@ -305,16 +308,28 @@ class Index:
 class Server:
     """Persistent kernel + host-mapped slot ring (algas_server_*)."""
 
-    def __init__(self, index: Index, params: Params, deferred: bool = False):
+    def __init__(self, index: Index, params: Params, deferred: bool = False, emulated_dim: int = 0):
         """deferred=True: algas_server_create_deferred -- stage queries with
-        submit(), then start() launches the kernel."""
+        submit(), then start() launches the kernel.  emulated_dim > 0:
+        algas_server_create_emulated -- a TEST HARNESS whose device side is a
+        host thread following the ring protocol (no GPU; results are a fixed
+        function of the query, not a search); index must be None."""
         self.index = index
         self.params = params
         h = ctypes.c_void_p()
-        create = lib().algas_server_create_deferred if deferred else lib().algas_server_create
-        _check(create(index.handle, ctypes.byref(params), ctypes.byref(h)))
+        if emulated_dim > 0:
+            assert index is None, "an emulated server has no index"
+            _check(lib().algas_server_create_emulated(ctypes.byref(params), int(emulated_dim), 1 if deferred else 0,
+                                                      ctypes.byref(h)))
+        else:
+            create = lib().algas_server_create_deferred if deferred else lib().algas_server_create
+            _check(create(index.handle, ctypes.byref(params), ctypes.byref(h)))
         self._h = h
         self.kmax = params.k
+
+    def emulated_stall(self, tag: int) -> None:
+        """Emulated server: never finish the query with this tag."""
+        _check(lib().algas_server_emulated_stall(self._h, ctypes.c_uint64(tag)))
 
     def start(self, quit_when_idle: bool = False) -> None:
         """Launch a deferred server's kernel (algas_server_start); with

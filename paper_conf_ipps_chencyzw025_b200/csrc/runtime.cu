@@ -170,6 +170,11 @@ struct algas_server {
   uint64_t uid = 0;  // server identity for the per-thread stream cache
   std::mutex io_mu;
   std::vector<cudaStream_t> io_streams;
+  // emulated ring device (algas_server_create_emulated; protocol tests on
+  // hosts without a GPU): a host thread in place of the persistent kernel
+  bool emulated = false;
+  std::thread emu;
+  std::atomic<uint64_t> emu_stall_tag{~0ull};  // a query with this tag is never finished
   std::mutex cq_mu;
   struct Done {
     uint64_t tag;
@@ -392,9 +397,136 @@ static void poller_main(algas_server* s, int me, int nth) {
   }
 }
 
+// host-side bookkeeping of a server's ring (both the real and the emulated device)
+static void init_host_state(algas_server* s, int slots, const algas_params* params) {
+  const int nsub = 2 * slots;
+  s->uid = g_server_uid.fetch_add(1);
+  s->watchdog_ns =
+      params->watchdog_ms < 0 ? 0 : (int64_t)(params->watchdog_ms > 0 ? params->watchdog_ms : 10000) * 1000000;
+  for (auto& a : *s->hstate) a.store(0);
+  s->epoch.assign(nsub, 0);
+  s->tags.assign(nsub, 0);
+  s->kq.assign(nsub, s->kmax);
+  s->t_submit.resize(nsub);
+  s->queue_ns.assign(nsub, 0);
+  s->next_ep.assign(slots, 1);
+  s->next_sub.assign(slots, 1);  // the kernel serves sub-slot 1 first, then alternates
+  s->slot_lock.reset(new std::atomic<int>[slots]);
+  for (int q = 0; q < slots; ++q) s->slot_lock[q].store(0);
+  s->slot_busy.reset(new std::atomic<int>[slots]);
+  for (int q = 0; q < slots; ++q) s->slot_busy[q].store(0);
+  s->n_idle_slots.store(slots);
+}
+
+// Emulated ring device: the persistent kernel's side of the host-mapped ring
+// protocol (kernels.cuh, mode 0) run by a host thread, for state-machine
+// tests without a GPU.  Per slot it serves sub-slot 1 first, then alternates;
+// it takes an entry when its state reads READY with an epoch other than the
+// one it last served from that entry (or QUIT: the slot stops), and finishes
+// a query by writing T per-CTA lists and releasing each CTA's Finish word
+// (= the epoch) -- the same words, in the same order, as the kernel.  The
+// lists are a fixed function of the staged query and tag, NOT a search: CTA
+// r's entry i is (id = tag*1000 + i*T + r, dist = q[0] + i*T + r), plus, for
+// T > 1, a repeat of CTA 0's first id at a larger distance (the host merge
+// must drop it).  A query whose tag equals emu_stall_tag is never finished
+// (watchdog tests).
+static void emu_device_main(algas_server* s) {
+  const int slots = s->slots, T = s->T, kmax = s->kmax;
+  std::vector<int> sub(slots, 1), quit(slots, 0);
+  std::vector<uint32_t> last(2 * slots, 0);
+  for (;;) {
+    int live = 0, progress = 0;
+    for (int q = 0; q < slots; ++q) {
+      if (quit[q]) continue;
+      ++live;
+      const int u = 2 * q + sub[q];
+      const uint32_t st = __atomic_load_n(&s->ring_h[u].state, __ATOMIC_ACQUIRE);
+      const uint32_t kind = st & 0xFFu, ep = st >> 8;
+      if (kind == kSlotQuit) { quit[q] = 1; continue; }
+      if (kind != kSlotReady || ep == last[u]) continue;
+      const RingSlot& rs = s->ring_h[u];
+      if (rs.tag == s->emu_stall_tag.load(std::memory_order_relaxed)) continue;
+      const int k = rs.k;
+      const float q0 = s->ringq_h[(size_t)u * s->dim];
+      for (int r = 0; r < T; ++r) {
+        ResultEntry* out = s->res_h + ((size_t)u * T + r) * kmax;
+        for (int i = 0; i < kmax; ++i) {
+          if (i < k) {
+            out[i].id = (uint32_t)((rs.tag * 1000ull + (uint64_t)i * T + r) & 0x7FFFFFFFull);
+            out[i].dist = q0 + (float)(i * T + r);
+          } else {
+            out[i].id = kSentinel;
+            out[i].dist = std::numeric_limits<float>::infinity();
+          }
+        }
+        if (r == 1 && k >= 2) {  // CTA 0's first id again, farther: a duplicate to drop
+          out[k - 1].id = (uint32_t)((rs.tag * 1000ull) & 0x7FFFFFFFull);
+          out[k - 1].dist = q0 + (float)(k * T + 7);
+        }
+        CtaStats& cs = s->st_h[(size_t)u * T + r];
+        memset(&cs, 0, sizeof(cs));
+        cs.iters = 1;
+        __atomic_store_n(&s->done_h[(size_t)u * T + r], ep, __ATOMIC_RELEASE);  // Finish
+      }
+      last[u] = ep;
+      sub[q] ^= 1;
+      ++progress;
+    }
+    if (live == 0) return;
+    if (!progress) std::this_thread::yield();
+  }
+}
+
 extern "C" {
 
 static int server_create(const algas_index* cidx, const algas_params* params, algas_server** out, bool launch);
+
+int algas_server_create_emulated(const algas_params* params, int32_t dim, int32_t deferred, algas_server** out) {
+  if (!out || !params) return set_error(ALGAS_EINVAL, "null argument");
+  *out = nullptr;
+  const int slots = params->slots > 0 ? params->slots : 32;
+  const int T = params->ctas_per_query > 0 ? params->ctas_per_query : 1;
+  const int k = params->k, L = params->itopk, w = params->width;
+  if (dim < 4 || dim % 4 || slots < 1 || T < 1 || T > ALGAS_MAX_CTAS || k < 1 || L < k || w < 1)
+    return set_error(ALGAS_EINVAL, "emulated server: bad dim/slots/T/k/itopk/width");
+  algas_server* s = new algas_server();
+  s->emulated = true;
+  s->slots = slots;
+  s->T = T;
+  s->kmax = k;
+  s->dim = dim;
+  s->d4 = dim / 4;
+  s->plan.T = T;
+  s->plan.k = k;
+  s->plan.cfg.L = L;
+  s->plan.cfg.w = w;
+  const int nsub = 2 * slots;
+  s->ring_h = (RingSlot*)calloc(nsub, sizeof(RingSlot));
+  s->ringq_h = (float*)calloc((size_t)nsub * dim, 4);
+  s->res_h = (ResultEntry*)calloc((size_t)nsub * T * k, sizeof(ResultEntry));
+  s->st_h = (CtaStats*)calloc((size_t)nsub * T, sizeof(CtaStats));
+  s->done_h = (uint32_t*)calloc((size_t)nsub * T, sizeof(uint32_t));
+  s->hstate = new std::vector<std::atomic<int>>(nsub);
+  if (!s->ring_h || !s->ringq_h || !s->res_h || !s->st_h || !s->done_h) {
+    algas_server_destroy(s);
+    return set_error(ALGAS_ENOMEM, "emulated server: out of host memory");
+  }
+  init_host_state(s, slots, params);
+  if (!deferred) {
+    s->emu = std::thread(emu_device_main, s);
+    s->launched = true;
+  }
+  const int nth = std::max(1, std::min(params->host_threads > 0 ? params->host_threads : 1, slots));
+  for (int t = 0; t < nth; ++t) s->pollers.emplace_back(poller_main, s, t, nth);
+  *out = s;
+  return ALGAS_OK;
+}
+
+int algas_server_emulated_stall(algas_server* s, uint64_t tag) {
+  if (!s || !s->emulated) return set_error(ALGAS_EINVAL, "not an emulated server");
+  s->emu_stall_tag.store(tag);
+  return ALGAS_OK;
+}
 
 int algas_server_create(const algas_index* cidx, const algas_params* params, algas_server** out) {
   return server_create(cidx, params, out, true);
@@ -421,6 +553,11 @@ int algas_server_start(algas_server* s, int32_t quit_when_idle) {
   const auto now = std::chrono::steady_clock::now();
   for (int u = 0; u < 2 * s->slots; ++u)
     if ((*s->hstate)[u].load(std::memory_order_acquire) == 2) s->t_submit[u] = now;
+  if (s->emulated) {
+    s->emu = std::thread(emu_device_main, s);
+    s->launched = true;
+    return ALGAS_OK;
+  }
   const int rc = launch_persistent(s->plan, s->pa, s->stream);
   if (rc) return rc;
   s->launched = true;
@@ -465,8 +602,7 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   SRV_ALLOC(s->st_h, s->st_d, sizeof(CtaStats) * (size_t)nsub * s->T);
   SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)nsub * s->T);
 #undef SRV_ALLOC
-  s->uid = g_server_uid.fetch_add(1);
-  s->watchdog_ns = params->watchdog_ms < 0 ? 0 : (int64_t)(params->watchdog_ms > 0 ? params->watchdog_ms : 10000) * 1000000;
+  init_host_state(s, slots, params);
   s->mirror = params->state_mirror != 0;
   if (s->mirror) {
     s->mir_stride = (int64_t)sizeof(RingSlot) + (int64_t)s->dim * 4;  // 16-B multiple (dim % 4 == 0)
@@ -478,19 +614,7 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
     cudaMemset(s->mir_d, 0, (size_t)nsub * s->mir_stride);
   }
   s->hstate = new std::vector<std::atomic<int>>(nsub);
-  for (auto& a : *s->hstate) a.store(0);
-  s->epoch.assign(nsub, 0);
-  s->tags.assign(nsub, 0);
-  s->kq.assign(nsub, s->kmax);
-  s->t_submit.resize(nsub);
-  s->queue_ns.assign(nsub, 0);
-  s->next_ep.assign(slots, 1);
-  s->next_sub.assign(slots, 1);  // the kernel serves sub-slot 1 first, then alternates
-  s->slot_lock.reset(new std::atomic<int>[slots]);
-  for (int q = 0; q < slots; ++q) s->slot_lock[q].store(0);
-  s->slot_busy.reset(new std::atomic<int>[slots]);
-  for (int q = 0; q < slots; ++q) s->slot_busy[q].store(0);
-  s->n_idle_slots.store(slots);
+  init_host_state(s, slots, params);
   const size_t ctl_bytes = control_bytes(slots);
   if ((e = cudaMalloc(&s->ctl, ctl_bytes)) != cudaSuccess)
     return cleanup(set_error(ALGAS_ENOMEM, "cudaMalloc: %s", cudaGetErrorString(e)));
@@ -619,9 +743,11 @@ int algas_poll(algas_server* s, uint64_t* tags, uint32_t* ids, float* dists, alg
   *n_out = 0;
   if (max_results <= 0) return ALGAS_OK;
   // a persistent kernel that died is reported, not silently waited on
-  cudaError_t e = cudaStreamQuery(s->stream);
-  if (e != cudaSuccess && e != cudaErrorNotReady)
-    return set_error(ALGAS_ECUDA, "persistent kernel failed: %s", cudaGetErrorString(e));
+  if (!s->emulated) {
+    cudaError_t e = cudaStreamQuery(s->stream);
+    if (e != cudaSuccess && e != cudaErrorNotReady)
+      return set_error(ALGAS_ECUDA, "persistent kernel failed: %s", cudaGetErrorString(e));
+  }
   if (s->stuck.load(std::memory_order_acquire))
     return set_error(ALGAS_ESTATE, "watchdog: query tag %llu has been in its slot for more than %lld ms",
                      (unsigned long long)s->stuck_tag.load(), (long long)(s->watchdog_ns / 1000000));
@@ -651,6 +777,23 @@ int algas_server_inflight(const algas_server* s, int64_t* n) {
 int algas_server_destroy(algas_server* s) {
   if (!s) return ALGAS_OK;
   int rc = ALGAS_OK;
+  if (s->emulated) {
+    // Quit every slot, let the emulated device drain and exit, stop the pollers
+    if (s->ring_h)
+      for (int u = 0; u < 2 * s->slots; ++u) __atomic_store_n(&s->ring_h[u].state, (uint32_t)kSlotQuit, __ATOMIC_RELEASE);
+    if (s->emu.joinable()) s->emu.join();
+    s->stop.store(true);
+    for (auto& th : s->pollers)
+      if (th.joinable()) th.join();
+    free(s->ring_h);
+    free(s->ringq_h);
+    free(s->res_h);
+    free(s->st_h);
+    free(s->done_h);
+    delete s->hstate;
+    delete s;
+    return ALGAS_OK;
+  }
   if (s->ring_h && s->stream && s->launched) {
     // Quit: every slot, then wait for the kernel to exit
     for (int u = 0; u < 2 * s->slots; ++u) {
