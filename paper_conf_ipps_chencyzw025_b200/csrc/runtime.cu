@@ -602,7 +602,6 @@ static int server_create(const algas_index* cidx, const algas_params* params, al
   SRV_ALLOC(s->st_h, s->st_d, sizeof(CtaStats) * (size_t)nsub * s->T);
   SRV_ALLOC(s->done_h, s->done_d, sizeof(uint32_t) * (size_t)nsub * s->T);
 #undef SRV_ALLOC
-  init_host_state(s, slots, params);
   s->mirror = params->state_mirror != 0;
   if (s->mirror) {
     s->mir_stride = (int64_t)sizeof(RingSlot) + (int64_t)s->dim * 4;  // 16-B multiple (dim % 4 == 0)
