@@ -409,13 +409,18 @@ int algas_knn_partitioned(const float *data, int64_t n, int32_t dim, int32_t met
  * R33, the NN-descent step; not in the paper): `rounds` Jacobi rounds, each
  * giving every point p the first k by (dist, id) of its list and the
  * distances to the ids found in the first `fan` entries of the lists of its
- * first `fan` neighbours (p and ids already listed excluded).  ids / dists:
- * n x k in/out (rows sorted by (dist, id), SENTINEL / +inf padded), host or
- * device.  EINVAL: fan outside [1, min(k, 64)], k > 1024, bad dim/metric. */
+ * first `fan` neighbours (p and ids already listed excluded).  fan < 0:
+ * R35 rounds with |fan| -- p's first |fan| REVERSE neighbours (the points r
+ * whose first |fan| entries hold p, in (rank, r) order) are candidates
+ * themselves and their lists are joined like the forward ones.  ids /
+ * dists: n x k in/out (rows sorted by (dist, id), SENTINEL / +inf padded),
+ * host or device.  EINVAL: |fan| outside [1, min(k, 64)] (32 for R35),
+ * k > 1024, bad dim/metric. */
 int algas_knn_refine(const float *data, int64_t n, int32_t dim, int32_t metric, int32_t k, int32_t fan,
                      int32_t rounds, uint32_t *ids, float *dists);
 /* algas_build_graph with algas_knn_partitioned (+ refine_rounds rounds of
- * algas_knn_refine with refine_fan, 0 = none) as its kNN step; rows the
+ * algas_knn_refine with refine_fan, 0 = none; refine_fan < 0: R35 rounds
+ * with reverse neighbours) as its kNN step; rows the
  * partition left short (clusters of <= knn_degree points) are completed
  * with the exact kNN of those rows over the whole set before the prune. */
 int algas_build_graph_partitioned(const float *data, int64_t n, int32_t dim, int32_t metric,

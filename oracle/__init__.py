@@ -29,6 +29,9 @@ Parity status per function:
   * orc_knn_refine (f4, R33)               parity unpinned by the paper; pinned
     by its fixed point (an exact kNN list is unchanged), a hand-worked 1-d
     example and monotonicity (no row's k-th distance grows).
+  * orc_knn_refine_rev (f4, R35)           parity unpinned by the paper; pinned
+    by a hand-worked example (p-1 reached only through the reverse list), the
+    exact-list fixed point and the superset property over R33.
   * orc_prune (K10)                        parity unpinned by the paper (the
     CAGRA algorithm is only cited); pinned by a hand-worked
     example and invariants.
@@ -117,6 +120,8 @@ def lib():
             L.orc_prune.restype = i32
             L.orc_knn_refine.argtypes = [P, i64, i32, i32, i32, i32, P, P, P, P]
             L.orc_knn_refine.restype = i32
+            L.orc_knn_refine_rev.argtypes = [P, i64, i32, i32, i32, i32, P, P, P, P]
+            L.orc_knn_refine_rev.restype = i32
             _lib = L
     return _lib
 
@@ -226,16 +231,18 @@ def knn_partitioned(X, k: int, n_clusters: int, overlap: int, metric: int = L2):
     return ids, ds
 
 
-def knn_refine(X, ids, ds, fan: int, rounds: int = 1, metric: int = L2):
+def knn_refine(X, ids, ds, fan: int, rounds: int = 1, metric: int = L2, reverse: bool = False):
     """R33: `rounds` neighbour-of-neighbour refinement rounds (orc_knn_refine,
-    each a Jacobi round over the previous round's lists)."""
+    each a Jacobi round over the previous round's lists); reverse=True: R35,
+    the same with reverse neighbours (orc_knn_refine_rev)."""
     X = _f32(X)
     ids, ds = _u32(ids).copy(), _f32(ds).copy()
     n, k = ids.shape
     for _ in range(rounds):
         oi = np.empty_like(ids)
         od = np.empty_like(ds)
-        rc = lib().orc_knn_refine(_ptr(X), n, X.shape[1], metric, k, fan, _ptr(ids), _ptr(ds), _ptr(oi), _ptr(od))
+        fn = lib().orc_knn_refine_rev if reverse else lib().orc_knn_refine
+        rc = fn(_ptr(X), n, X.shape[1], metric, k, fan, _ptr(ids), _ptr(ds), _ptr(oi), _ptr(od))
         if rc != 0:
             raise RuntimeError("orc_knn_refine failed")
         ids, ds = oi, od

@@ -32,6 +32,10 @@
  *                                     (R33; not in the paper:
  *                                     parity unpinned by it, pinned by its
  *                                     exact fixed point and a hand example)
+ *   orc_knn_refine_rev (f4, R35)      the same round with reverse neighbours
+ *                                     joined (R35; not in the paper:
+ *                                     parity unpinned by it, pinned by a hand
+ *                                     example, fixed point, superset property)
  *   orc_prune        (K10)            CAGRA-style rank-based detour pruning +
  *                                     reverse edges (graph named at P:L293,
  *                                     algorithm from ref [25] P:L430, which is
@@ -580,5 +584,118 @@ int32_t orc_knn_refine(const float *X, int64_t n, int32_t d, int32_t metric, int
     }
     free(mark);
     free(c);
+    return 0;
+}
+
+
+/* ------------------------------------------------------------------ */
+/* f4 reading R35: the R33 round with reverse neighbours (the NN-descent  */
+/* local join over forward and reverse lists).  From the INPUT lists:     */
+/*   rev(p) = the first fan pairs (a, r), in (a, r) order, with           */
+/*            in[r][a] == p, a < fan, r != p  (p's reverse neighbours)    */
+/*   N(p)   = { in[p][a] : a < fan } u { r : (a, r) in rev(p) }           */
+/*   C(p)   = { r in rev(p) } u { x = in[q][b] : q in N(p), b < fan },    */
+/*            x != SENTINEL, x != p, x not in in[p], each x once           */
+/*   out[p] = first k of sort_by_(dist,id)( in[p] u {(F(p,x), x) : x in C} ) */
+/* padded with (SENTINEL, +inf).  Same layouts and return as            */
+/* orc_knn_refine.                                                        */
+/* ------------------------------------------------------------------ */
+typedef struct {
+    int32_t a;
+    uint32_t r;
+} orc_rv;
+static int rv_cmp(const void *x, const void *y)
+{
+    const orc_rv *u = (const orc_rv *)x, *v = (const orc_rv *)y;
+    if (u->a != v->a) return u->a < v->a ? -1 : 1;
+    if (u->r != v->r) return u->r < v->r ? -1 : 1;
+    return 0;
+}
+
+int32_t orc_knn_refine_rev(const float *X, int64_t n, int32_t d, int32_t metric, int32_t k, int32_t fan,
+                           const uint32_t *ids_in, const float *d_in, uint32_t *ids_out, float *d_out)
+{
+    uint8_t *mark;
+    orc_cand *c;
+    int64_t *cnt, *start, p, r, tot = 0;
+    int64_t *fill;
+    orc_rv *rv;
+    uint32_t *rev;
+    int32_t a, b, i, m, nr;
+    if (n < 1 || k < 1 || fan < 1 || fan > k) return -1;
+    cnt = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+    start = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+    fill = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+    rev = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)n * fan);
+    mark = (uint8_t *)calloc((size_t)((n + 7) / 8), 1);
+    c = (orc_cand *)malloc(sizeof(orc_cand) * (size_t)(k + 2 * fan * fan + fan));
+    if (!cnt || !start || !fill || !rev || !mark || !c) {
+        free(cnt); free(start); free(fill); free(rev); free(mark); free(c);
+        return -1;
+    }
+    /* reverse pairs (a, r) of every point, then the first fan by (a, r) */
+    for (r = 0; r < n; r++)
+        for (a = 0; a < fan; a++) {
+            uint32_t q = ids_in[r * k + a];
+            if (q != ORC_SENTINEL && (int64_t)q != r) cnt[q]++;
+        }
+    for (p = 0; p < n; p++) { start[p] = tot; tot += cnt[p]; }
+    rv = (orc_rv *)malloc(sizeof(orc_rv) * (size_t)(tot > 0 ? tot : 1));
+    if (!rv) { free(cnt); free(start); free(fill); free(rev); free(mark); free(c); return -1; }
+    for (r = 0; r < n; r++)
+        for (a = 0; a < fan; a++) {
+            uint32_t q = ids_in[r * k + a];
+            if (q == ORC_SENTINEL || (int64_t)q == r) continue;
+            rv[start[q] + fill[q]].a = a;
+            rv[start[q] + fill[q]].r = (uint32_t)r;
+            fill[q]++;
+        }
+    for (p = 0; p < n; p++) {
+        qsort(rv + start[p], (size_t)cnt[p], sizeof(orc_rv), rv_cmp);
+        for (i = 0; i < fan; i++) rev[p * fan + i] = i < cnt[p] ? rv[start[p] + i].r : ORC_SENTINEL;
+    }
+    for (p = 0; p < n; p++) {
+        m = 0;
+        bm_set(mark, (uint32_t)p);
+        for (i = 0; i < k; i++) {             /* the current list */
+            uint32_t x = ids_in[p * k + i];
+            if (x == ORC_SENTINEL) continue;
+            bm_set(mark, x);
+            c[m].dist = d_in[p * k + i];
+            c[m].id = x;
+            c[m].checked = 0;
+            m++;
+        }
+        for (i = 0; i < fan; i++) {           /* the reverse neighbours themselves */
+            uint32_t x = rev[p * fan + i];
+            if (x == ORC_SENTINEL || bm_test(mark, x)) continue;
+            bm_set(mark, x);
+            c[m].dist = orc_distance(X + p * (int64_t)d, X + (int64_t)x * d, d, metric);
+            c[m].id = x;
+            c[m].checked = 0;
+            m++;
+        }
+        for (nr = 0; nr < 2 * fan; nr++) {    /* lists of the forward, then the reverse neighbours */
+            uint32_t q = nr < fan ? ids_in[p * k + nr] : rev[p * fan + (nr - fan)];
+            if (q == ORC_SENTINEL) continue;
+            for (b = 0; b < fan; b++) {
+                uint32_t x = ids_in[(int64_t)q * k + b];
+                if (x == ORC_SENTINEL || bm_test(mark, x)) continue;
+                bm_set(mark, x);
+                c[m].dist = orc_distance(X + p * (int64_t)d, X + (int64_t)x * d, d, metric);
+                c[m].id = x;
+                c[m].checked = 0;
+                m++;
+            }
+        }
+        qsort(c, (size_t)m, sizeof(orc_cand), cand_cmp);
+        for (i = 0; i < k; i++) {
+            ids_out[p * k + i] = i < m ? c[i].id : ORC_SENTINEL;
+            d_out[p * k + i] = i < m ? c[i].dist : __builtin_inff();
+        }
+        mark[p >> 3] = 0;
+        for (i = 0; i < m; i++) mark[c[i].id >> 3] = 0;
+    }
+    free(cnt); free(start); free(fill); free(rev); free(mark); free(c); free(rv);
     return 0;
 }

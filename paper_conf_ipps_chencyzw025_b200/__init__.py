@@ -429,8 +429,11 @@ def build_graph_partitioned(data, degree: int, n_clusters: int, overlap: int = 2
     return out
 
 
-def knn_refine(data, ids, dists, fan: int, rounds: int = 1, metric: int = L2):
-    """algas_knn_refine: neighbour-of-neighbour refinement rounds (R33); returns new (ids, dists)."""
+def knn_refine(data, ids, dists, fan: int, rounds: int = 1, metric: int = L2, reverse: bool = False):
+    """algas_knn_refine: neighbour-of-neighbour refinement rounds (R33; reverse=True: R35 with
+    reverse neighbours, passed as a negative fan); returns new (ids, dists)."""
+    if reverse:
+        fan = -abs(int(fan))
     n, dim = int(data.shape[0]), int(data.shape[1])
     ids = ids.clone() if _is_torch(ids) else np.array(ids, np.uint32, copy=True)
     dists = dists.clone() if _is_torch(dists) else np.array(dists, np.float32, copy=True)

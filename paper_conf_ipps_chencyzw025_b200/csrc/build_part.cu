@@ -209,11 +209,13 @@ __global__ void __launch_bounds__(128) merge_lists_kernel(const uint64_t* __rest
 template <int METRIC>
 __global__ void __launch_bounds__(128) refine_kernel(const float4* __restrict__ X, int d4, int64_t n, int k, int fan,
                                                      int hb, int per_warp, const uint32_t* __restrict__ in_ids,
-                                                     const float* __restrict__ in_d, uint32_t* __restrict__ out_ids,
-                                                     float* __restrict__ out_d) {
+                                                     const float* __restrict__ in_d, const uint32_t* __restrict__ rev,
+                                                     uint32_t* __restrict__ out_ids, float* __restrict__ out_d) {
   extern __shared__ __align__(16) uint8_t sm[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int hcap = 1 << hb, ncand = fan * fan;
+  // R33: fan x fan candidate slots; R35 (rev != nullptr): fan reverse
+  // neighbours, then the lists of the fan forward and the fan reverse ones
+  const int hcap = 1 << hb, ncand = rev ? fan + 2 * fan * fan : fan * fan;
   uint8_t* base = sm + (size_t)warp * per_warp;  // 16-B multiple
   uint64_t* L = reinterpret_cast<uint64_t*>(base);
   uint64_t* tmp = L + k;
@@ -237,8 +239,16 @@ __global__ void __launch_bounds__(128) refine_kernel(const float4* __restrict__ 
     const int t = t0 + lane;
     uint32_t x = kSentinel;
     if (t < ncand) {
-      const uint32_t q = in_ids[p * k + t / fan];
-      if (q != kSentinel) x = in_ids[(int64_t)q * k + t % fan];
+      if (rev == nullptr) {
+        const uint32_t q = in_ids[p * k + t / fan];
+        if (q != kSentinel) x = in_ids[(int64_t)q * k + t % fan];
+      } else if (t < fan) {
+        x = rev[p * fan + t];  // a reverse neighbour itself
+      } else {
+        const int u = t - fan, nr = u / fan;
+        const uint32_t q = nr < fan ? in_ids[p * k + nr] : rev[p * fan + (nr - fan)];
+        if (q != kSentinel) x = in_ids[(int64_t)q * k + u % fan];
+      }
     }
     const bool keep = x != kSentinel && smem_visit(hash, hb, x) == kVisNew;
     const unsigned msk = __ballot_sync(0xffffffffu, keep);
@@ -331,20 +341,21 @@ int launch_merge_lists(const uint64_t* lists, const uint32_t* slot_of, int64_t n
 }
 
 int launch_refine(const float* X, int d, int metric, int64_t n, int k, int fan, const uint32_t* in_ids,
-                  const float* in_d, uint32_t* out_ids, float* out_d) {
+                  const float* in_d, const uint32_t* rev, uint32_t* out_ids, float* out_d) {
+  const int ncand = rev ? fan + 2 * fan * fan : fan * fan;
   int hb = 6;
-  while ((1 << hb) < 2 * (k + fan * fan + 1)) ++hb;
-  const size_t per_warp = ((size_t)16 * k + ((size_t)4 << hb) + (size_t)4 * fan * fan + 15) & ~(size_t)15;
+  while ((1 << hb) < 2 * (k + ncand + 1)) ++hb;
+  const size_t per_warp = ((size_t)16 * k + ((size_t)4 << hb) + (size_t)4 * ncand + 15) & ~(size_t)15;
   const size_t smem = 4 * per_warp;
   void* fn = metric == kL2 ? (void*)refine_kernel<kL2> : (void*)refine_kernel<kIP>;
   ALGAS_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const unsigned g = (unsigned)((n + 3) / 4);
   if (metric == kL2)
     refine_kernel<kL2><<<g, 128, smem>>>(reinterpret_cast<const float4*>(X), d / 4, n, k, fan, hb, (int)per_warp,
-                                         in_ids, in_d, out_ids, out_d);
+                                         in_ids, in_d, rev, out_ids, out_d);
   else
     refine_kernel<kIP><<<g, 128, smem>>>(reinterpret_cast<const float4*>(X), d / 4, n, k, fan, hb, (int)per_warp,
-                                         in_ids, in_d, out_ids, out_d);
+                                         in_ids, in_d, rev, out_ids, out_d);
   ALGAS_CUDA_TRY(cudaGetLastError());
   ALGAS_CUDA_TRY(cudaDeviceSynchronize());
   return ALGAS_OK;

@@ -246,7 +246,7 @@ int launch_cluster_knn(const float* X, int d, int metric, const uint32_t* mem, c
 int launch_merge_lists(const uint64_t* lists, const uint32_t* slot_of, int64_t n, int c, int k, uint32_t* out_ids,
                        float* out_d);
 int launch_refine(const float* X, int d, int metric, int64_t n, int k, int fan, const uint32_t* in_ids,
-                  const float* in_d, uint32_t* out_ids, float* out_d);
+                  const float* in_d, const uint32_t* rev, uint32_t* out_ids, float* out_d);
 constexpr int kPartMaxKnn = 128;  // list length the batched cluster kNN keeps in shared memory
 
 // graph build's contraction on the tensor cores (knn_tc.cu): D (qb x nb, row

@@ -1008,10 +1008,77 @@ int algas_knn_partitioned(const float* data, int64_t n, int32_t dim, int32_t met
   return ALGAS_OK;
 }
 
-int algas_knn_refine(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t k, int32_t fan,
+// Reverse neighbour lists of one R35 round (device, from the round's input
+// lists in[n][k]): rev[p][j], j < fan = the first fan pairs (a, r) in (a, r)
+// order with in[r][a] == p, a < fan, r != p (SENTINEL-padded) -- counts,
+// offsets, a scatter of (a << 32 | r) keys, a segmented sort per point.
+__global__ void rev_count_kernel(const uint32_t* in, int64_t n, int k, int fan, uint32_t* cnt) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n * fan) return;
+  const int64_t r = i / fan;
+  const uint32_t p = in[r * k + i % fan];
+  if (p != kSentinel && (int64_t)p != r) atomicAdd(cnt + p, 1u);
+}
+__global__ void rev_scatter_kernel(const uint32_t* in, int64_t n, int k, int fan, const uint64_t* off,
+                                   uint32_t* fill, unsigned long long* keys) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n * fan) return;
+  const int64_t r = i / fan;
+  const int a = (int)(i % fan);
+  const uint32_t p = in[r * k + a];
+  if (p == kSentinel || (int64_t)p == r) return;
+  keys[off[p] + atomicAdd(fill + p, 1u)] = ((unsigned long long)a << 32) | (unsigned long long)r;
+}
+__global__ void rev_take_kernel(const unsigned long long* sorted, const uint64_t* off, int64_t n, int fan,
+                                uint32_t* rev) {
+  const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= n) return;
+  const uint64_t o = off[p], m = off[p + 1] - o;
+  for (int j = 0; j < fan; ++j) rev[p * fan + j] = (uint64_t)j < m ? (uint32_t)sorted[o + j] : kSentinel;
+}
+int build_rev_lists(const uint32_t* in, int64_t n, int k, int fan, uint32_t* rev) {
+  Dev hcnt, hoff, hfill, hk1, hk2, htmp;
+  const int64_t E = n * fan;
+  ALGAS_CUDA_TRY(cudaMalloc(&hcnt.p, (size_t)n * 4));
+  ALGAS_CUDA_TRY(cudaMemset(hcnt.p, 0, (size_t)n * 4));
+  const unsigned g = (unsigned)((E + 255) / 256);
+  rev_count_kernel<<<g, 256>>>(in, n, k, fan, (uint32_t*)hcnt.p);
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  std::vector<uint32_t> cnt(n);
+  ALGAS_CUDA_TRY(cudaMemcpy(cnt.data(), hcnt.p, (size_t)n * 4, cudaMemcpyDeviceToHost));
+  std::vector<uint64_t> off(n + 1);
+  uint64_t acc = 0;
+  for (int64_t i = 0; i < n; ++i) { off[i] = acc; acc += cnt[i]; }
+  off[n] = acc;
+  ALGAS_CUDA_TRY(cudaMalloc(&hoff.p, (size_t)(n + 1) * 8));
+  ALGAS_CUDA_TRY(cudaMemcpy(hoff.p, off.data(), (size_t)(n + 1) * 8, cudaMemcpyHostToDevice));
+  ALGAS_CUDA_TRY(cudaMalloc(&hfill.p, (size_t)n * 4));
+  ALGAS_CUDA_TRY(cudaMemset(hfill.p, 0, (size_t)n * 4));
+  ALGAS_CUDA_TRY(cudaMalloc(&hk1.p, std::max<size_t>((size_t)acc * 8, 16)));
+  ALGAS_CUDA_TRY(cudaMalloc(&hk2.p, std::max<size_t>((size_t)acc * 8, 16)));
+  rev_scatter_kernel<<<g, 256>>>(in, n, k, fan, (const uint64_t*)hoff.p, (uint32_t*)hfill.p,
+                                 (unsigned long long*)hk1.p);
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  const uint64_t* offp = (const uint64_t*)hoff.p;
+  size_t tmp = 0;
+  ALGAS_CUDA_TRY(cub::DeviceSegmentedSort::SortKeys(nullptr, tmp, (const unsigned long long*)hk1.p,
+                                                    (unsigned long long*)hk2.p, (int)acc, (int)n, offp, offp + 1));
+  ALGAS_CUDA_TRY(cudaMalloc(&htmp.p, std::max<size_t>(tmp, 16)));
+  ALGAS_CUDA_TRY(cub::DeviceSegmentedSort::SortKeys(htmp.p, tmp, (const unsigned long long*)hk1.p,
+                                                    (unsigned long long*)hk2.p, (int)acc, (int)n, offp, offp + 1));
+  rev_take_kernel<<<(unsigned)((n + 255) / 256), 256>>>((const unsigned long long*)hk2.p, offp, n, fan, rev);
+  ALGAS_CUDA_TRY(cudaGetLastError());
+  ALGAS_CUDA_TRY(cudaDeviceSynchronize());
+  return ALGAS_OK;
+}
+
+int algas_knn_refine(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t k, int32_t fan_arg,
                      int32_t rounds, uint32_t* ids, float* dists) {
+  const bool reverse = fan_arg < 0;  // R35: reverse neighbours joined too
+  const int fan = reverse ? -fan_arg : fan_arg;
   if (!data || !ids || !dists || n < 1 || n >= (1LL << 31) || dim < 4 || dim % 4 != 0 || k < 1 || k > 1024 ||
-      fan < 1 || fan > k || fan > 64 || rounds < 0 || (metric != ALGAS_L2 && metric != ALGAS_IP && metric != ALGAS_COSINE))
+      fan < 1 || fan > k || fan > (reverse ? 32 : 64) || rounds < 0 ||
+      (metric != ALGAS_L2 && metric != ALGAS_IP && metric != ALGAS_COSINE))
     return set_error(ALGAS_EINVAL, "algas_knn_refine: bad arguments");
   if (rounds == 0) return ALGAS_OK;
   Dev hx, hxn, a_i, a_d, b_i, b_d;
@@ -1034,9 +1101,12 @@ int algas_knn_refine(const float* data, int64_t n, int32_t dim, int32_t metric, 
   ALGAS_CUDA_TRY(cudaMalloc(&b_d.p, bytes));
   ALGAS_CUDA_TRY(cudaMemcpy(a_i.p, ids, bytes, cudaMemcpyDefault));
   ALGAS_CUDA_TRY(cudaMemcpy(a_d.p, dists, bytes, cudaMemcpyDefault));
-  for (int r = 0; r < rounds; ++r) {  // Jacobi rounds (R33)
-    if ((rc = launch_refine(X, dim, met, n, k, fan, (const uint32_t*)a_i.p, (const float*)a_d.p, (uint32_t*)b_i.p,
-                            (float*)b_d.p)))
+  Dev hrev;
+  if (reverse) ALGAS_CUDA_TRY(cudaMalloc(&hrev.p, (size_t)n * fan * 4));
+  for (int r = 0; r < rounds; ++r) {  // Jacobi rounds (R33 / R35)
+    if (reverse && (rc = build_rev_lists((const uint32_t*)a_i.p, n, k, fan, (uint32_t*)hrev.p))) return rc;
+    if ((rc = launch_refine(X, dim, met, n, k, fan, (const uint32_t*)a_i.p, (const float*)a_d.p,
+                            reverse ? (const uint32_t*)hrev.p : nullptr, (uint32_t*)b_i.p, (float*)b_d.p)))
       return rc;
     std::swap(a_i.p, b_i.p);
     std::swap(a_d.p, b_d.p);
@@ -1058,10 +1128,14 @@ int algas_build_graph_partitioned(const float* data, int64_t n, int32_t dim, int
   int rc = algas_knn_partitioned(data, n, dim, metric, K, n_clusters, overlap, (uint32_t*)guard_k.p,
                                  (float*)guard_d.p);
   if (rc) return rc;
-  if (refine_rounds > 0 &&
-      (rc = algas_knn_refine(data, n, dim, metric, K, std::min(std::max(refine_fan, 1), std::min(K, 64)),
-                             refine_rounds, (uint32_t*)guard_k.p, (float*)guard_d.p)))
-    return rc;
+  if (refine_rounds > 0) {
+    // refine_fan < 0: R35 rounds (reverse neighbours joined too), fan |refine_fan|
+    const bool rv = refine_fan < 0;
+    const int f = std::min(std::max(rv ? -refine_fan : refine_fan, 1), std::min(K, rv ? 32 : 64));
+    if ((rc = algas_knn_refine(data, n, dim, metric, K, rv ? -f : f, refine_rounds, (uint32_t*)guard_k.p,
+                               (float*)guard_d.p)))
+      return rc;
+  }
   // rows the partition left short (clusters of <= K points) are completed by
   // the exact kNN of those rows over the whole set (the prune needs full rows)
   std::vector<uint32_t> hk((size_t)n * K);

@@ -27,6 +27,7 @@ def main():
     ap.add_argument("--overlap", type=int, nargs="+", default=[2])
     ap.add_argument("--refine", type=int, nargs="+", default=[0, 1], help="refinement rounds (DESIGN.md R33)")
     ap.add_argument("--fan", type=int, default=16)
+    ap.add_argument("--reverse", action="store_true", help="R35 rounds (reverse neighbours joined)")
     ap.add_argument("--no-exact", action="store_true")
     ap.add_argument("--search-L", type=int, nargs="*", default=[],
                     help="also search each partitioned graph at these L (T=4, 1024 threads, SHARED, w=12/16)")
@@ -66,7 +67,8 @@ def main():
             for rounds in a.refine:
                 torch.cuda.synchronize()
                 t0 = time.time()
-                ri, _ = algas.knn_refine(Xd, ids, dd, fan=a.fan, rounds=rounds, metric=w.metric) if rounds else (ids, dd)
+                ri, _ = (algas.knn_refine(Xd, ids, dd, fan=a.fan, rounds=rounds, metric=w.metric, reverse=a.reverse)
+                          if rounds else (ids, dd))
                 torch.cuda.synchronize()
                 t_ref = time.time() - t0
                 rih = ri.cpu().numpy().view(np.uint32)
@@ -74,7 +76,7 @@ def main():
                                for j, i in enumerate(sample)])
                 t0 = time.time()
                 gp = algas.build_graph_partitioned(Xd, w.degree, m, c, knn_degree=w.knn_degree, metric=w.metric,
-                                                   refine_fan=a.fan, refine_rounds=rounds)
+                                                   refine_fan=-a.fan if a.reverse else a.fan, refine_rounds=rounds)
                 torch.cuda.synchronize()
                 t_build = time.time() - t0
                 rp = algas.Index(Xd, gp, w.metric).search(Q, params=p)
@@ -89,6 +91,7 @@ def main():
                     curve.append([L, float((rr["ids"][:, :w.k, None] == ti[:, None, :w.k]).any(2).mean()),
                                   round(a.nq / (rr["info"].kernel_ms / 1e3))])
                 out["partitioned"].append({"clusters": m, "overlap": c, "refine_rounds": rounds, "fan": a.fan,
+                                           "reverse": a.reverse,
                                            "knn_s": t_knn, "refine_s": t_ref, "build_s": t_build,
                                            "knn_graph_recall_sample": float(hit), "search_recall": rec,
                                            "search_T4_L_recall_qps": curve})

@@ -645,3 +645,35 @@ def test_knn_refine_monotone_and_improves_partitioned_lists():
         np.testing.assert_allclose(rd[i, :len(real)], ref, rtol=1e-5)
         assert i not in real.tolist() and len(set(real.tolist())) == len(real)
     assert oracle.recall(ri, ei, 10) > oracle.recall(pi, ei, 10) + 0.05
+
+
+def test_knn_refine_reverse_hand_example():
+    """R35 on the same lines: in[p] = [p+1, p+3], fan = 2.  p's reverse pairs
+    are (0, p-1) (in[p-1] = [p, p+2]) and (1, p-3) (in[p-3] = [p-2, p]), so
+    rev(p) = [p-1, p-3]: p-1 (at 1) becomes a candidate, which the forward-
+    only round never reaches, and for 3 <= p <= 5 the first two are p-1, p+1
+    (dist 1 each, id order).  p = 1: rev(1) = [0], first two 0, 2."""
+    X, ids, ds = _line_lists(12)
+    o, d = oracle.knn_refine(X, ids, ds, fan=2, rounds=1, reverse=True)
+    for p in range(3, 6):
+        assert o[p].tolist() == [p - 1, p + 1] and d[p].tolist() == [1.0, 1.0], (p, o[p], d[p])
+    assert o[1].tolist() == [0, 2] and d[1].tolist() == [1.0, 1.0]
+    f, _ = oracle.knn_refine(X, ids, ds, fan=2, rounds=1, reverse=False)
+    assert all(p - 1 not in f[p].tolist() for p in range(1, 6))
+
+
+@pytest.mark.parametrize("metric", [oracle.L2, oracle.IP])
+def test_knn_refine_reverse_fixed_point_and_superset(metric):
+    """An exact list is a fixed point of R35 too; and R35's candidate set
+    contains R33's, so every row's sorted distances are elementwise <= the
+    forward-only round's (first k of a superset)."""
+    X = synth.lattice(400, 16, seed=61, metric=metric)
+    ei, ed = oracle.knn_graph(X, 12, metric)
+    ri, rd = oracle.knn_refine(X, ei, ed, fan=4, rounds=1, metric=metric, reverse=True)
+    np.testing.assert_array_equal(ri, ei)
+    np.testing.assert_array_equal(rd, ed)
+    pi, pd = oracle.knn_partitioned(X, 12, 8, 2, metric)
+    fi, fd = oracle.knn_refine(X, pi, pd, fan=6, rounds=1, metric=metric)
+    bi, bd = oracle.knn_refine(X, pi, pd, fan=6, rounds=1, metric=metric, reverse=True)
+    assert np.all(bd <= fd)
+    assert oracle.recall(bi, ei, 12) >= oracle.recall(fi, ei, 12)

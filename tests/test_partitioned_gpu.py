@@ -111,3 +111,26 @@ def test_knn_refine_raises_recall_float():
         ref = ((X[real].astype(np.float64) - X[i]) ** 2).sum(1)
         np.testing.assert_allclose(rd[i, :len(real)], ref, rtol=1e-5)
         assert np.all(np.diff(rd[i, :len(real)]) >= 0)
+
+
+# ------------------------------------------------------------------ reverse-neighbour rounds (R35)
+@pytest.mark.parametrize("metric", [algas.L2, algas.IP])
+@pytest.mark.parametrize("fan,rounds", [(4, 1), (8, 2)])
+def test_knn_refine_reverse_lattice_bit_exact(metric, fan, rounds):
+    """algas_knn_refine with reverse neighbours == oracle.knn_refine(reverse)
+    bit for bit on lattice data, from the (oracle's) partitioned lists."""
+    X = synth.lattice(900, 32, seed=47, metric=metric)
+    pi, pd = oracle.knn_partitioned(X, 16, 9, 2, metric)
+    gi, gd = algas.knn_refine(X, pi, pd, fan=fan, rounds=rounds, metric=metric, reverse=True)
+    oi, od = oracle.knn_refine(X, pi, pd, fan=fan, rounds=rounds, metric=metric, reverse=True)
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(_bits(gd), _bits(od))
+
+
+def test_knn_refine_reverse_hand_example_gpu():
+    """The oracle's R35 hand example: p-1 is reached through the reverse list."""
+    from test_oracle import _line_lists
+    X, ids, ds = _line_lists(12)
+    gi, gd = algas.knn_refine(X, ids, ds, fan=2, rounds=1, reverse=True)
+    for p in range(3, 6):
+        assert gi[p].tolist() == [p - 1, p + 1] and gd[p].tolist() == [1.0, 1.0]
