@@ -152,6 +152,9 @@ def dist_init():
     return rank, world, local
 
 
+REFINE_OVERRIDE = None  # (fan, rounds) for partitioned builds (--refine; fan < 0: R35 reverse rounds)
+
+
 def build_workload(w, nq, dev, ncal=10000):
     """Synthetic data + graph + ground truth on this rank's GPU (setup, untimed).
     Returns the measured query set (Q, truth) and an independent calibration
@@ -172,8 +175,10 @@ def build_workload(w, nq, dev, ncal=10000):
     t_gen = time.time() - t0
     if w.build == "partitioned":  # DESIGN.md R30 / R33: shards too large for the exact O(n^2) build
         m = w.part_clusters or max(1, w.n // 4096)
+        rf = REFINE_OVERRIDE[0] if REFINE_OVERRIDE else w.refine_fan
+        rr = REFINE_OVERRIDE[1] if REFINE_OVERRIDE else w.refine_rounds
         G = algas.build_graph_partitioned(Xd, w.degree, m, w.part_overlap, knn_degree=w.knn_degree, metric=w.metric,
-                                          refine_fan=w.refine_fan, refine_rounds=w.refine_rounds)
+                                          refine_fan=rf, refine_rounds=rr)
     else:
         knn, _ = algas.knn(Xd, Xd, w.knn_degree, w.metric, self_base=0)
         G = algas.prune(knn, w.degree) if w.prune else knn[:, :w.degree].contiguous()
@@ -816,8 +821,12 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-ncu", action="store_true", help="no in-run ncu pass for roofline.traffic")
+    ap.add_argument("--refine", default=None, help="partitioned builds: 'fan,rounds' (fan < 0: reverse rounds, R35)")
     ap.add_argument("--ncu-timeout", type=float, default=240.0)
     a = ap.parse_args()
+    if a.refine:
+        global REFINE_OVERRIDE
+        REFINE_OVERRIDE = tuple(int(v) for v in a.refine.split(","))
     if a.warmup < 3:
         a.warmup = 3
     rank, world, local = dist_init()

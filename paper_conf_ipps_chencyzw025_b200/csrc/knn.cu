@@ -295,7 +295,7 @@ static int knn_direct(const float* base, int64_t n, const float* queries, int64_
   if ((rc = to_device(base, (size_t)n * dim * 4, hx, (const void**)&X))) return rc;
   if ((rc = to_device(queries, (size_t)nq * dim * 4, hq, (const void**)&Q))) return rc;
   const int64_t QB = std::min<int64_t>(nq, 4096);
-  const int64_t NB = std::min<int64_t>(n, 65536);
+  const int64_t NB = std::min<int64_t>((n + 3) & ~int64_t(3), 65536);  // row stride of the distance block: a multiple of 4 (16-B rows for the tcgen05 epilogue)
   ALGAS_CUDA_TRY(cudaMalloc(&hstate.p, (size_t)QB * k * 8));
   ALGAS_CUDA_TRY(cudaMalloc(&hD.p, (size_t)QB * NB * 4));
   const bool dev_out = is_device_ptr(out_ids) && is_device_ptr(out_dists);
@@ -476,7 +476,7 @@ static int knn_screened(const float* X, int64_t n, const float* Q, int64_t nq, i
   const int margin = std::max(32, k / 2);
   const int K2 = (int)std::min<int64_t>(k + margin, 256);
   const int64_t QB = std::min<int64_t>(nq, 4096);
-  const int64_t NB = std::min<int64_t>(n, 65536);
+  const int64_t NB = std::min<int64_t>((n + 3) & ~int64_t(3), 65536);  // row stride of the distance block: a multiple of 4 (16-B rows for the tcgen05 epilogue)
   Dev hxh, hxl, hqh, hql, hxn, hqn, hmax, hstate, hD, hid, hd, hfail, hrows, hself, hqf, hfid, hfd;
   ALGAS_CUDA_TRY(cudaMalloc(&hxh.p, (size_t)n * d * 4));
   ALGAS_CUDA_TRY(cudaMalloc(&hxl.p, (size_t)n * d * 4));

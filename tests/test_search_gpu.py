@@ -174,6 +174,20 @@ def test_knn_tcgen05_screen_certifies_and_matches_cublas(knn_mode, monkeypatch, 
     np.testing.assert_array_equal(_bits(td), _bits(dd))
 
 
+@pytest.mark.parametrize("n", [3051, 1001, 70_003])
+def test_knn_screened_base_not_a_multiple_of_four(knn_mode, n):
+    """Screened path with a base size that is not a multiple of 4 (e.g. the
+    partitioned build's centre assignment: n / 4096 centres): the distance
+    block's row stride is padded for the tcgen05 epilogue; result == O1."""
+    X = synth.lattice(n, 32, seed=29)
+    Q = synth.lattice(300, 32, seed=30)
+    knn_mode("screened")
+    gi, gd = algas.knn(X, Q, 16, algas.L2)
+    oi, od = oracle.brute_force(X, Q, 16, oracle.L2)
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(_bits(gd), _bits(od))
+
+
 def test_knn_screened_lattice_matches_oracle(knn_mode):
     """Integer lattice: the screened path equals O1 bit for bit, including
     (dist, id) tie order (ties defeat the certificate -> direct fallback)."""
