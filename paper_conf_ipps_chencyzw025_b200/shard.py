@@ -83,3 +83,75 @@ class ShardedIndex:
         ds = np.asarray(r["dists"]) if isinstance(r["dists"], np.ndarray) else r["dists"].cpu().numpy()
         gi, gd = gather_and_merge(to_global(ids, self.offset), ds, params.k, group=group, device=device)
         return dict(ids=gi, dists=gd, local=r)
+
+
+class ShardedServer:
+    """Sharded-index SERVING: rank g runs a persistent `Server` (its slot ring,
+    dynamic batching) on its shard of the base set.  Rank 0 holds the query
+    stream; every batch of it is broadcast to all ranks (one collective per
+    batch), each rank streams the batch through its own server's host FIFO
+    (`enqueue`) and collects its per-shard top-k by tag, and the per-shard
+    lists (GLOBAL ids) of each batch are all-gathered and merged on every rank
+    with the host TopK merge & filter of the multi-CTA path.
+
+    All batches are broadcast and enqueued before the first is collected, so
+    the shards' searches of batch i+1 overlap the exchange of batch i.
+    `server`: this rank's Server (or an emulated one in host-logic tests);
+    `offset`: first global id of this rank's shard."""
+
+    def __init__(self, server, offset: int, k: int, group=None, device=None):
+        self.server = server
+        self.offset = int(offset)
+        self.k = int(k)
+        self.group = group
+        self.device = device
+
+    def _bcast(self, t):
+        import torch.distributed as dist
+        src = dist.get_global_rank(self.group, 0) if self.group is not None else 0
+        dist.broadcast(t, src=src, group=self.group)
+        return t
+
+    def serve(self, queries=None, batch: int = 256, tag0: int = 0, timeout_s: float = 60.0):
+        """Collective (every rank calls it).  queries: [nq, d] fp32 on group
+        rank 0 (ignored elsewhere).  Returns merged (ids [nq, k], dists) on
+        every rank."""
+        import time
+
+        import torch
+        import torch.distributed as dist
+        dev = self.device if self.device is not None else torch.device("cpu")
+        me = dist.get_rank(self.group)
+        hdr = torch.zeros(2, dtype=torch.int64, device=dev)
+        if me == 0:
+            hdr[0], hdr[1] = int(queries.shape[0]), int(queries.shape[1])
+        self._bcast(hdr)
+        nq, d = int(hdr[0]), int(hdr[1])
+        spans = [(lo, min(nq, lo + batch)) for lo in range(0, nq, batch)]
+        for lo, hi in spans:  # broadcast + enqueue every batch
+            qb = torch.empty((hi - lo, d), dtype=torch.float32, device=dev)
+            if me == 0:
+                qb.copy_(torch.from_numpy(np.ascontiguousarray(queries[lo:hi], dtype=np.float32)))
+            self._bcast(qb)
+            self.server.enqueue(np.ascontiguousarray(qb.cpu().numpy()), tag0=tag0 + lo)
+        out_i = np.empty((nq, self.k), np.uint32)
+        out_d = np.empty((nq, self.k), np.float32)
+        got_i = np.full((nq, self.k), SENTINEL, np.uint32)
+        got_d = np.full((nq, self.k), np.inf, np.float32)
+        have = np.zeros(nq, bool)
+        t0 = time.time()
+        for lo, hi in spans:  # collect in batch order, exchange + merge each batch
+            while not have[lo:hi].all():
+                if time.time() - t0 > timeout_s:
+                    raise TimeoutError(f"rank {me}: shard results missing after {timeout_s} s")
+                tags, ids, ds, _ = self.server.poll(1024)
+                for t, i, dd in zip(tags, ids, ds):
+                    q = int(t) - tag0
+                    got_i[q], got_d[q] = i[:self.k], dd[:self.k]
+                    have[q] = True
+                if len(tags) == 0:
+                    time.sleep(0.0002)
+            gi, gd = gather_and_merge(to_global(got_i[lo:hi], self.offset), got_d[lo:hi], self.k,
+                                      group=self.group, device=self.device)
+            out_i[lo:hi], out_d[lo:hi] = gi, gd
+        return out_i, out_d

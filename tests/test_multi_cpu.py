@@ -143,3 +143,35 @@ def test_shard_range_partitions():
             assert max(b - a for a, b in rs) - min(b - a for a, b in rs) <= 1
     ids = np.array([0, 5, 0xFFFFFFFF], np.uint32)
     np.testing.assert_array_equal(shard.to_global(ids, 100), [100, 105, 0xFFFFFFFF])
+
+
+def _sharded_server_emulated(rank, world):
+    """Each rank serves its 'shard' with an emulated ring device (host logic
+    only); rank 0 alone holds the query stream."""
+    import paper_conf_ipps_chencyzw025_b200 as algas
+    from paper_conf_ipps_chencyzw025_b200 import shard
+    Q = synth.uniform(300, 8, seed=90).astype(np.float32)
+    Q[:, 0] = np.round(Q[:, 0] * 100)  # exact small-integer q[0] (the emulated dists)
+    offset = rank * 10_000_000
+    p = algas.default_params(k=6, itopk=16, width=4, ctas_per_query=2, slots=4)
+    with algas.Server(None, p, emulated_dim=8) as srv:
+        ss = shard.ShardedServer(srv, offset, 6)
+        gi, gd = ss.serve(Q if rank == 0 else None, batch=64, tag0=5)
+    return dict(ids=gi, dists=gd, Q=Q)
+
+
+def test_sharded_server_broadcast_enqueue_gather_merge():
+    """ShardedServer: rank 0's stream is broadcast, every rank's server
+    answers every query, and the merged lists equal the (dist, id)-sorted
+    union of the ranks' per-shard lists with global ids -- on every rank."""
+    res = _run(_sharded_server_emulated)
+    Q = res[0]["Q"]
+    for q in range(Q.shape[0]):
+        tag = 5 + q
+        union = [(Q[q, 0] + j, tag * 1000 + j + r * 10_000_000) for r in range(2) for j in range(6)]
+        union.sort()
+        exp_i = np.array([u[1] for u in union[:6]], np.uint32)
+        exp_d = np.array([u[0] for u in union[:6]], np.float32)
+        for r in range(2):
+            np.testing.assert_array_equal(res[r]["ids"][q], exp_i)
+            np.testing.assert_array_equal(res[r]["dists"][q], exp_d)

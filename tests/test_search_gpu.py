@@ -509,6 +509,40 @@ def test_sharded_index_nccl_world1_equals_index():
     np.testing.assert_array_equal(r["dists"], b["dists"])
 
 
+def test_sharded_server_nccl_world1_equals_server():
+    """ShardedServer (broadcast -> per-shard persistent server -> NCCL
+    all-gather -> merge) with world_size 1 returns the persistent server's own
+    answers, which equal the batch search (the oracle trajectory)."""
+    import os
+    import socket
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_chencyzw025_b200 import shard
+    X, Q, G = lattice_case(2000, 32, algas.L2, 16, seed=331)
+    Q = np.ascontiguousarray(np.concatenate([Q] * 5))  # 5 batches of the stream
+    p = algas.default_params(k=10, itopk=32, width=2, offset_beam=8, n_seeds=8, ctas_per_query=2,
+                             threads_per_cta=128, seed=2, slots=8)
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ["MASTER_PORT"] = str(port)
+    idx = algas.Index(X, G)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        with algas.Server(idx, p) as srv:
+            gi, gd = shard.ShardedServer(srv, 0, 10, device=torch.device("cuda", 0)).serve(Q, batch=len(Q) // 5,
+                                                                                            tag0=100)
+    finally:
+        dist.destroy_process_group()
+    b = idx.search(Q, params=p, tag0=100)
+    np.testing.assert_array_equal(gi, b["ids"])
+    np.testing.assert_array_equal(gd, b["dists"])
+
+
 # ------------------------------------------------------------------ SHARED visited mode (P:L211)
 def _shared(p):
     p.visited_mode = algas.VISITED_SHARED if hasattr(algas, "VISITED_SHARED") else 1
