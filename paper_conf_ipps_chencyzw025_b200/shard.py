@@ -97,7 +97,11 @@ class ShardedServer:
     All batches are broadcast and enqueued before the first is collected, so
     the shards' searches of batch i+1 overlap the exchange of batch i.
     `server`: this rank's Server (or an emulated one in host-logic tests);
-    `offset`: first global id of this rank's shard."""
+    `offset`: first global id of this rank's shard.  The exchange launches
+    small torch / NCCL kernels; with CUDA's lazy module loading the first
+    launch of a kernel can wait for the device to go idle, which a running
+    persistent kernel never does: create the server deferred, call
+    `warmup()`, then start it."""
 
     def __init__(self, server, offset: int, k: int, group=None, device=None):
         self.server = server
@@ -105,6 +109,24 @@ class ShardedServer:
         self.k = int(k)
         self.group = group
         self.device = device
+
+    def warmup(self, dim: int, batch: int) -> None:
+        """Collective.  Runs every device operation of `serve` once (header
+        and batch broadcasts, the all-gather + merge) on dummy data, so their
+        kernels are loaded before the persistent kernel starts."""
+        import torch
+        dev = self.device if self.device is not None else torch.device("cpu")
+        hdr = torch.zeros(2, dtype=torch.int64, device=dev)
+        hdr[0] = 1
+        self._bcast(hdr)
+        qb = torch.empty((batch, dim), dtype=torch.float32, device=dev)
+        qb.copy_(torch.zeros((batch, dim), dtype=torch.float32))
+        self._bcast(qb)
+        _ = int(hdr[0]), qb.cpu()
+        gather_and_merge(np.full((batch, self.k), SENTINEL, np.uint32), np.full((batch, self.k), np.inf, np.float32),
+                         self.k, group=self.group, device=self.device)
+        if dev.type == "cuda":
+            torch.cuda.synchronize(dev)
 
     def _bcast(self, t):
         import torch.distributed as dist

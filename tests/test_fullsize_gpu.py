@@ -33,8 +33,9 @@ SENT = algas.SENTINEL
 N_STREAM = 2000
 # sampled queries the oracle checks one by one: the whole 2000-query stream
 # at the C2 headline point (paired SE of the recall difference ~0.001, so the
-# north-star 0.005 bound is meaningful), fewer at C4 (k = 100) / C3 (960-d)
-N_SAMPLE = {"C2": 2000, "C4": 150, "C3": 120}
+# north-star 0.005 bound is meaningful), fewer at C4 (k = 100) / C3 (960-d):
+# 300 / 480 queries (the SHARED bound below is ~3 sigma of the seed spread)
+N_SAMPLE = {"C2": 2000, "C4": 300, "C3": 480}
 _cache = {}
 
 
@@ -182,7 +183,7 @@ def _search_case(name, n_sample, itopk, width, T, threads, shared):
     if shared:
         # SHARED: which CTA claims a point first is timing-dependent
         # on the GPU; the oracle's step-by-step round robin is one admissible
-        # interleaving (R25).  Bound (C3 / C4 samples of 120 / 150
+        # interleaving (R25).  Bound (C3 / C4 samples of 480 / 300
         # queries): within 0.015 of it (~3 sigma of the seed-to-seed spread at
         # this sample size); always: never below PRIVATE mode (the oracle's,
         # same parameters): sharing must not lose.

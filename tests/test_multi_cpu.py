@@ -154,8 +154,10 @@ def _sharded_server_emulated(rank, world):
     Q[:, 0] = np.round(Q[:, 0] * 100)  # exact small-integer q[0] (the emulated dists)
     offset = rank * 10_000_000
     p = algas.default_params(k=6, itopk=16, width=4, ctas_per_query=2, slots=4)
-    with algas.Server(None, p, emulated_dim=8) as srv:
+    with algas.Server(None, p, emulated_dim=8, deferred=True) as srv:
         ss = shard.ShardedServer(srv, offset, 6)
+        ss.warmup(8, 64)
+        srv.start()
         gi, gd = ss.serve(Q if rank == 0 else None, batch=64, tag0=5)
     return dict(ids=gi, dists=gd, Q=Q)
 

@@ -533,9 +533,14 @@ def test_sharded_server_nccl_world1_equals_server():
     idx = algas.Index(X, G)
     dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
     try:
-        with algas.Server(idx, p) as srv:
-            gi, gd = shard.ShardedServer(srv, 0, 10, device=torch.device("cuda", 0)).serve(Q, batch=len(Q) // 5,
-                                                                                            tag0=100)
+        # deferred server: the exchange's kernels are loaded (warmup) before
+        # the persistent kernel starts (CUDA lazy loading waits for an idle
+        # device, which a running persistent kernel never gives)
+        with algas.Server(idx, p, deferred=True) as srv:
+            ss = shard.ShardedServer(srv, 0, 10, device=torch.device("cuda", 0))
+            ss.warmup(Q.shape[1], len(Q) // 5)
+            srv.start()
+            gi, gd = ss.serve(Q, batch=len(Q) // 5, tag0=100)
     finally:
         dist.destroy_process_group()
     b = idx.search(Q, params=p, tag0=100)
