@@ -44,7 +44,7 @@ def _peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             mp = json.load(f)
-        return float(mp["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs"
+        return float(mp["hbm_gbs"]), "MEASURED_PEAKS.json"
     except Exception:
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
@@ -372,7 +372,7 @@ def cpu_baseline(W, w, p, gpu_ids, budget_s=8.0):
     _, st1 = _oracle_parallel(X, G, Q[:npar], op1, w.metric, 0, cores)
     lat_us = s["lats"] * 1e6
     return {"value": round(s["n"] / s["el"], 1), "unit": "queries/s", "cores": 1, "kind": "oracle",
-            "sample": f"O2 T=1 L={L_cpu} w={op.w}, {s['n']} q 1-by-1, core {cores[0]}, {s['el']:.0f}s",
+            "sample": f"O2 T=1 L={L_cpu} w={op.w}, {s['n']} q, core {cores[0]}, {s['el']:.0f}s",
             "p50_us": round(float(np.percentile(lat_us, 50)), 1), "p99_us": round(float(np.percentile(lat_us, 99)), 1),
             "recall": round(recall_at(s["ids"], truth[:s["n"]], w.k), 4),
             "all_cores": {"value": round(qps_all, 1), "cores": len(cores)},
@@ -415,7 +415,7 @@ def ncu_traffic(a, p, W):
             with open(os.path.join(ROOT, "gpurun_out", "ncu_traffic.log"), "w") as f:
                 f.write(" ".join(cmd[:12]) + "\n--- stdout\n" + r.stdout[-20000:] + "\n--- stderr\n" + r.stderr[-20000:])
             return None, f"ncu rc={r.returncode}: no dram counters (gpurun_out/ncu_traffic.log)"
-        return tot, "ncu dram rd+wr, 1 launch, this run"
+        return tot, "ncu, this run"
     except Exception as e:  # noqa: BLE001 -- the bench line must still print
         return None, f"ncu failed: {type(e).__name__}"
     finally:
@@ -590,7 +590,7 @@ def run_algas(a, rank, world, local):
                    "itopk": p.itopk, "width": p.width, "offset_beam": p.offset_beam,
                    "ctas_per_query": p.ctas_per_query, "threads_per_cta": p.threads_per_cta,
                    "visited": "shared" if p.visited_mode else "private",
-                   "recall": round(float(np.mean(recs)), 4), "op_from": "calibration set",
+                   "recall": round(float(np.mean(recs)), 4), "op_from": "calibration",
                    "target_met": target_met, "graph": w.build,
                    "parallelism": f"replicas x{world}", "l2": "256MB flush/step"},
         "latency_us": {"p50": round(float(np.percentile(lat, 50)), 1), "p99": round(float(np.percentile(lat, 99)), 1),
@@ -697,7 +697,7 @@ def run_e2e(a, idx, p, Q, truth, w, world, dev, detail):
             "h2d_bytes_per_step": int(a.nq * (w.dim * 4 + 32)),
             "d2h_bytes_per_step": int(a.nq * (p.ctas_per_query * (w.k * 8 + 32) + 4)),
             "recall": round(rec, 4), "p50_us": lat_b[0], "p99_us": lat_b[1],
-            "batch": per_b, "state_mirror": a.state_mirror, "def": "enqueue->poll; closed loop [p50,p99,qps]"}
+            "batch": per_b, "state_mirror": a.state_mirror, "def": "batch: closed loop [p50,p99,qps]"}
 
 
 def tuner_point(idx, W, w, slots, p_best, stream):
